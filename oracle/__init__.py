@@ -1,0 +1,157 @@
+"""CPU oracle for SpecInfer's token-tree verification hot path — TEST INFRASTRUCTURE ONLY.
+
+Plain fp64 C (``specinfer_oracle.c``) behind ctypes, operating on numpy host arrays.
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py`` (its ``cpu_baseline`` leg and
+``--impl reference``) may import this package.  The product path
+(``paper_conf_asplos_miaoozcwzwzyssc24_b200``) never imports it; the two share no code.
+
+Each wrapper cites the PAPER.md passage its C function follows (see the C file header).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "specinfer_oracle.c")
+_LIB = os.path.join(_HERE, "liboracle.so")
+
+_lib = None
+
+
+def build(force: bool = False) -> str:
+    """Compile the oracle with gcc (-O2 -fopenmp, fp64, no fast-math)."""
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        tmp = _LIB + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", "-O2", "-fopenmp", "-fPIC", "-shared", "-std=c11",
+                               "-Wall", "-o", tmp, _SRC, "-lm"])
+        os.replace(tmp, _LIB)
+    return _LIB
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        _lib = ctypes.CDLL(build())
+        i32, i64, u64, dbl, vp = (ctypes.c_int32, ctypes.c_int64, ctypes.c_uint64,
+                                  ctypes.c_double, ctypes.c_void_p)
+        _lib.oracle_validate_tree.argtypes = [i32, i32, i32, vp, vp, i32, i32]
+        _lib.oracle_validate_tree.restype = ctypes.c_int
+        _lib.oracle_tree_attention.argtypes = [i32, i32, i32, i32, i32, i32, i32, dbl,
+                                               vp, vp, vp, vp, vp, vp, vp, vp]
+        _lib.oracle_kv_commit.argtypes = [i32, i32, i32, i32, i32, i64, i32, vp, vp, vp, vp, vp]
+        _lib.oracle_verify_greedy.argtypes = [i32, i32, i32, i32, i32, i32, vp, vp, vp, vp, vp,
+                                              vp, vp, vp, vp]
+        _lib.oracle_verify_mss.argtypes = [i32, i32, i32, i32, i32, i32, vp, vp, vp, vp, vp, vp,
+                                           vp, dbl, u64, u64, vp, vp, vp, vp, vp]
+        _lib.oracle_philox4x32_10.argtypes = [vp, vp, vp]
+    return _lib
+
+
+def _p(a):
+    return None if a is None else a.ctypes.data_as(ctypes.c_void_p)
+
+
+def _c(a, dtype):
+    return np.ascontiguousarray(a, dtype=dtype)
+
+
+def bf16_bits(x) -> np.ndarray:
+    """View a bf16 array (numpy uint16 bits or torch bf16 tensor on CPU) as uint16 bits."""
+    if hasattr(x, "view") and hasattr(x, "dtype") and str(x.dtype) == "torch.bfloat16":
+        import torch
+        return x.contiguous().view(torch.int16).numpy().view(np.uint16)
+    return _c(x, np.uint16)
+
+
+def validate_tree(parent, depth, prefix_len, n_nodes, nmax, max_depth, smax) -> int:
+    parent = _c(parent, np.int32)
+    depth = None if depth is None else _c(depth, np.int32)
+    return lib().oracle_validate_tree(nmax, max_depth, smax, _p(parent), _p(depth),
+                                      int(prefix_len), int(n_nodes))
+
+
+def tree_attention(q, k, v, parent, depth, prefix_len, n_nodes, *, max_depth=255,
+                   sm_scale=None, out=None) -> np.ndarray:
+    """c1 (Def. 4.1).  q [B][Nmax][Hq][D], k/v [B][Hkv][Smax][D] as bf16
+    bits (uint16); returns fp64 out [B][Nmax][Hq][D] (rows i >= n_nodes[b] are NaN)."""
+    q, k, v = bf16_bits(q), bf16_bits(k), bf16_bits(v)
+    B, Nmax, Hq, D = q.shape
+    _, Hkv, Smax, _ = k.shape
+    assert k.shape == v.shape and k.shape[0] == B and k.shape[3] == D and Hq % Hkv == 0
+    if sm_scale is None:
+        sm_scale = 1.0 / np.sqrt(D)
+    parent = _c(parent, np.int32).reshape(B, Nmax)
+    depth = None if depth is None else _c(depth, np.int32).reshape(B, Nmax)
+    prefix_len, n_nodes = _c(prefix_len, np.int32), _c(n_nodes, np.int32)
+    if out is None:
+        out = np.full((B, Nmax, Hq, D), np.nan, dtype=np.float64)
+    lib().oracle_tree_attention(B, Nmax, Hq, Hkv, D, Smax, max_depth, float(sm_scale), _p(q),
+                                _p(k), _p(v), _p(parent), _p(depth), _p(prefix_len),
+                                _p(n_nodes), _p(out))
+    return out
+
+
+def kv_commit(k_all, v_all, prefix_len, accepted_nodes, n_accepted):
+    """c2 (L635-644).  k_all/v_all [L][B][Hkv][Smax][D] uint16, modified in place, as is
+    prefix_len (int32 [B])."""
+    assert k_all.dtype == np.uint16 and k_all.flags.c_contiguous and v_all.flags.c_contiguous
+    L, B, Hkv, Smax, D = k_all.shape
+    accepted_nodes = _c(accepted_nodes, np.int32)
+    n_accepted = _c(n_accepted, np.int32)
+    assert prefix_len.dtype == np.int32 and prefix_len.flags.c_contiguous
+    lib().oracle_kv_commit(L, B, Hkv, Smax, D, B * Hkv * Smax * D, accepted_nodes.shape[1],
+                           _p(k_all), _p(v_all), _p(prefix_len), _p(accepted_nodes),
+                           _p(n_accepted))
+
+
+def verify_greedy(logits, tree_tokens, parent, n_nodes, *, depth=None, prefix_len=None,
+                  smax=1 << 30, max_depth=255, path_len=None):
+    """c3 (Alg. 2).  Returns (accepted_nodes, accepted_tokens, n_accepted)."""
+    logits = _c(logits, np.float32)
+    B, Nmax, V = logits.shape
+    path_len = path_len or (max_depth + 1 if max_depth < 255 else Nmax + 1)
+    an = np.empty((B, path_len), np.int32)
+    at = np.empty((B, path_len), np.int32)
+    na = np.empty((B,), np.int32)
+    lib().oracle_verify_greedy(B, Nmax, V, smax, max_depth, path_len, _p(logits),
+                               _p(_c(tree_tokens, np.int32)), _p(_c(parent, np.int32)),
+                               _p(None if depth is None else _c(depth, np.int32)),
+                               _p(None if prefix_len is None else _c(prefix_len, np.int32)),
+                               _p(_c(n_nodes, np.int32)), _p(an), _p(at), _p(na))
+    return an, at, na
+
+
+def verify_mss(logits, tree_tokens, parent, n_nodes, draft_probs, *, temperature=1.0, seed=0,
+               offset=0, request_ids=None, depth=None, prefix_len=None, smax=1 << 30,
+               max_depth=255, path_len=None):
+    """c4 (Alg. 2).  Returns (accepted_nodes, accepted_tokens, n_accepted, margin)."""
+    logits = _c(logits, np.float32)
+    draft_probs = _c(draft_probs, np.float32)
+    B, Nmax, V = logits.shape
+    assert draft_probs.shape == logits.shape
+    path_len = path_len or (max_depth + 1 if max_depth < 255 else Nmax + 1)
+    an = np.empty((B, path_len), np.int32)
+    at = np.empty((B, path_len), np.int32)
+    na = np.empty((B,), np.int32)
+    mg = np.empty((B,), np.float64)
+    rids = None if request_ids is None else _c(request_ids, np.int32)
+    lib().oracle_verify_mss(B, Nmax, V, smax, max_depth, path_len, _p(logits),
+                            _p(_c(tree_tokens, np.int32)), _p(_c(parent, np.int32)),
+                            _p(None if depth is None else _c(depth, np.int32)),
+                            _p(None if prefix_len is None else _c(prefix_len, np.int32)),
+                            _p(_c(n_nodes, np.int32)), _p(draft_probs), float(temperature),
+                            int(seed) & (2**64 - 1), int(offset) & (2**64 - 1), _p(rids),
+                            _p(an), _p(at), _p(na), _p(mg))
+    return an, at, na, mg
+
+
+def philox4x32_10(ctr, key) -> np.ndarray:
+    c = _c(ctr, np.uint32)
+    k = _c(key, np.uint32)
+    o = np.empty(4, np.uint32)
+    lib().oracle_philox4x32_10(_p(c), _p(k), _p(o))
+    return o
