@@ -1,0 +1,163 @@
+/*
+ * specinfer.h — C ABI of libspecinfer.so: the data-parallel hot path of SpecInfer's token-tree
+ * verification (SpecInfer, ASPLOS'24), hand-written CUDA for B200 (sm_100a).
+ *
+ * PAPER.md passages the calls implement (line numbers of /root/reference/PAPER.md):
+ *   specinfer_tree_prepare    Def. 3.1 L450-454 (token tree, S_u); L657-674 (topology-aware mask)
+ *   specinfer_tree_attention  Alg. 2 line 6 TreeParallelDecode L385; Def. 4.1;
+ *                             Eq. 1-4; footnote L627-628; L645-674 (one fused kernel)
+ *   specinfer_verify_greedy   Alg. 2 VerifyGreedy L395-401; §4.3
+ *   specinfer_verify_mss      Alg. 2 VerifyStochastic L403-425; Fig. 5; Thm 4.2
+ *   specinfer_kv_commit       depth-first KV-cache update L635-644; tree-topology KV layout L659-661
+ * Readings of the paper where it is silent or garbled are numbered R1..R23 in DESIGN.md.
+ *
+ * General conventions
+ *   - Every data pointer is a DEVICE pointer unless stated otherwise; the caller owns every
+ *     buffer (allocation, lifetime, freeing).  The library never allocates device memory and
+ *     keeps no global mutable state except a per-device capability cache.
+ *   - Every call is asynchronous and stream-ordered on `stream` (a cudaStream_t; NULL = the
+ *     legacy default stream).  Calls are CUDA-graph capturable.
+ *   - Host-checkable errors (NULL pointer, unsupported shape, non-sm_100 device) are returned
+ *     synchronously before any launch: SPECINFER_ERR_INVALID_ARG / SPECINFER_ERR_UNSUPPORTED.
+ *     Launch failures return SPECINFER_ERR_CUDA (from cudaGetLastError).
+ *   - Tree defects are only visible on the device; kernels record them in a sticky status word
+ *     inside the workspace, skip the offending request (no attention output, n_accepted = 0)
+ *     and continue.  Read it with specinfer_read_device_status (the CUDA async-error model).
+ *   - Nothing throws across the ABI.
+ *
+ * Shapes and layouts (row-major, innermost last; B = batch, Nmax = max_nodes, Hq/Hkv = q/kv
+ * heads, D = head_dim = 128, Smax = max_seq, L = num_layers, V = vocab, Dmax = max_depth):
+ *   parent, depth, tree_tokens   int32 [B][Nmax]  node 0 is the root (parent -1, depth 0);
+ *                                 nodes in topological order: 0 <= parent[i] < i (R5)
+ *   prefix_len                   int32 [B]  committed KV length P_b, excluding the root (R18)
+ *   n_nodes                      int32 [B]  1 <= n_b <= Nmax; rows i >= n_b are padding
+ *   q, out                       bf16  [B][Nmax][Hq][D]
+ *   k_cache, v_cache (one layer) bf16  [B][Hkv][Smax][D]; committed keys at slots [0, P_b),
+ *                                 tree node i's key at slot P_b + i ("tree topology", L659-661)
+ *   logits, draft_probs          fp32  [B][Nmax][V]
+ *   accepted_nodes/tokens        int32 [B][Dmax+1]; n_accepted int32 [B]
+ */
+#ifndef SPECINFER_H_
+#define SPECINFER_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct CUstream_st *specinfer_stream_t; /* == cudaStream_t */
+
+typedef enum {
+    SPECINFER_OK = 0,
+    SPECINFER_ERR_INVALID_ARG = 1, /* NULL pointer or inconsistent shape */
+    SPECINFER_ERR_UNSUPPORTED = 2, /* head_dim != 128, Nmax > 256, Hq % Hkv != 0, G > 64, device not sm_100 */
+    SPECINFER_ERR_CUDA = 3,        /* a CUDA launch/runtime call failed */
+    SPECINFER_ERR_BAD_TREE = 4,    /* (device status) at least one request's tree was invalid */
+    SPECINFER_ERR_WORKSPACE = 5    /* workspace NULL or misaligned (needs 256-byte alignment) */
+} specinfer_status_t;
+
+typedef struct {
+    int32_t batch;        /* B */
+    int32_t max_nodes;    /* Nmax, 1..256 */
+    int32_t num_q_heads;  /* Hq */
+    int32_t num_kv_heads; /* Hkv; Hq % Hkv == 0, G = Hq/Hkv <= 64 */
+    int32_t head_dim;     /* D, must be 128 */
+    int32_t max_seq;      /* Smax; every request needs P_b + n_b <= Smax */
+    int32_t num_layers;   /* L (kv_commit only) */
+    int32_t vocab;        /* V (verify only) */
+    int32_t max_depth;    /* Dmax; every node needs depth <= Dmax; path buffers hold Dmax+1 */
+    float sm_scale;       /* 0 => 1/sqrt(head_dim) (R1: A = QK^T / sqrt(d)) */
+    int64_t layer_stride; /* elements between consecutive layers' caches (kv_commit);
+                             0 => B*Hkv*Smax*D (caches laid out [L][B][Hkv][Smax][D]) */
+} specinfer_shape_t;
+
+/* Bytes of device workspace the calls below need for `shape` (host call, no CUDA work other
+ * than a device-attribute query).  One workspace holds one stream's state: it must not be
+ * shared by calls in flight on different streams. */
+size_t specinfer_workspace_size(const specinfer_shape_t *shape);
+
+/* a0 (K1).  Validates every request's tree (parent/depth/n_nodes/prefix_len against Smax and
+ * Dmax), builds the ancestor-or-self and descendant bitsets of the topology-aware mask
+ * (L657-674) and the tree-attention work schedule, resets the status word and counters.
+ * Must be called once per iteration (per tree) before the other calls that take `workspace`;
+ * its results stay valid for every layer of that iteration.
+ * workspace: device, >= specinfer_workspace_size bytes, 256-byte aligned. */
+specinfer_status_t specinfer_tree_prepare(const specinfer_shape_t *shape, const int32_t *parent,
+                                          const int32_t *depth, const int32_t *prefix_len,
+                                          const int32_t *n_nodes, void *workspace,
+                                          specinfer_stream_t stream);
+
+/* a1-a3 (K2).  Tree attention for ONE layer (Def. 4.1): for each request b, q-head h
+ * (kv-head g = h / (Hq/Hkv)) and node i < n_b,
+ *   out[b][i][h] = sum_j softmax_j(sm_scale q.k_j) v_j  over key slots j in
+ *                  [0, P_b) U { P_b + a : a ancestor-or-self of i }          (R2, L657-674)
+ * computed in fp32 from bf16 inputs (tcgen05 tensor cores, TMA-staged K/V tiles shared by all
+ * G*n_b query rows of a kv-head), rounded to bf16.  Masked keys get exactly zero weight.
+ * Cache slots >= P_b + n_b are never used (may hold anything, NaN included).
+ * parent/depth are accepted for the record of the call (the mask comes from `workspace`,
+ * which tree_prepare built from the same arrays).  Rows i >= n_b, and all rows of an invalid
+ * request, are left untouched.  k_cache/v_cache must be 16-byte aligned. */
+specinfer_status_t specinfer_tree_attention(const specinfer_shape_t *shape, const void *q,
+                                            const void *k_cache, const void *v_cache,
+                                            const int32_t *parent, const int32_t *depth,
+                                            const int32_t *prefix_len, const int32_t *n_nodes,
+                                            void *out, void *workspace, specinfer_stream_t stream);
+
+/* a4 (K4).  VerifyGreedy (Alg. 2): O(u) = lowest token id attaining max logits[u];
+ * from the root, repeatedly move to the lowest-index child whose token equals O(u) (R7);
+ * finally emit O(u).  Writes accepted_nodes[b] = [0, v1..vL], accepted_tokens[b] =
+ * [t_v1..t_vL, O(vL)], n_accepted[b] = L + 1; unused entries -1.  Invalid trees: n_accepted 0.
+ * Needs the workspace of tree_prepare for the same tree. */
+specinfer_status_t specinfer_verify_greedy(const specinfer_shape_t *shape, const float *logits,
+                                           const int32_t *tree_tokens, const int32_t *parent,
+                                           const int32_t *n_nodes, int32_t *accepted_nodes,
+                                           int32_t *accepted_tokens, int32_t *n_accepted,
+                                           void *workspace, specinfer_stream_t stream);
+
+/* a5 (K5).  VerifyStochastic / multi-step speculative sampling (Alg. 2) with the RNG
+ * contract of DESIGN.md R9/R15 (Philox4x32-10, key = seed, counters from the global request
+ * id request_ids[b] (NULL => b), the node, the rejection round and `offset` (low 32 bits)):
+ * p = softmax(logits[u]/temperature); children tried in Philox-uniform order; accept child s
+ * with token x iff p[x] > 0 and r*q_s[x] <= p[x] (q_s = draft_probs[s], the distribution s was
+ * drawn from, R12); on reject p <- norm(max(0, p - q_s)) (kept if all zero, R11); after the
+ * last rejection (or at a leaf) sample x_next ~ p by an exponential race.  Outputs as for
+ * verify_greedy.  temperature > 0.  Needs the workspace of tree_prepare for the same tree. */
+specinfer_status_t specinfer_verify_mss(const specinfer_shape_t *shape, const float *logits,
+                                        const int32_t *tree_tokens, const int32_t *parent,
+                                        const int32_t *n_nodes, const float *draft_probs,
+                                        float temperature, uint64_t seed, uint64_t offset,
+                                        const int32_t *request_ids, int32_t *accepted_nodes,
+                                        int32_t *accepted_tokens, int32_t *n_accepted,
+                                        void *workspace, specinfer_stream_t stream);
+
+/* a6 (K6).  Depth-first KV-cache commit (L635-644): for every layer l < L, request b with
+ * n = n_accepted[b] > 0 and kv-head g: slot P_b + j <- old slot P_b + accepted_nodes[b][j]
+ * for j < n (bit copy of K and V rows), then prefix_len[b] += n (device, in/out).
+ * k_cache_all/v_cache_all: [L] caches `layer_stride` elements apart. */
+specinfer_status_t specinfer_kv_commit(const specinfer_shape_t *shape, void *k_cache_all,
+                                       void *v_cache_all, int32_t *prefix_len,
+                                       const int32_t *accepted_nodes, const int32_t *n_accepted,
+                                       specinfer_stream_t stream);
+
+/* Synchronises `stream` and returns SPECINFER_OK or SPECINFER_ERR_BAD_TREE from the sticky
+ * device status word; *bad_request_mask_out (host, may be NULL) receives the status bits. */
+specinfer_status_t specinfer_read_device_status(const void *workspace, specinfer_stream_t stream,
+                                                int32_t *status_bits_out);
+
+/* Debug/KAT entry: out[i][0..4) = Philox4x32-10(ctr = ctr_key[i][0..4), key = ctr_key[i][4..6))
+ * computed by the device implementation used in verify_mss.  ctr_key/out are device pointers. */
+specinfer_status_t specinfer_philox_debug(const uint32_t *ctr_key, uint32_t *out, int32_t n,
+                                          specinfer_stream_t stream);
+
+/* Number of kernel launches each call issues (for launch accounting in benchmarks). */
+int32_t specinfer_launches_per_call(const char *call_name);
+
+const char *specinfer_status_string(specinfer_status_t status);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* SPECINFER_H_ */

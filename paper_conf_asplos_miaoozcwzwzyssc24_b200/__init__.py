@@ -1,0 +1,263 @@
+"""Thin Python binding of libspecinfer.so (include/specinfer.h) — argument marshalling only.
+
+SpecInfer's token-tree verification hot path on B200 (sm_100a): tree attention with the
+topology-aware causal mask, greedy and multi-step-speculative-sampling verification, and the
+depth-first KV-cache commit.  Every step runs in the hand-written CUDA kernels of the library;
+PyTorch only provides device memory and streams.  There is no CPU fallback: if the library is
+missing or the device is not sm_100, calls raise.
+
+Function names are the C ABI names.  Tensors must be CUDA, contiguous, of the documented dtype
+and shape; violations raise ValueError before anything is launched.
+"""
+from __future__ import annotations
+
+import ctypes
+import dataclasses
+import os
+from typing import Optional
+
+import torch
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libspecinfer.so")
+
+SPECINFER_OK = 0
+STATUS_NAMES = {0: "OK", 1: "ERR_INVALID_ARG", 2: "ERR_UNSUPPORTED", 3: "ERR_CUDA", 4: "ERR_BAD_TREE",
+                5: "ERR_WORKSPACE"}
+
+EXPORTED_SYMBOLS = (
+    "specinfer_workspace_size", "specinfer_tree_prepare", "specinfer_tree_attention",
+    "specinfer_verify_greedy", "specinfer_verify_mss", "specinfer_kv_commit",
+    "specinfer_read_device_status", "specinfer_philox_debug", "specinfer_launches_per_call",
+    "specinfer_status_string",
+)
+
+
+class SpecInferError(RuntimeError):
+    def __init__(self, call: str, status: int, msg: str):
+        super().__init__(f"{call} failed: {STATUS_NAMES.get(status, status)} ({msg})")
+        self.status = status
+
+
+class Shape(ctypes.Structure):
+    _fields_ = [("batch", ctypes.c_int32), ("max_nodes", ctypes.c_int32), ("num_q_heads", ctypes.c_int32),
+                ("num_kv_heads", ctypes.c_int32), ("head_dim", ctypes.c_int32), ("max_seq", ctypes.c_int32),
+                ("num_layers", ctypes.c_int32), ("vocab", ctypes.c_int32), ("max_depth", ctypes.c_int32),
+                ("sm_scale", ctypes.c_float), ("layer_stride", ctypes.c_int64)]
+
+    def __repr__(self):
+        return "Shape(" + ", ".join(f"{n}={getattr(self, n)}" for n, _ in self._fields_) + ")"
+
+
+def make_shape(batch, max_nodes, num_q_heads, num_kv_heads, max_seq, *, num_layers=1, vocab=0,
+               max_depth=None, sm_scale=0.0, layer_stride=0, head_dim=128) -> Shape:
+    return Shape(batch, max_nodes, num_q_heads, num_kv_heads, head_dim, max_seq, num_layers, vocab,
+                 max_nodes - 1 if max_depth is None else max_depth, float(sm_scale), layer_stride)
+
+
+_lib = None
+
+
+def load_library(path: str = LIB_PATH):
+    """Loads libspecinfer.so (built by build_lib.py / __graft_entry__.build()).  Raises if absent."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(path):
+        raise ImportError(f"{path} not found: build it with `python -m "
+                          f"paper_conf_asplos_miaoozcwzwzyssc24_b200.build_lib` (no CPU fallback exists)")
+    lib = ctypes.CDLL(path)
+    vp, i32, u64, f32 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_uint64, ctypes.c_float
+    sp = ctypes.POINTER(Shape)
+    lib.specinfer_workspace_size.argtypes = [sp]
+    lib.specinfer_workspace_size.restype = ctypes.c_size_t
+    lib.specinfer_tree_prepare.argtypes = [sp, vp, vp, vp, vp, vp, vp]
+    lib.specinfer_tree_attention.argtypes = [sp, vp, vp, vp, vp, vp, vp, vp, vp, vp, vp]
+    lib.specinfer_verify_greedy.argtypes = [sp, vp, vp, vp, vp, vp, vp, vp, vp, vp]
+    lib.specinfer_verify_mss.argtypes = [sp, vp, vp, vp, vp, vp, f32, u64, u64, vp, vp, vp, vp, vp, vp]
+    lib.specinfer_kv_commit.argtypes = [sp, vp, vp, vp, vp, vp, vp]
+    lib.specinfer_read_device_status.argtypes = [vp, vp, ctypes.POINTER(i32)]
+    lib.specinfer_philox_debug.argtypes = [vp, vp, i32, vp]
+    lib.specinfer_launches_per_call.argtypes = [ctypes.c_char_p]
+    lib.specinfer_launches_per_call.restype = i32
+    lib.specinfer_status_string.argtypes = [i32]
+    lib.specinfer_status_string.restype = ctypes.c_char_p
+    for name in ("specinfer_tree_prepare", "specinfer_tree_attention", "specinfer_verify_greedy",
+                 "specinfer_verify_mss", "specinfer_kv_commit", "specinfer_read_device_status",
+                 "specinfer_philox_debug"):
+        getattr(lib, name).restype = i32
+    _lib = lib
+    return lib
+
+
+def _check(call: str, status: int):
+    if status != SPECINFER_OK:
+        msg = load_library().specinfer_status_string(status).decode()
+        raise SpecInferError(call, status, msg)
+
+
+def _stream(t: torch.Tensor):
+    return ctypes.c_void_p(torch.cuda.current_stream(t.device).cuda_stream)
+
+
+def _req(name, t, dtype, shape=None, device=None):
+    if not isinstance(t, torch.Tensor):
+        raise ValueError(f"{name}: expected a torch.Tensor")
+    if not t.is_cuda:
+        raise ValueError(f"{name}: must be a CUDA tensor (no CPU path)")
+    if t.dtype != dtype:
+        raise ValueError(f"{name}: dtype {t.dtype}, expected {dtype}")
+    if not t.is_contiguous():
+        raise ValueError(f"{name}: must be contiguous")
+    if shape is not None and tuple(t.shape) != tuple(shape):
+        raise ValueError(f"{name}: shape {tuple(t.shape)}, expected {tuple(shape)}")
+    if device is not None and t.device != device:
+        raise ValueError(f"{name}: on {t.device}, expected {device}")
+    return ctypes.c_void_p(t.data_ptr())
+
+
+def _opt(name, t, dtype, shape, device):
+    return None if t is None else _req(name, t, dtype, shape, device)
+
+
+def specinfer_workspace_size(shape: Shape) -> int:
+    return int(load_library().specinfer_workspace_size(ctypes.byref(shape)))
+
+
+def alloc_workspace(shape: Shape, device) -> torch.Tensor:
+    n = specinfer_workspace_size(shape)
+    if n == 0:
+        raise ValueError(f"unsupported shape {shape}")
+    ws = torch.empty(n + 256, dtype=torch.uint8, device=device)
+    off = (-ws.data_ptr()) % 256
+    return ws[off:off + n]
+
+
+def _tree_args(shape: Shape, parent, depth, prefix_len, n_nodes, dev):
+    B, N = shape.batch, shape.max_nodes
+    return (_req("parent", parent, torch.int32, (B, N), dev), _req("depth", depth, torch.int32, (B, N), dev),
+            _req("prefix_len", prefix_len, torch.int32, (B,), dev), _req("n_nodes", n_nodes, torch.int32, (B,), dev))
+
+
+def specinfer_tree_prepare(shape: Shape, parent, depth, prefix_len, n_nodes, workspace: torch.Tensor):
+    dev = parent.device
+    args = _tree_args(shape, parent, depth, prefix_len, n_nodes, dev)
+    ws = _req("workspace", workspace, torch.uint8, None, dev)
+    _check("specinfer_tree_prepare",
+           load_library().specinfer_tree_prepare(ctypes.byref(shape), *args, ws, _stream(parent)))
+
+
+def specinfer_tree_attention(shape: Shape, q, k_cache, v_cache, parent, depth, prefix_len, n_nodes,
+                             out, workspace):
+    dev = q.device
+    B, N, Hq, Hkv, S = shape.batch, shape.max_nodes, shape.num_q_heads, shape.num_kv_heads, shape.max_seq
+    qp = _req("q", q, torch.bfloat16, (B, N, Hq, 128), dev)
+    kp = _req("k_cache", k_cache, torch.bfloat16, (B, Hkv, S, 128), dev)
+    vp = _req("v_cache", v_cache, torch.bfloat16, (B, Hkv, S, 128), dev)
+    op = _req("out", out, torch.bfloat16, (B, N, Hq, 128), dev)
+    args = _tree_args(shape, parent, depth, prefix_len, n_nodes, dev)
+    ws = _req("workspace", workspace, torch.uint8, None, dev)
+    _check("specinfer_tree_attention",
+           load_library().specinfer_tree_attention(ctypes.byref(shape), qp, kp, vp, *args, op, ws, _stream(q)))
+
+
+def specinfer_verify_greedy(shape: Shape, logits, tree_tokens, parent, n_nodes, accepted_nodes,
+                            accepted_tokens, n_accepted, workspace):
+    dev = logits.device
+    B, N, V, Lp = shape.batch, shape.max_nodes, shape.vocab, shape.max_depth + 1
+    args = (_req("logits", logits, torch.float32, (B, N, V), dev),
+            _req("tree_tokens", tree_tokens, torch.int32, (B, N), dev),
+            _req("parent", parent, torch.int32, (B, N), dev), _req("n_nodes", n_nodes, torch.int32, (B,), dev),
+            _req("accepted_nodes", accepted_nodes, torch.int32, (B, Lp), dev),
+            _req("accepted_tokens", accepted_tokens, torch.int32, (B, Lp), dev),
+            _req("n_accepted", n_accepted, torch.int32, (B,), dev),
+            _req("workspace", workspace, torch.uint8, None, dev))
+    _check("specinfer_verify_greedy",
+           load_library().specinfer_verify_greedy(ctypes.byref(shape), *args, _stream(logits)))
+
+
+def specinfer_verify_mss(shape: Shape, logits, tree_tokens, parent, n_nodes, draft_probs, temperature,
+                         seed, offset, request_ids, accepted_nodes, accepted_tokens, n_accepted, workspace):
+    dev = logits.device
+    B, N, V, Lp = shape.batch, shape.max_nodes, shape.vocab, shape.max_depth + 1
+    if not (temperature > 0):
+        raise ValueError("temperature must be > 0")
+    a = (_req("logits", logits, torch.float32, (B, N, V), dev),
+         _req("tree_tokens", tree_tokens, torch.int32, (B, N), dev),
+         _req("parent", parent, torch.int32, (B, N), dev), _req("n_nodes", n_nodes, torch.int32, (B,), dev),
+         _req("draft_probs", draft_probs, torch.float32, (B, N, V), dev))
+    rid = _opt("request_ids", request_ids, torch.int32, (B,), dev)
+    o = (_req("accepted_nodes", accepted_nodes, torch.int32, (B, Lp), dev),
+         _req("accepted_tokens", accepted_tokens, torch.int32, (B, Lp), dev),
+         _req("n_accepted", n_accepted, torch.int32, (B,), dev),
+         _req("workspace", workspace, torch.uint8, None, dev))
+    _check("specinfer_verify_mss",
+           load_library().specinfer_verify_mss(ctypes.byref(shape), *a, ctypes.c_float(temperature),
+                                               ctypes.c_uint64(int(seed) & (2**64 - 1)),
+                                               ctypes.c_uint64(int(offset) & (2**64 - 1)), rid, *o,
+                                               _stream(logits)))
+
+
+def specinfer_kv_commit(shape: Shape, k_cache_all, v_cache_all, prefix_len, accepted_nodes, n_accepted):
+    dev = k_cache_all.device
+    B, Lp = shape.batch, shape.max_depth + 1
+    for nm, t in (("k_cache_all", k_cache_all), ("v_cache_all", v_cache_all)):
+        _req(nm, t, torch.bfloat16, None, dev)
+        stride = shape.layer_stride or B * shape.num_kv_heads * shape.max_seq * 128
+        if t.numel() < (shape.num_layers - 1) * stride + B * shape.num_kv_heads * shape.max_seq * 128:
+            raise ValueError(f"{nm}: too small for {shape.num_layers} layers")
+    _check("specinfer_kv_commit", load_library().specinfer_kv_commit(
+        ctypes.byref(shape), ctypes.c_void_p(k_cache_all.data_ptr()), ctypes.c_void_p(v_cache_all.data_ptr()),
+        _req("prefix_len", prefix_len, torch.int32, (B,), dev),
+        _req("accepted_nodes", accepted_nodes, torch.int32, (B, Lp), dev),
+        _req("n_accepted", n_accepted, torch.int32, (B,), dev), _stream(k_cache_all)))
+
+
+def specinfer_read_device_status(workspace: torch.Tensor) -> int:
+    """Synchronises the current stream; returns the status bits (bit 0 = some tree invalid)."""
+    bits = ctypes.c_int32(0)
+    st = load_library().specinfer_read_device_status(ctypes.c_void_p(workspace.data_ptr()), _stream(workspace),
+                                                    ctypes.byref(bits))
+    if st not in (0, 4):
+        _check("specinfer_read_device_status", st)
+    return int(bits.value)
+
+
+def specinfer_philox_debug(ctr_key: torch.Tensor) -> torch.Tensor:
+    """ctr_key int64/uint32-valued tensor [n][6] -> [n][4] uint32 words as int64 (device Philox)."""
+    dev = ctr_key.device
+    ck = ctr_key.to(torch.int64).bitwise_and(0xFFFFFFFF).to(torch.int32).contiguous()
+    out = torch.empty((ck.shape[0], 4), dtype=torch.int32, device=dev)
+    _check("specinfer_philox_debug", load_library().specinfer_philox_debug(
+        ctypes.c_void_p(ck.data_ptr()), ctypes.c_void_p(out.data_ptr()), ck.shape[0], _stream(ck)))
+    return out.to(torch.int64).bitwise_and(0xFFFFFFFF)
+
+
+def specinfer_launches_per_call(name: str) -> int:
+    return int(load_library().specinfer_launches_per_call(name.encode()))
+
+
+# ------------------------------------------------------------------------------------------
+# convenience: a prepared verification iteration (used by bench.py and the tests)
+# ------------------------------------------------------------------------------------------
+
+@dataclasses.dataclass
+class TreeState:
+    shape: Shape
+    parent: torch.Tensor
+    depth: torch.Tensor
+    prefix_len: torch.Tensor
+    n_nodes: torch.Tensor
+    workspace: torch.Tensor
+
+    @classmethod
+    def create(cls, shape: Shape, parent, depth, prefix_len, n_nodes, workspace=None):
+        ws = workspace if workspace is not None else alloc_workspace(shape, parent.device)
+        return cls(shape, parent, depth, prefix_len, n_nodes, ws)
+
+    def prepare(self):
+        specinfer_tree_prepare(self.shape, self.parent, self.depth, self.prefix_len, self.n_nodes, self.workspace)
+
+    def attention(self, q, k, v, out):
+        specinfer_tree_attention(self.shape, q, k, v, self.parent, self.depth, self.prefix_len, self.n_nodes,
+                                 out, self.workspace)

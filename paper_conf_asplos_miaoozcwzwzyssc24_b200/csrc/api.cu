@@ -1,0 +1,236 @@
+// api.cu — the extern "C" boundary of libspecinfer.so (include/specinfer.h).
+//
+// Host-side argument validation, per-device capability cache (sm_100 check, SM count, max
+// dynamic shared memory), workspace layout, and the launches of the K1..K6 kernels.
+#include <math.h>
+#include <string.h>
+
+#include <mutex>
+
+#include "common.cuh"
+
+namespace specinfer {
+cudaError_t launch_tree_prepare(const specinfer_shape_t &s, const WsLayout &w, const int32_t *parent,
+                                const int32_t *depth, const int32_t *prefix_len, const int32_t *n_nodes,
+                                char *ws, cudaStream_t stream);
+cudaError_t launch_tree_attention(const specinfer_shape_t &s, const WsLayout &w, const void *q, const void *k,
+                                  const void *v, const int32_t *prefix_len, const int32_t *n_nodes, void *out,
+                                  char *ws, int num_sms, size_t max_smem, cudaStream_t stream);
+cudaError_t launch_verify_greedy(const specinfer_shape_t &s, const WsLayout &w, const float *logits,
+                                 const int32_t *tree_tokens, const int32_t *parent, const int32_t *n_nodes,
+                                 int32_t *acc_nodes, int32_t *acc_tokens, int32_t *n_acc, char *ws,
+                                 cudaStream_t stream);
+cudaError_t launch_verify_mss(const specinfer_shape_t &s, const WsLayout &w, const float *logits,
+                              const int32_t *tree_tokens, const int32_t *parent, const int32_t *n_nodes,
+                              const float *draft_probs, float temperature, uint64_t seed, uint64_t offset,
+                              const int32_t *request_ids, int32_t *acc_nodes, int32_t *acc_tokens,
+                              int32_t *n_acc, char *ws, cudaStream_t stream);
+cudaError_t launch_kv_commit(const specinfer_shape_t &s, void *k_all, void *v_all, int32_t *prefix_len,
+                             const int32_t *acc_nodes, const int32_t *n_acc, cudaStream_t stream);
+cudaError_t launch_philox_debug(const uint32_t *ck, uint32_t *out, int n, cudaStream_t stream);
+}  // namespace specinfer
+
+using namespace specinfer;
+
+namespace {
+
+struct DeviceInfo {
+    bool valid = false;
+    bool sm100 = false;
+    int num_sms = 0;
+    size_t max_smem = 0;
+};
+
+DeviceInfo g_dev[64];
+std::mutex g_mu;
+
+bool device_info(DeviceInfo *out) {
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return false;
+    std::lock_guard<std::mutex> lk(g_mu);
+    DeviceInfo &d = g_dev[dev];
+    if (!d.valid) {
+        int major = 0, minor = 0, sms = 0, smem = 0;
+        if (cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev) != cudaSuccess) return false;
+        cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        cudaDeviceGetAttribute(&smem, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+        d.sm100 = (major == 10 && minor == 0);
+        d.num_sms = sms;
+        d.max_smem = (size_t)smem;
+        d.valid = true;
+    }
+    *out = d;
+    return true;
+}
+
+specinfer_status_t check_shape(const specinfer_shape_t *s) {
+    if (!s) return SPECINFER_ERR_INVALID_ARG;
+    if (s->batch < 1 || s->max_nodes < 1 || s->num_q_heads < 1 || s->num_kv_heads < 1 || s->max_seq < 1 ||
+        s->max_depth < 0)
+        return SPECINFER_ERR_INVALID_ARG;
+    if (s->head_dim != kHeadDim) return SPECINFER_ERR_UNSUPPORTED;
+    if (s->max_nodes > kMaxNodes) return SPECINFER_ERR_UNSUPPORTED;
+    if (s->num_q_heads % s->num_kv_heads != 0) return SPECINFER_ERR_UNSUPPORTED;
+    if (s->num_q_heads / s->num_kv_heads > 64) return SPECINFER_ERR_UNSUPPORTED;
+    if ((long long)s->batch * s->num_kv_heads * s->max_seq > (1ll << 31) - 1) return SPECINFER_ERR_UNSUPPORTED;
+    return SPECINFER_OK;
+}
+
+specinfer_status_t check_device(DeviceInfo *d) {
+    if (!device_info(d)) return SPECINFER_ERR_CUDA;
+    if (!d->sm100) return SPECINFER_ERR_UNSUPPORTED;
+    return SPECINFER_OK;
+}
+
+specinfer_status_t check_ws(const void *ws) {
+    if (!ws || (reinterpret_cast<uintptr_t>(ws) & 255u) != 0) return SPECINFER_ERR_WORKSPACE;
+    return SPECINFER_OK;
+}
+
+specinfer_status_t from_cuda(cudaError_t e) { return e == cudaSuccess ? SPECINFER_OK : SPECINFER_ERR_CUDA; }
+
+#define SPI_TRY(x)                                 \
+    do {                                           \
+        specinfer_status_t _s = (x);               \
+        if (_s != SPECINFER_OK) return _s;         \
+    } while (0)
+
+}  // namespace
+
+extern "C" {
+
+size_t specinfer_workspace_size(const specinfer_shape_t *shape) {
+    if (check_shape(shape) != SPECINFER_OK) return 0;
+    DeviceInfo d;
+    const int sms = device_info(&d) ? d.num_sms : 148;
+    return ws_layout(*shape, sms > 0 ? sms : 148).total;
+}
+
+specinfer_status_t specinfer_tree_prepare(const specinfer_shape_t *shape, const int32_t *parent,
+                                          const int32_t *depth, const int32_t *prefix_len, const int32_t *n_nodes,
+                                          void *workspace, specinfer_stream_t stream) {
+    SPI_TRY(check_shape(shape));
+    if (!parent || !depth || !prefix_len || !n_nodes) return SPECINFER_ERR_INVALID_ARG;
+    SPI_TRY(check_ws(workspace));
+    DeviceInfo d;
+    SPI_TRY(check_device(&d));
+    const WsLayout w = ws_layout(*shape, d.num_sms);
+    return from_cuda(launch_tree_prepare(*shape, w, parent, depth, prefix_len, n_nodes,
+                                         reinterpret_cast<char *>(workspace), (cudaStream_t)stream));
+}
+
+specinfer_status_t specinfer_tree_attention(const specinfer_shape_t *shape, const void *q, const void *k_cache,
+                                            const void *v_cache, const int32_t *parent, const int32_t *depth,
+                                            const int32_t *prefix_len, const int32_t *n_nodes, void *out,
+                                            void *workspace, specinfer_stream_t stream) {
+    SPI_TRY(check_shape(shape));
+    if (!q || !k_cache || !v_cache || !parent || !depth || !prefix_len || !n_nodes || !out)
+        return SPECINFER_ERR_INVALID_ARG;
+    if ((reinterpret_cast<uintptr_t>(q) | reinterpret_cast<uintptr_t>(k_cache) |
+         reinterpret_cast<uintptr_t>(v_cache) | reinterpret_cast<uintptr_t>(out)) & 15u)
+        return SPECINFER_ERR_INVALID_ARG;
+    SPI_TRY(check_ws(workspace));
+    DeviceInfo d;
+    SPI_TRY(check_device(&d));
+    const WsLayout w = ws_layout(*shape, d.num_sms);
+    return from_cuda(launch_tree_attention(*shape, w, q, k_cache, v_cache, prefix_len, n_nodes, out,
+                                           reinterpret_cast<char *>(workspace), d.num_sms, d.max_smem,
+                                           (cudaStream_t)stream));
+}
+
+specinfer_status_t specinfer_verify_greedy(const specinfer_shape_t *shape, const float *logits,
+                                           const int32_t *tree_tokens, const int32_t *parent, const int32_t *n_nodes,
+                                           int32_t *accepted_nodes, int32_t *accepted_tokens, int32_t *n_accepted,
+                                           void *workspace, specinfer_stream_t stream) {
+    SPI_TRY(check_shape(shape));
+    if (shape->vocab < 1) return SPECINFER_ERR_INVALID_ARG;
+    if (!logits || !tree_tokens || !parent || !n_nodes || !accepted_nodes || !accepted_tokens || !n_accepted)
+        return SPECINFER_ERR_INVALID_ARG;
+    SPI_TRY(check_ws(workspace));
+    DeviceInfo d;
+    SPI_TRY(check_device(&d));
+    const WsLayout w = ws_layout(*shape, d.num_sms);
+    return from_cuda(launch_verify_greedy(*shape, w, logits, tree_tokens, parent, n_nodes, accepted_nodes,
+                                          accepted_tokens, n_accepted, reinterpret_cast<char *>(workspace),
+                                          (cudaStream_t)stream));
+}
+
+specinfer_status_t specinfer_verify_mss(const specinfer_shape_t *shape, const float *logits,
+                                        const int32_t *tree_tokens, const int32_t *parent, const int32_t *n_nodes,
+                                        const float *draft_probs, float temperature, uint64_t seed, uint64_t offset,
+                                        const int32_t *request_ids, int32_t *accepted_nodes,
+                                        int32_t *accepted_tokens, int32_t *n_accepted, void *workspace,
+                                        specinfer_stream_t stream) {
+    SPI_TRY(check_shape(shape));
+    if (shape->vocab < 1 || !(temperature > 0.f) || !isfinite(temperature)) return SPECINFER_ERR_INVALID_ARG;
+    if (!logits || !tree_tokens || !parent || !n_nodes || !draft_probs || !accepted_nodes || !accepted_tokens ||
+        !n_accepted)
+        return SPECINFER_ERR_INVALID_ARG;
+    SPI_TRY(check_ws(workspace));
+    DeviceInfo d;
+    SPI_TRY(check_device(&d));
+    const WsLayout w = ws_layout(*shape, d.num_sms);
+    return from_cuda(launch_verify_mss(*shape, w, logits, tree_tokens, parent, n_nodes, draft_probs, temperature,
+                                       seed, offset, request_ids, accepted_nodes, accepted_tokens, n_accepted,
+                                       reinterpret_cast<char *>(workspace), (cudaStream_t)stream));
+}
+
+specinfer_status_t specinfer_kv_commit(const specinfer_shape_t *shape, void *k_cache_all, void *v_cache_all,
+                                       int32_t *prefix_len, const int32_t *accepted_nodes, const int32_t *n_accepted,
+                                       specinfer_stream_t stream) {
+    SPI_TRY(check_shape(shape));
+    if (shape->num_layers < 1) return SPECINFER_ERR_INVALID_ARG;
+    if (!k_cache_all || !v_cache_all || !prefix_len || !accepted_nodes || !n_accepted)
+        return SPECINFER_ERR_INVALID_ARG;
+    if ((reinterpret_cast<uintptr_t>(k_cache_all) | reinterpret_cast<uintptr_t>(v_cache_all)) & 15u)
+        return SPECINFER_ERR_INVALID_ARG;
+    DeviceInfo d;
+    SPI_TRY(check_device(&d));
+    return from_cuda(launch_kv_commit(*shape, k_cache_all, v_cache_all, prefix_len, accepted_nodes, n_accepted,
+                                      (cudaStream_t)stream));
+}
+
+specinfer_status_t specinfer_read_device_status(const void *workspace, specinfer_stream_t stream,
+                                                int32_t *status_bits_out) {
+    SPI_TRY(check_ws(workspace));
+    int32_t bits = 0;
+    // the status word sits at offset 0 of every workspace layout
+    cudaError_t e = cudaMemcpyAsync(&bits, workspace, sizeof(bits), cudaMemcpyDeviceToHost, (cudaStream_t)stream);
+    if (e == cudaSuccess) e = cudaStreamSynchronize((cudaStream_t)stream);
+    if (e != cudaSuccess) return SPECINFER_ERR_CUDA;
+    if (status_bits_out) *status_bits_out = bits;
+    return (bits & kStatusBadTree) ? SPECINFER_ERR_BAD_TREE : SPECINFER_OK;
+}
+
+specinfer_status_t specinfer_philox_debug(const uint32_t *ctr_key, uint32_t *out, int32_t n,
+                                          specinfer_stream_t stream) {
+    if (n < 0 || (n > 0 && (!ctr_key || !out))) return SPECINFER_ERR_INVALID_ARG;
+    DeviceInfo d;
+    SPI_TRY(check_device(&d));
+    return from_cuda(launch_philox_debug(ctr_key, out, n, (cudaStream_t)stream));
+}
+
+int32_t specinfer_launches_per_call(const char *name) {
+    if (!name) return -1;
+    if (!strcmp(name, "tree_prepare")) return 2;     // validate+bitsets, schedule (+1 memset)
+    if (!strcmp(name, "tree_attention")) return 1;   // split combine fused (last piece merges)
+    if (!strcmp(name, "verify_greedy")) return 1;    // argmax + walk fused (last CTA walks)
+    if (!strcmp(name, "verify_mss")) return 1;
+    if (!strcmp(name, "kv_commit")) return 2;        // copy, prefix update
+    return -1;
+}
+
+const char *specinfer_status_string(specinfer_status_t s) {
+    switch (s) {
+        case SPECINFER_OK: return "ok";
+        case SPECINFER_ERR_INVALID_ARG: return "invalid argument";
+        case SPECINFER_ERR_UNSUPPORTED: return "unsupported shape or device (needs sm_100, head_dim 128, Nmax <= 256)";
+        case SPECINFER_ERR_CUDA: return "CUDA error";
+        case SPECINFER_ERR_BAD_TREE: return "invalid token tree in at least one request";
+        case SPECINFER_ERR_WORKSPACE: return "workspace NULL or not 256-byte aligned";
+    }
+    return "unknown status";
+}
+
+}  // extern "C"

@@ -1,0 +1,447 @@
+"""GPU parity: the CUDA path (through the C ABI) against the fp64 CPU oracle.
+
+Bars (BASELINE.json north_star): tree attention max|err| <= 1e-2 and mean|err| <= 1e-3 on the
+same bf16-rounded inputs; greedy verification, KV commit and accepted paths bit-exact; MSS
+bit-exact except decisions whose relative margin is < 1e-5 (fp32 vs fp64).
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import workloads as W
+
+pytestmark = pytest.mark.gpu
+
+if torch.cuda.is_available():
+    import paper_conf_asplos_miaoozcwzwzyssc24_b200 as spi
+
+MAX_ABS, MEAN_ABS = 1e-2, 1e-3
+DEV = "cuda:0"
+
+
+def _shape(tb, Hq, Hkv, smax, **kw):
+    return spi.make_shape(tb.parent.shape[0], tb.max_nodes, Hq, Hkv, smax, max_depth=tb.max_depth, **kw)
+
+
+def _gpu_attention(tb, ai, Hq, Hkv, layer=0, sm_scale=0.0):
+    shape = _shape(tb, Hq, Hkv, ai.smax, sm_scale=sm_scale)
+    st = spi.TreeState.create(shape, tb.parent, tb.depth, tb.prefix_len, tb.n_nodes)
+    st.prepare()
+    out = torch.full(ai.q.shape[1:], float("nan"), dtype=torch.bfloat16, device=DEV)
+    st.attention(ai.q[layer], ai.k_cache[layer], ai.v_cache[layer], out)
+    torch.cuda.synchronize()
+    return out, st
+
+
+def _check_rows(got, ref, tb, bs=None, heads=None):
+    n = tb.n_nodes.cpu().numpy()
+    bs = range(got.shape[0]) if bs is None else bs
+    errs = []
+    for b in bs:
+        g = got[b, :n[b]].float().cpu().numpy()
+        r = ref[b, :n[b]]
+        if heads is not None:
+            g, r = g[:, heads], r[:, heads]
+        assert np.all(np.isfinite(g)), f"non-finite output in request {b}"
+        errs.append(np.abs(g - r).reshape(-1))
+    e = np.concatenate(errs)
+    assert e.max() <= MAX_ABS and e.mean() <= MEAN_ABS, (e.max(), e.mean())
+    return e.max(), e.mean()
+
+
+def _oracle_attention(ai, tb, layer=0, bs=None):
+    q, k, v = ai.q[layer].cpu(), ai.k_cache[layer].cpu(), ai.v_cache[layer].cpu()
+    par, dep, pl, nn_ = tb.parent.cpu(), tb.depth.cpu(), tb.prefix_len.cpu(), tb.n_nodes.cpu()
+    if bs is None:
+        return oracle.tree_attention(q, k, v, par, dep, pl, nn_)
+    ref = np.full(q.shape, np.nan)
+    for b in bs:
+        ref[b:b + 1] = oracle.tree_attention(q[b:b + 1], k[b:b + 1], v[b:b + 1], par[b:b + 1], dep[b:b + 1],
+                                             pl[b:b + 1], nn_[b:b + 1])
+    return ref
+
+
+# ---------------------------------------------------------------------------------------------
+# tree attention
+# ---------------------------------------------------------------------------------------------
+
+@pytest.mark.parametrize("Hq,Hkv,Nmax", [(2, 2, 8), (8, 4, 4), (4, 4, 16), (4, 2, 16), (2, 2, 32),
+                                         (8, 1, 8), (4, 4, 64), (8, 2, 20), (3, 3, 100), (16, 2, 40),
+                                         (1, 1, 256)])
+@pytest.mark.parametrize("P", [0, 1, 127, 128, 300])
+def test_attention_random_trees(Hq, Hkv, Nmax, P):
+    """Random trees (ragged n_b), ragged prefixes around tile boundaries, NaN-poisoned unused
+    cache slots; covers NT = 16/32/64 and multi-chunk items."""
+    B = 3
+    rng = np.random.default_rng(1000 * Hq + 10 * Nmax + P)
+    trees = [W.random_tree(int(rng.integers(1, Nmax + 1)), 8, 4, rng) for _ in range(B)]
+    pls = [P, max(P - 1, 0), P + 45]
+    tb = W.make_tree_batch(trees, pls, max_nodes=Nmax, max_depth=8, device=DEV)
+    smax = max(pls) + Nmax + 7
+    ai = W.make_attention_inputs(tb, 1, Hq, Hkv, smax, seed=P + Nmax, device=DEV, poison=True)
+    out, _ = _gpu_attention(tb, ai, Hq, Hkv)
+    ref = _oracle_attention(ai, tb)
+    _check_rows(out, ref, tb)
+    # padded rows are untouched
+    n = tb.n_nodes.cpu().numpy()
+    for b in range(B):
+        assert torch.isnan(out[b, n[b]:].float()).all()
+
+
+@pytest.mark.parametrize("peaky", [False, True])
+def test_attention_chain_and_figures(golden, peaky):
+    """Fig. 4 tree (L682), a 40-node chain (= causal decoding), root-only trees; peaky q (x4)
+    stresses the online-softmax rescaling."""
+    g = golden("fig4_mask.json")
+    fig4 = (np.asarray(g["parent"], np.int32), None)
+    p4 = fig4[0]
+    d4 = np.zeros(len(p4), np.int32)
+    for i in range(1, len(p4)):
+        d4[i] = d4[p4[i]] + 1
+    trees = [(p4, d4), W.chain_tree(40), (np.array([-1], np.int32), np.array([0], np.int32)),
+             W.expansion_tree((2, 2, 1))]
+    tb = W.make_tree_batch(trees, [0, 513, 700, 5], max_nodes=40, max_depth=39, device=DEV)
+    smax = 800
+    ai = W.make_attention_inputs(tb, 1, 8, 8, smax, seed=7, device=DEV, peaky=peaky, poison=True)
+    out, _ = _gpu_attention(tb, ai, 8, 8)
+    _check_rows(out, _oracle_attention(ai, tb), tb)
+
+
+def test_attention_custom_scale_and_empty_prefix():
+    trees = [W.expansion_tree((3, 3))] * 2
+    tb = W.make_tree_batch(trees, [0, 0], device=DEV)
+    ai = W.make_attention_inputs(tb, 1, 4, 4, 20, seed=3, device=DEV, poison=True)
+    out, _ = _gpu_attention(tb, ai, 4, 4, sm_scale=0.2)
+    ref = oracle.tree_attention(ai.q[0].cpu(), ai.k_cache[0].cpu(), ai.v_cache[0].cpu(), tb.parent.cpu(),
+                                tb.depth.cpu(), tb.prefix_len.cpu(), tb.n_nodes.cpu(), sm_scale=0.2)
+    _check_rows(out, ref, tb)
+
+
+def test_attention_invalid_tree_status():
+    """A bad tree sets the sticky device status and leaves its rows untouched; other requests
+    are computed normally."""
+    trees = [W.expansion_tree((2, 2)), W.expansion_tree((2, 2))]
+    tb = W.make_tree_batch(trees, [10, 10], device=DEV)
+    tb.parent[1, 3] = 5   # parent not < i
+    ai = W.make_attention_inputs(tb, 1, 2, 2, 30, seed=4, device=DEV)
+    out, st = _gpu_attention(tb, ai, 2, 2)
+    assert spi.specinfer_read_device_status(st.workspace) & 1
+    assert torch.isnan(out[1].float()).all()
+    ref = _oracle_attention(ai, tb)
+    _check_rows(out, ref, tb, bs=[0])
+
+
+def test_host_validation_errors():
+    tb = W.make_tree_batch([W.chain_tree(4)], [3], device=DEV)
+    ai = W.make_attention_inputs(tb, 1, 2, 2, 16, seed=5, device=DEV)
+    shape = _shape(tb, 2, 2, 16)
+    st = spi.TreeState.create(shape, tb.parent, tb.depth, tb.prefix_len, tb.n_nodes)
+    out = torch.empty(ai.q.shape[1:], dtype=torch.bfloat16, device=DEV)
+    with pytest.raises(ValueError):
+        st.attention(ai.q[0].float(), ai.k_cache[0], ai.v_cache[0], out)
+    with pytest.raises(ValueError):
+        st.attention(ai.q[0], ai.k_cache[0].cpu(), ai.v_cache[0], out)
+    bad = spi.make_shape(1, 4, 2, 2, 16, head_dim=64)
+    with pytest.raises(spi.SpecInferError):
+        spi.specinfer_tree_prepare(bad, tb.parent, tb.depth, tb.prefix_len, tb.n_nodes, st.workspace)
+
+
+def test_attention_cuda_graph_replay():
+    """The calls are stream-ordered and graph-capturable (bench.py replays a CUDA graph)."""
+    cfg = W.CONFIGS["C1"]
+    tb = W.config_tree_batch(cfg, device=DEV)
+    smax = cfg.prefix + tb.max_nodes
+    ai = W.make_attention_inputs(tb, 1, 32, 32, smax, seed=1, device=DEV)
+    shape = _shape(tb, 32, 32, smax)
+    st = spi.TreeState.create(shape, tb.parent, tb.depth, tb.prefix_len, tb.n_nodes)
+    out = torch.zeros(ai.q.shape[1:], dtype=torch.bfloat16, device=DEV)
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        st.prepare()
+        st.attention(ai.q[0], ai.k_cache[0], ai.v_cache[0], out)
+    torch.cuda.synchronize()
+    first = out.clone()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        st.prepare()
+        st.attention(ai.q[0], ai.k_cache[0], ai.v_cache[0], out)
+    out.zero_()
+    for _ in range(3):
+        g.replay()
+    torch.cuda.synchronize()
+    assert torch.equal(out, first)
+
+
+# ---------------------------------------------------------------------------------------------
+# the BASELINE.json configs at full size (attention: one layer per config; each layer is an
+# independent call of the same kernel in the same launch configuration bench.py times)
+# ---------------------------------------------------------------------------------------------
+
+def test_config_c1_full():
+    cfg = W.CONFIGS["C1"]
+    tb = W.config_tree_batch(cfg, device=DEV)
+    smax = cfg.prefix + tb.max_nodes
+    ai = W.make_attention_inputs(tb, 1, cfg.num_q_heads, cfg.num_kv_heads, smax, seed=cfg.seed, device=DEV)
+    out, _ = _gpu_attention(tb, ai, cfg.num_q_heads, cfg.num_kv_heads)
+    _check_rows(out, _oracle_attention(ai, tb), tb)
+
+
+@pytest.mark.parametrize("name,bs,heads", [("C2", [0, 7, 15], None), ("C3", [0, 31], list(range(8, 16))),
+                                           ("C4", [0, 63], [0, 1, 55])])
+def test_config_full_size_sampled(name, bs, heads):
+    """Full batch/prefix/tree of the config (ragged prefixes), one layer; sampled requests and
+    heads against the oracle, every row against an fp32 torch reference on the GPU."""
+    cfg = W.CONFIGS[name]
+    tb = W.config_tree_batch(cfg, device=DEV, ragged=True)
+    smax = cfg.prefix + tb.max_nodes + 3
+    ai = W.make_attention_inputs(tb, 1, cfg.num_q_heads, cfg.num_kv_heads, smax, seed=cfg.seed, device=DEV,
+                                 poison=True)
+    out, _ = _gpu_attention(tb, ai, cfg.num_q_heads, cfg.num_kv_heads)
+    if heads is not None:
+        q = ai.q[0][:, :, heads].contiguous()
+        G = cfg.num_q_heads // cfg.num_kv_heads
+        kvh = sorted({h // G for h in heads})
+        # oracle on the sampled requests with only the needed heads: remap heads to a small GQA problem
+        ref_full = np.full((len(bs), tb.max_nodes, len(heads), 128), np.nan)
+        for bi, b in enumerate(bs):
+            for hi, h in enumerate(heads):
+                g = h // G
+                r = oracle.tree_attention(ai.q[0][b:b + 1, :, h:h + 1].cpu(), ai.k_cache[0][b:b + 1, g:g + 1].cpu(),
+                                          ai.v_cache[0][b:b + 1, g:g + 1].cpu(), tb.parent[b:b + 1].cpu(),
+                                          tb.depth[b:b + 1].cpu(), tb.prefix_len[b:b + 1].cpu(),
+                                          tb.n_nodes[b:b + 1].cpu())
+                ref_full[bi, :, hi] = r[0, :, 0]
+        n = tb.n_nodes.cpu().numpy()
+        for bi, b in enumerate(bs):
+            g = out[b, :n[b], heads].float().cpu().numpy()
+            e = np.abs(g - ref_full[bi, :n[b]])
+            assert e.max() <= MAX_ABS and e.mean() <= MEAN_ABS, (b, e.max(), e.mean())
+    else:
+        ref = _oracle_attention(ai, tb, bs=bs)
+        _check_rows(out, ref, tb, bs=bs)
+    # every row: fp32 torch reference on the GPU (secondary check, not the parity oracle)
+    _torch_reference_check(out, ai, tb, cfg.num_q_heads, cfg.num_kv_heads)
+
+
+def _torch_reference_check(out, ai, tb, Hq, Hkv):
+    B, N = tb.parent.shape
+    G = Hq // Hkv
+    anc = torch.zeros((B, N, N), dtype=torch.bool, device=DEV)
+    par = tb.parent.cpu().numpy()
+    n = tb.n_nodes.cpu().numpy()
+    for b in range(B):
+        for i in range(n[b]):
+            u = i
+            while u >= 0:
+                anc[b, i, u] = True
+                u = par[b, u]
+    pl = tb.prefix_len
+    for b in range(B):
+        P, nb = int(pl[b]), int(n[b])
+        k = ai.k_cache[0, b, :, :P + nb].float()
+        v = ai.v_cache[0, b, :, :P + nb].float()
+        q = ai.q[0, b, :nb].float().permute(1, 0, 2)          # [Hq][nb][D]
+        mask = torch.ones((nb, P + nb), dtype=torch.bool, device=DEV)
+        mask[:, P:] = anc[b, :nb, :nb]
+        ref = torch.nn.functional.scaled_dot_product_attention(
+            q, k.repeat_interleave(G, 0), v.repeat_interleave(G, 0), attn_mask=mask)
+        e = (out[b, :nb].float().permute(1, 0, 2) - ref).abs()
+        assert e.max().item() <= MAX_ABS and e.mean().item() <= MEAN_ABS
+
+
+@pytest.mark.parametrize("n,B,P", [(8, 64, 512), (32, 8, 2048), (128, 4, 8192), (256, 2, 2048), (64, 1, 512)])
+def test_config_c5_points(n, B, P):
+    """C5 sweep points (random trees, depth <= 8), one layer, sampled requests vs the oracle."""
+    tb = W.random_tree_batch(B, n, P, seed=n + B + P, device=DEV)
+    smax = P + n
+    ai = W.make_attention_inputs(tb, 1, 32, 32, smax, seed=5, device=DEV)
+    out, _ = _gpu_attention(tb, ai, 32, 32)
+    bs = [0, B - 1] if B > 1 else [0]
+    _check_rows(out, _oracle_attention(ai, tb, bs=bs), tb, bs=bs)
+
+
+# ---------------------------------------------------------------------------------------------
+# verification
+# ---------------------------------------------------------------------------------------------
+
+def _verify_setup(tb, V, mode, seed, Hq=2, Hkv=2):
+    smax = int(tb.prefix_len.max()) + tb.max_nodes + 1
+    shape = _shape(tb, Hq, Hkv, smax, vocab=V)
+    st = spi.TreeState.create(shape, tb.parent, tb.depth, tb.prefix_len, tb.n_nodes)
+    st.prepare()
+    vi = W.make_verify_inputs(tb, V, seed=seed, mode=mode, device=DEV)
+    B, Lp = tb.parent.shape[0], tb.max_depth + 1
+    outs = [torch.empty((B, Lp), dtype=torch.int32, device=DEV), torch.empty((B, Lp), dtype=torch.int32, device=DEV),
+            torch.empty((B,), dtype=torch.int32, device=DEV)]
+    return shape, st, vi, outs
+
+
+@pytest.mark.parametrize("V", [7, 1000, 32000, 50272])
+def test_verify_greedy_parity(V):
+    rng = np.random.default_rng(V)
+    trees = [W.random_tree(int(rng.integers(1, 60)), 8, 4, rng) for _ in range(12)]
+    tb = W.make_tree_batch(trees, [5] * 12, max_nodes=64, max_depth=8, device=DEV)
+    shape, st, vi, (an, at, na) = _verify_setup(tb, V, "greedy", seed=V)
+    spi.specinfer_verify_greedy(shape, vi.logits, vi.tree_tokens, tb.parent, tb.n_nodes, an, at, na, st.workspace)
+    torch.cuda.synchronize()
+    r = oracle.verify_greedy(vi.logits.cpu().numpy(), vi.tree_tokens.cpu().numpy(), tb.parent.cpu().numpy(),
+                             tb.n_nodes.cpu().numpy(), path_len=9)
+    for x, y in zip(r, (an, at, na)):
+        assert np.array_equal(x, y.cpu().numpy())
+    # repeated call on the same workspace (counters reset) gives the same answer
+    spi.specinfer_verify_greedy(shape, vi.logits, vi.tree_tokens, tb.parent, tb.n_nodes, an, at, na, st.workspace)
+    torch.cuda.synchronize()
+    assert np.array_equal(r[2], na.cpu().numpy())
+
+
+def test_verify_greedy_fig2_and_ties(golden):
+    g = golden("fig2_greedy.json")
+    vocab = {w: i for i, w in enumerate(g["vocab"])}
+    par = np.asarray(g["parent"], np.int32)
+    dep = np.zeros(len(par), np.int32)
+    for i in range(1, len(par)):
+        dep[i] = dep[par[i]] + 1
+    tb = W.make_tree_batch([(par, dep)], [0], max_depth=int(dep.max()), device=DEV)
+    shape, st, vi, (an, at, na) = _verify_setup(tb, len(vocab), "greedy", seed=1)
+    lg = torch.zeros((1, len(par), len(vocab)), device=DEV)
+    for u, w in enumerate(g["llm_output"]):
+        lg[0, u, vocab[w]] = 1.0
+    toks = torch.tensor([[vocab[w] for w in g["tree_tokens"]]], dtype=torch.int32, device=DEV)
+    spi.specinfer_verify_greedy(shape, lg, toks, tb.parent, tb.n_nodes, an, at, na, st.workspace)
+    torch.cuda.synchronize()
+    assert na.item() == 3
+    assert an[0, :3].tolist() == g["expected_accepted_nodes"]
+    assert [g["vocab"][t] for t in at[0, :3].tolist()] == g["expected_tokens"]
+    # ties: all-zero logits -> token 0 everywhere
+    lg.zero_()
+    spi.specinfer_verify_greedy(shape, lg, toks, tb.parent, tb.n_nodes, an, at, na, st.workspace)
+    torch.cuda.synchronize()
+    assert at[0, 0].item() == 0 and na.item() == 1
+
+
+def _mss_compare(got, ref, margins, excuse=1e-5):
+    an, at, na = [x.cpu().numpy() for x in got]
+    r_an, r_at, r_na, _ = ref
+    bad = [b for b in range(len(na)) if not (na[b] == r_na[b] and np.array_equal(an[b], r_an[b])
+                                              and np.array_equal(at[b], r_at[b]))]
+    unexcused = [b for b in bad if margins[b] >= excuse]
+    assert not unexcused, f"MSS mismatches with margin >= {excuse}: {unexcused[:10]} (margins {margins[unexcused[:10]]})"
+    assert len(bad) <= max(1, int(1e-3 * len(na))), f"too many boundary cases: {len(bad)}"
+    return len(bad)
+
+
+@pytest.mark.parametrize("V,T", [(5, 1.0), (1000, 0.7), (32000, 1.0), (50272, 1.3)])
+def test_verify_mss_parity(V, T):
+    rng = np.random.default_rng(V + 1)
+    B = 48
+    trees = [W.random_tree(int(rng.integers(1, 40)), 8, 5, rng) for _ in range(B)]
+    tb = W.make_tree_batch(trees, [3] * B, max_nodes=40, max_depth=8, device=DEV)
+    shape, st, vi, outs = _verify_setup(tb, V, "mss", seed=V, Hq=1, Hkv=1)
+    rids = torch.arange(1000, 1000 + B, dtype=torch.int32, device=DEV)
+    spi.specinfer_verify_mss(shape, vi.logits, vi.tree_tokens, tb.parent, tb.n_nodes, vi.draft_probs, T, 1234,
+                             17, rids, *outs, st.workspace)
+    torch.cuda.synchronize()
+    ref = oracle.verify_mss(vi.logits.cpu().numpy(), vi.tree_tokens.cpu().numpy(), tb.parent.cpu().numpy(),
+                            tb.n_nodes.cpu().numpy(), vi.draft_probs.cpu().numpy(), temperature=T, seed=1234,
+                            offset=17, request_ids=rids.cpu().numpy(), path_len=9)
+    _mss_compare(outs, ref, ref[3])
+
+
+def test_verify_mss_config_c4_full():
+    """C4 (B=64, 233-node tree <8,4,1,...>, V=50272), full size, MSS."""
+    cfg = W.CONFIGS["C4"]
+    tb = W.config_tree_batch(cfg, device=DEV)
+    shape, st, vi, outs = _verify_setup(tb, cfg.vocab, "mss", seed=cfg.seed, Hq=1, Hkv=1)
+    spi.specinfer_verify_mss(shape, vi.logits, vi.tree_tokens, tb.parent, tb.n_nodes, vi.draft_probs, 1.0, 4, 0,
+                             None, *outs, st.workspace)
+    torch.cuda.synchronize()
+    ref = oracle.verify_mss(vi.logits.cpu().numpy(), vi.tree_tokens.cpu().numpy(), tb.parent.cpu().numpy(),
+                            tb.n_nodes.cpu().numpy(), vi.draft_probs.cpu().numpy(), seed=4, offset=0,
+                            path_len=cfg.max_depth + 1)
+    _mss_compare(outs, ref, ref[3])
+
+
+def test_verify_config_c2_full_greedy_and_mss():
+    cfg = W.CONFIGS["C2"]
+    tb = W.config_tree_batch(cfg, device=DEV)
+    for mode in ("greedy", "mss"):
+        shape, st, vi, (an, at, na) = _verify_setup(tb, cfg.vocab, mode, seed=cfg.seed)
+        if mode == "greedy":
+            spi.specinfer_verify_greedy(shape, vi.logits, vi.tree_tokens, tb.parent, tb.n_nodes, an, at, na,
+                                        st.workspace)
+            torch.cuda.synchronize()
+            r = oracle.verify_greedy(vi.logits.cpu().numpy(), vi.tree_tokens.cpu().numpy(), tb.parent.cpu().numpy(),
+                                     tb.n_nodes.cpu().numpy(), path_len=9)
+            for x, y in zip(r, (an, at, na)):
+                assert np.array_equal(x, y.cpu().numpy())
+        else:
+            spi.specinfer_verify_mss(shape, vi.logits, vi.tree_tokens, tb.parent, tb.n_nodes, vi.draft_probs, 1.0,
+                                     2, 0, None, an, at, na, st.workspace)
+            torch.cuda.synchronize()
+            r = oracle.verify_mss(vi.logits.cpu().numpy(), vi.tree_tokens.cpu().numpy(), tb.parent.cpu().numpy(),
+                                  tb.n_nodes.cpu().numpy(), vi.draft_probs.cpu().numpy(), seed=2, offset=0,
+                                  path_len=9)
+            _mss_compare((an, at, na), r, r[3])
+
+
+def test_philox_kat_on_device(golden):
+    g = golden("philox_kat.json")
+    ck = torch.tensor([[int(x, 16) for x in v["ctr"] + v["key"]] for v in g["vectors"]], dtype=torch.int64,
+                      device=DEV)
+    out = spi.specinfer_philox_debug(ck).cpu().numpy()
+    for row, v in zip(out, g["vectors"]):
+        assert [f"{int(x):08x}" for x in row] == v["out"]
+
+
+def test_verify_invalid_tree():
+    tb = W.make_tree_batch([W.chain_tree(5), W.chain_tree(5)], [0, 0], device=DEV)
+    tb.depth[0, 3] = 7   # depth mismatch
+    shape, st, vi, (an, at, na) = _verify_setup(tb, 50, "greedy", seed=3)
+    spi.specinfer_verify_greedy(shape, vi.logits, vi.tree_tokens, tb.parent, tb.n_nodes, an, at, na, st.workspace)
+    torch.cuda.synchronize()
+    assert na[0].item() == 0 and (an[0] == -1).all() and (at[0] == -1).all() and na[1].item() >= 1
+    spi.specinfer_verify_mss(shape, vi.logits, vi.tree_tokens, tb.parent, tb.n_nodes, vi.draft_probs, 1.0, 1, 0,
+                             None, an, at, na, st.workspace)
+    torch.cuda.synchronize()
+    assert na[0].item() == 0 and (an[0] == -1).all()
+    assert spi.specinfer_read_device_status(st.workspace) & 1
+
+
+# ---------------------------------------------------------------------------------------------
+# KV commit
+# ---------------------------------------------------------------------------------------------
+
+@pytest.mark.parametrize("L,Hkv", [(1, 2), (3, 8)])
+def test_kv_commit_parity(L, Hkv):
+    rng = np.random.default_rng(L * 10 + Hkv)
+    B = 9
+    trees = [W.random_tree(int(rng.integers(1, 30)), 8, 3, rng) for _ in range(B)]
+    pls = [int(x) for x in rng.integers(0, 100, B)]
+    tb = W.make_tree_batch(trees, pls, max_nodes=30, max_depth=8, device=DEV)
+    smax = max(pls) + 32
+    ai = W.make_attention_inputs(tb, 1, Hkv, Hkv, smax, seed=9, device=DEV, cache_layers=L)
+    shape = _shape(tb, Hkv, Hkv, smax, num_layers=L, vocab=64)
+    st = spi.TreeState.create(shape, tb.parent, tb.depth, tb.prefix_len, tb.n_nodes)
+    st.prepare()
+    vi = W.make_verify_inputs(tb, 64, seed=5, mode="greedy", device=DEV, tau=0.05)
+    an = torch.empty((B, 9), dtype=torch.int32, device=DEV)
+    at, na = torch.empty_like(an), torch.empty((B,), dtype=torch.int32, device=DEV)
+    spi.specinfer_verify_greedy(shape, vi.logits, vi.tree_tokens, tb.parent, tb.n_nodes, an, at, na, st.workspace)
+    na[2] = 0   # a request with nothing accepted (e.g. invalid tree) is left alone
+    k, v = ai.k_cache.clone(), ai.v_cache.clone()
+    pl = tb.prefix_len.clone()
+    spi.specinfer_kv_commit(shape, k, v, pl, an, na)
+    torch.cuda.synchronize()
+    kh = ai.k_cache.cpu().view(torch.int16).numpy().view(np.uint16).copy()
+    vh = ai.v_cache.cpu().view(torch.int16).numpy().view(np.uint16).copy()
+    plh = tb.prefix_len.cpu().numpy().copy()
+    oracle.kv_commit(kh, vh, plh, an.cpu().numpy(), na.cpu().numpy())
+    assert np.array_equal(plh, pl.cpu().numpy())
+    kg = k.cpu().view(torch.int16).numpy().view(np.uint16)
+    vg = v.cpu().view(torch.int16).numpy().view(np.uint16)
+    for b in range(B):
+        e = int(plh[b]) if na[b].item() > 0 else smax
+        assert np.array_equal(kh[:, b, :, :e], kg[:, b, :, :e])
+        assert np.array_equal(vh[:, b, :, :e], vg[:, b, :, :e])
+    assert int(na.cpu().numpy()[[0, 1, 3]].max()) >= 2  # some request committed a moved path
