@@ -147,6 +147,8 @@ class Workload:
         mode = "mss" if self.verify == ("mss",) else "greedy"
         self.vi = W.make_verify_inputs(self.tb, self.V, seed=seed, mode=mode, device=device)
         self.rids = torch.arange(rank * self.B, (rank + 1) * self.B, dtype=torch.int32, device=device)
+        self.bytes_launch = self.attn_bytes_per_launch()   # before any commit moves prefix_len
+        self.flops_launch = self.attn_flops_per_launch()
 
     def tree_tokens_per_step(self) -> int:
         return int(self.tb.n_nodes.sum().item())
@@ -280,8 +282,8 @@ def run_ours(args, ws, rank, local):
 
     # ---- roofline of the dominant kernel (tree attention), measured in the timed region ----
     attn_launch_s = attn_ms_max / (K * L) / 1e3
-    bytes_launch = wl.attn_bytes_per_launch()
-    flops_launch = wl.attn_flops_per_launch()
+    bytes_launch = wl.bytes_launch
+    flops_launch = wl.flops_launch
     peaks = {}
     try:
         peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
@@ -353,6 +355,8 @@ def run_ours(args, ws, rank, local):
 
     cpu = None
     if rank == 0 and ws == 1 and not args.no_cpu:
+        wl.tb.prefix_len.copy_(prefix0)   # undo the last step's commit: the sample is a fresh iteration
+        torch.cuda.synchronize(device)
         cpu = cpu_baseline(wl)
 
     line = {

@@ -151,6 +151,12 @@ specinfer_status_t specinfer_read_device_status(const void *workspace, specinfer
 specinfer_status_t specinfer_philox_debug(const uint32_t *ctr_key, uint32_t *out, int32_t n,
                                           specinfer_stream_t stream);
 
+/* Debug only: when `trace` (device, >= 8*64*8 uint64) is non-NULL, subsequent tree_attention
+ * launches record per-tile clock64() timestamps of CTAs 0-7 (trace[cta][tile][event]:
+ * 0/1 TMA issue of K/V, 2 S-MMA issue, 3 PV-MMA issue, 4 softmax start, 5 P ready, 6 tile
+ * done).  NULL (the default) disables it.  Not thread-safe; process-global. */
+void specinfer_debug_set_trace(void *trace);
+
 /* Number of kernel launches each call issues (for launch accounting in benchmarks). */
 int32_t specinfer_launches_per_call(const char *call_name);
 

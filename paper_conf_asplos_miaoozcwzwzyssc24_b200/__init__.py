@@ -28,7 +28,8 @@ STATUS_NAMES = {0: "OK", 1: "ERR_INVALID_ARG", 2: "ERR_UNSUPPORTED", 3: "ERR_CUD
 EXPORTED_SYMBOLS = (
     "specinfer_workspace_size", "specinfer_tree_prepare", "specinfer_tree_attention",
     "specinfer_verify_greedy", "specinfer_verify_mss", "specinfer_kv_commit",
-    "specinfer_read_device_status", "specinfer_philox_debug", "specinfer_launches_per_call",
+    "specinfer_read_device_status", "specinfer_philox_debug", "specinfer_debug_set_trace",
+    "specinfer_launches_per_call",
     "specinfer_status_string",
 )
 
@@ -78,6 +79,8 @@ def load_library(path: str = LIB_PATH):
     lib.specinfer_kv_commit.argtypes = [sp, vp, vp, vp, vp, vp, vp]
     lib.specinfer_read_device_status.argtypes = [vp, vp, ctypes.POINTER(i32)]
     lib.specinfer_philox_debug.argtypes = [vp, vp, i32, vp]
+    lib.specinfer_debug_set_trace.argtypes = [vp]
+    lib.specinfer_debug_set_trace.restype = None
     lib.specinfer_launches_per_call.argtypes = [ctypes.c_char_p]
     lib.specinfer_launches_per_call.restype = i32
     lib.specinfer_status_string.argtypes = [i32]
@@ -231,6 +234,11 @@ def specinfer_philox_debug(ctr_key: torch.Tensor) -> torch.Tensor:
     _check("specinfer_philox_debug", load_library().specinfer_philox_debug(
         ctypes.c_void_p(ck.data_ptr()), ctypes.c_void_p(out.data_ptr()), ck.shape[0], _stream(ck)))
     return out.to(torch.int64).bitwise_and(0xFFFFFFFF)
+
+
+def specinfer_debug_set_trace(trace: Optional[torch.Tensor]):
+    """Debug only: per-tile timestamps of tree_attention CTAs 0-7 into `trace` (int64 [8][64][8])."""
+    load_library().specinfer_debug_set_trace(None if trace is None else ctypes.c_void_p(trace.data_ptr()))
 
 
 def specinfer_launches_per_call(name: str) -> int:

@@ -3,6 +3,7 @@
 // Host-side argument validation, per-device capability cache (sm_100 check, SM count, max
 // dynamic shared memory), workspace layout, and the launches of the K1..K6 kernels.
 #include <math.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <mutex>
@@ -12,7 +13,7 @@
 namespace specinfer {
 cudaError_t launch_tree_prepare(const specinfer_shape_t &s, const WsLayout &w, const int32_t *parent,
                                 const int32_t *depth, const int32_t *prefix_len, const int32_t *n_nodes,
-                                char *ws, cudaStream_t stream);
+                                char *ws, int num_ctas, cudaStream_t stream);
 cudaError_t launch_tree_attention(const specinfer_shape_t &s, const WsLayout &w, const void *q, const void *k,
                                   const void *v, const int32_t *prefix_len, const int32_t *n_nodes, void *out,
                                   char *ws, int num_sms, size_t max_smem, cudaStream_t stream);
@@ -28,6 +29,8 @@ cudaError_t launch_verify_mss(const specinfer_shape_t &s, const WsLayout &w, con
 cudaError_t launch_kv_commit(const specinfer_shape_t &s, void *k_all, void *v_all, int32_t *prefix_len,
                              const int32_t *acc_nodes, const int32_t *n_acc, cudaStream_t stream);
 cudaError_t launch_philox_debug(const uint32_t *ck, uint32_t *out, int n, cudaStream_t stream);
+extern unsigned long long *g_attn_trace;
+extern int g_attn_debug_flags;
 }  // namespace specinfer
 
 using namespace specinfer;
@@ -88,6 +91,9 @@ specinfer_status_t check_ws(const void *ws) {
     return SPECINFER_OK;
 }
 
+// the persistent tree-attention grid: one CTA per SM (tree_prepare builds its schedule)
+int attention_grid(int num_sms) { return num_sms; }
+
 specinfer_status_t from_cuda(cudaError_t e) { return e == cudaSuccess ? SPECINFER_OK : SPECINFER_ERR_CUDA; }
 
 #define SPI_TRY(x)                                 \
@@ -117,7 +123,8 @@ specinfer_status_t specinfer_tree_prepare(const specinfer_shape_t *shape, const 
     SPI_TRY(check_device(&d));
     const WsLayout w = ws_layout(*shape, d.num_sms);
     return from_cuda(launch_tree_prepare(*shape, w, parent, depth, prefix_len, n_nodes,
-                                         reinterpret_cast<char *>(workspace), (cudaStream_t)stream));
+                                         reinterpret_cast<char *>(workspace), attention_grid(d.num_sms),
+                                         (cudaStream_t)stream));
 }
 
 specinfer_status_t specinfer_tree_attention(const specinfer_shape_t *shape, const void *q, const void *k_cache,
@@ -135,7 +142,7 @@ specinfer_status_t specinfer_tree_attention(const specinfer_shape_t *shape, cons
     SPI_TRY(check_device(&d));
     const WsLayout w = ws_layout(*shape, d.num_sms);
     return from_cuda(launch_tree_attention(*shape, w, q, k_cache, v_cache, prefix_len, n_nodes, out,
-                                           reinterpret_cast<char *>(workspace), d.num_sms, d.max_smem,
+                                           reinterpret_cast<char *>(workspace), attention_grid(d.num_sms), d.max_smem,
                                            (cudaStream_t)stream));
 }
 
@@ -209,6 +216,13 @@ specinfer_status_t specinfer_philox_debug(const uint32_t *ctr_key, uint32_t *out
     DeviceInfo d;
     SPI_TRY(check_device(&d));
     return from_cuda(launch_philox_debug(ctr_key, out, n, (cudaStream_t)stream));
+}
+
+void specinfer_debug_set_trace(void *trace) {
+    g_attn_trace = reinterpret_cast<unsigned long long *>(trace);
+    // experiment switches for pipeline studies (results invalid when set); never set in production
+    const char *f = getenv("SPECINFER_DEBUG_FLAGS");
+    g_attn_debug_flags = f ? atoi(f) : 0;
 }
 
 int32_t specinfer_launches_per_call(const char *name) {

@@ -26,8 +26,11 @@ struct WsLayout {
     size_t req_ok;      // int32[B]
     size_t anc;         // uint32[B][Nmax][8]   ancestor-or-self bitsets
     size_t desc;        // uint32[B][Nmax][8]   descendant-or-self bitsets
+    size_t rowmask;     // uint64[B][chunks][Nmax] query rows of chunk c that see tree key j
     size_t item_start;  // int32[n_items + 1]   tile prefix of the attention schedule
     size_t item_cnt;    // uint32[n_items]       split-combine counters
+    size_t item_info;   // int4[n_items]         {first tile, end tile, P_b, n_b}
+    size_t cta_info;    // int4[max_ctas][2]     {t0, t1, first item, total tiles}, item_info[first item]
     size_t part_o;      // float[max_ctas][2][NT][128]
     size_t part_ml;     // float[max_ctas][2][2][NT]
     size_t argmax;      // int32[B][Nmax]
@@ -65,8 +68,11 @@ inline WsLayout ws_layout(const specinfer_shape_t &s, int num_sms) {
     w.req_ok = take(size_t(B) * 4);
     w.anc = take(size_t(B) * N * kBitWords * 4);
     w.desc = take(size_t(B) * N * kBitWords * 4);
+    w.rowmask = take(size_t(B) * w.chunks * N * 8);
     w.item_start = take(size_t(w.n_items + 1) * 4);
     w.item_cnt = take(size_t(w.n_items) * 4);
+    w.item_info = take(size_t(w.n_items + 1) * 16);  // + sentinel
+    w.cta_info = take(size_t(w.max_ctas) * 32);
     w.part_o = take(size_t(w.max_ctas) * 2 * w.nt * kHeadDim * 4);
     w.part_ml = take(size_t(w.max_ctas) * 2 * 2 * w.nt * 4);
     w.argmax = take(size_t(B) * N * 4);
@@ -170,6 +176,25 @@ __device__ __forceinline__ void tma_load_3d(void *dst, const CUtensorMap *map, u
         " [%0], [%1, {%3, %4, %5}], [%2];" ::"r"(smem_u32(dst)),
         "l"(reinterpret_cast<uint64_t>(map)), "r"(smem_u32(bar)), "r"(x), "r"(y), "r"(z)
         : "memory");
+}
+
+// bulk async copy shared -> global (no tensor map), tracked by bulk groups of this thread
+__device__ __forceinline__ void bulk_store_s2g(void *gdst, const void *ssrc, uint32_t bytes) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(gdst), "r"(smem_u32(ssrc)),
+                 "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+// waits until all committed bulk copies of this thread have finished READING shared memory
+__device__ __forceinline__ void bulk_wait_read_all() {
+    asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+
+// ---- programmatic dependent launch ---------------------------------------------------------
+__device__ __forceinline__ void grid_dependency_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void grid_launch_dependents() {
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
 }
 
 // ---- tcgen05 / TMEM ------------------------------------------------------------------------

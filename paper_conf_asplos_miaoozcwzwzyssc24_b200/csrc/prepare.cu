@@ -13,8 +13,8 @@ namespace specinfer {
 __global__ void __launch_bounds__(256) tree_validate_bitsets_kernel(
     const int32_t *__restrict__ parent, const int32_t *__restrict__ depth,
     const int32_t *__restrict__ prefix_len, const int32_t *__restrict__ n_nodes, int Nmax,
-    int max_depth, int Smax, int32_t *__restrict__ status, int32_t *__restrict__ req_ok,
-    uint32_t *__restrict__ anc, uint32_t *__restrict__ desc) {
+    int max_depth, int Smax, int G, int npc, int chunks, int32_t *__restrict__ status, int32_t *__restrict__ req_ok,
+    uint32_t *__restrict__ anc, uint32_t *__restrict__ desc, unsigned long long *__restrict__ rowmask) {
     const int b = blockIdx.x;
     __shared__ int32_t s_par[kMaxNodes];
     __shared__ uint32_t s_anc[kMaxNodes][kBitWords];
@@ -75,6 +75,20 @@ __global__ void __launch_bounds__(256) tree_validate_bitsets_kernel(
 #pragma unroll
         for (int k = 0; k < kBitWords; ++k) desc[((size_t)b * Nmax + j) * kBitWords + k] = w[k];
     }
+    // row masks of the tree part for the attention kernel: bit r of rowmask[b][c][j] is set iff
+    // query row r of chunk c (node c*npc + r/G) exists and has tree node j on its root path
+    const int rc = G * npc;
+    for (int idx = threadIdx.x; idx < chunks * Nmax; idx += blockDim.x) {
+        const int c = idx / Nmax, j = idx - c * Nmax;
+        unsigned long long m = 0ull;
+        if (ok && j < n) {
+            for (int r = 0; r < rc; ++r) {
+                const int node = c * npc + r / G;
+                if (node < n && ((s_anc[node][j >> 5] >> (j & 31)) & 1u)) m |= 1ull << r;
+            }
+        }
+        rowmask[((size_t)b * chunks + c) * Nmax + j] = m;
+    }
     if (threadIdx.x == 0) {
         req_ok[b] = ok ? 1 : 0;
         if (!ok) atomicOr(status, kStatusBadTree);
@@ -85,8 +99,8 @@ __global__ void __launch_bounds__(256) tree_validate_bitsets_kernel(
 __global__ void __launch_bounds__(1024) schedule_kernel(
     const int32_t *__restrict__ prefix_len, const int32_t *__restrict__ n_nodes,
     const int32_t *__restrict__ req_ok, int B, int Hkv, int chunks, int npc,
-    int32_t *__restrict__ item_start, uint32_t *__restrict__ item_cnt,
-    uint32_t *__restrict__ verify_cnt, int32_t *__restrict__ status) {
+    int32_t *__restrict__ item_start, uint32_t *__restrict__ item_cnt, int4 *__restrict__ item_info,
+    int4 *__restrict__ cta_info, int num_ctas, uint32_t *__restrict__ verify_cnt, int32_t *__restrict__ status) {
     const int n_items = B * Hkv * chunks;
     const int per = (n_items + blockDim.x - 1) / blockDim.x;
     const int lo = threadIdx.x * per;
@@ -124,35 +138,56 @@ __global__ void __launch_bounds__(1024) schedule_kernel(
     __syncthreads();
     int run = v - local + (wid > 0 ? s_warp[wid - 1] : 0);
     for (int x = lo; x < hi; ++x) {
+        const int tl = tiles_of(x);
+        const int b = x / (chunks * Hkv);
         item_start[x] = run;
-        run += tiles_of(x);
+        item_info[x] = make_int4(run, run + tl, prefix_len[b], n_nodes[b]);
+        run += tl;
         item_cnt[x] = 0u;
     }
+    __shared__ int s_total;
     if (threadIdx.x == blockDim.x - 1) {
         item_start[n_items] = run;
+        item_info[n_items] = make_int4(run, run, 0, 0);
         status[1] = run;
+        s_total = run;
     }
     for (int b = threadIdx.x; b < B; b += blockDim.x) verify_cnt[b] = 0u;
+    __syncthreads();
+    // per-CTA slice [t0, t1) of the tile sequence for the attention grid, and its first item
+    const long long T = s_total;
+    for (int c = threadIdx.x; c < num_ctas; c += blockDim.x) {
+        const int t0 = (int)((long long)c * T / num_ctas);
+        const int t1 = (int)((long long)(c + 1) * T / num_ctas);
+        int lo2 = 0, hi2 = n_items;  // last item with start <= t0
+        while (hi2 - lo2 > 1) {
+            const int mid = (lo2 + hi2) >> 1;
+            if (item_start[mid] <= t0) lo2 = mid; else hi2 = mid;
+        }
+        cta_info[2 * c] = make_int4(t0, t1, lo2, (int)T);
+        cta_info[2 * c + 1] = lo2 < n_items ? item_info[lo2] : make_int4(0, 0, 0, 0);
+    }
 }
 
 cudaError_t launch_tree_prepare(const specinfer_shape_t &s, const WsLayout &w,
                                 const int32_t *parent, const int32_t *depth,
                                 const int32_t *prefix_len, const int32_t *n_nodes, char *ws,
-                                cudaStream_t stream) {
+                                int num_ctas, cudaStream_t stream) {
     int32_t *status = reinterpret_cast<int32_t *>(ws + w.status);
     cudaError_t e = cudaMemsetAsync(status, 0, 64 * 4, stream);
     if (e != cudaSuccess) return e;
     tree_validate_bitsets_kernel<<<s.batch, 256, 0, stream>>>(
-        parent, depth, prefix_len, n_nodes, s.max_nodes, s.max_depth, s.max_seq, status,
-        reinterpret_cast<int32_t *>(ws + w.req_ok), reinterpret_cast<uint32_t *>(ws + w.anc),
-        reinterpret_cast<uint32_t *>(ws + w.desc));
+        parent, depth, prefix_len, n_nodes, s.max_nodes, s.max_depth, s.max_seq,
+        s.num_q_heads / s.num_kv_heads, w.npc, w.chunks, status, reinterpret_cast<int32_t *>(ws + w.req_ok),
+        reinterpret_cast<uint32_t *>(ws + w.anc), reinterpret_cast<uint32_t *>(ws + w.desc),
+        reinterpret_cast<unsigned long long *>(ws + w.rowmask));
     e = cudaGetLastError();
     if (e != cudaSuccess) return e;
     schedule_kernel<<<1, 1024, 0, stream>>>(
         prefix_len, n_nodes, reinterpret_cast<int32_t *>(ws + w.req_ok), s.batch,
         s.num_kv_heads, w.chunks, w.npc, reinterpret_cast<int32_t *>(ws + w.item_start),
-        reinterpret_cast<uint32_t *>(ws + w.item_cnt),
-        reinterpret_cast<uint32_t *>(ws + w.verify_cnt), status);
+        reinterpret_cast<uint32_t *>(ws + w.item_cnt), reinterpret_cast<int4 *>(ws + w.item_info),
+        reinterpret_cast<int4 *>(ws + w.cta_info), num_ctas, reinterpret_cast<uint32_t *>(ws + w.verify_cnt), status);
     return cudaGetLastError();
 }
 

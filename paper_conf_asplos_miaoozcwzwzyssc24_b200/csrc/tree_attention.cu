@@ -7,21 +7,25 @@
 // (the topology-aware causal mask, one fused kernel for all tree tokens, L657-674).
 //
 // How (B200-first design):
-//  * Work = the whole KV stream of one layer, B*Hkv items x ceil((P_b+n_b)/128) tiles of 128
-//    keys, split evenly over a persistent grid (one CTA per SM) at tile granularity
-//    (stream-K).  Items cut by a CTA boundary write fp32 partials (O, m, l) and the last piece
-//    to finish merges them (log-sum-exp), so one launch per layer and no tail wave.
-//  * Each KV tile is read from HBM once by TMA (128B-swizzled, 2 x 16 KB boxes per tile) into
-//    a ring of 32 KB smem slots and shared by ALL G*n_b query rows of the kv-head.
+//  * Work = the whole KV stream of one layer: items (b, kv-head, row chunk) x ceil((P_b+n_b)/128)
+//    tiles of 128 keys, split evenly over a persistent grid (one CTA per SM) at tile
+//    granularity (stream-K).  Items cut by a CTA boundary write fp32 partials (O, m, l); the
+//    last piece to finish merges them (log-sum-exp): one launch per layer, no tail wave.
+//  * Each KV tile is read from HBM once by TMA (128B-swizzled 16 KB boxes) and shared by ALL
+//    G*n_b query rows of the kv-head.  K and V have separate smem rings (K tiles are released
+//    right after S = K Q^T, so K prefetch never waits for a PV), fed by two producer lanes.
 //  * "Swapped" tensor-core formulation for few query rows: S^T = K Q^T (UMMA M = 128 keys,
-//    N = NT query rows, K = 128 dims) and O^T += V^T P^T (M = 128 dims, N = NT, K = 128 keys),
+//    N = NT query rows, K = 128 dims) and O^T += V^T P^T (M = 128 dims, N = NT, K = 128 keys);
 //    tcgen05.mma kind::f16 issued by one thread, fp32 accumulators in TMEM.
-//  * 4 softmax warps own one key (TMEM lane) each: fp32 scale + mask (ancestor bitsets from
-//    tree_prepare) + exp2, P rounded to bf16 into smem (MN-major, swizzled) for the PV MMA.
-//    Running row maxima are kept "stale" until a tile raises some row by more than 2^8
-//    (exactly rescaled then, O^T rescaled in TMEM), so the common path needs no reduction
-//    across lanes other than the row sums (transpose-reduce with warp shuffles).
-//  * warp 0: TMA producer; warp 1: TMEM allocator + MMA issuer; warps 2-5: softmax/epilogue.
+//  * 4 softmax warps own one key (TMEM lane) each: fp32 scale, tree mask (row masks from
+//    tree_prepare; committed keys need none), exp2, P rounded to bf16 into smem (MN-major,
+//    swizzled) for the PV MMA, row sums kept per thread and reduced once per segment.  The
+//    running row maxima stay "stale" until a tile raises a row by more than 2^8; then they are
+//    recomputed exactly and O^T is rescaled in TMEM (the rare path).
+//  * Segment metadata is decoded once by the producer and passed through an smem ring, so no
+//    consumer waits on a global load at item boundaries.
+//  * warp 0: TMA producers (lane 0: Q + K + segment ring, lane 1: V); warp 1: TMEM allocator +
+//    MMA issuer; warps 2-5: softmax / epilogue / split combine.
 #include "common.cuh"
 
 namespace specinfer {
@@ -30,19 +34,46 @@ struct AttnParams {
     const int32_t *prefix_len;
     const int32_t *n_nodes;
     const int32_t *item_start;
+    const int4 *item_info;
+    const int4 *cta_info;
     uint32_t *item_cnt;
-    const uint32_t *desc;
+    const unsigned long long *rowmask;
     float *part_o;
     float *part_ml;
     __nv_bfloat16 *out;
-    int B, Nmax, Hq, Hkv, G, Smax, chunks, npc, n_items, num_slots;
+    int B, Nmax, Hq, Hkv, G, Smax, chunks, npc, n_items, nk_slots, nv_slots;
     float scale_log2;
+    unsigned long long *trace;  // optional per-tile timestamps (debug), nullptr in production
+    int debug_flags;            // experiments only: 1 = skip K/V TMA, 2 = skip MMAs (results invalid)
 };
+
+// debug timestamps: trace[cta][tile][event], CTAs < kTraceCtas, tiles < kTraceTiles
+constexpr int kTraceCtas = 8, kTraceTiles = 64, kTraceEv = 12;
+__device__ __forceinline__ unsigned long long globaltimer_ns() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+// kernel-level timestamps of every CTA (ns): [entry, exit, first K issue, 0]
+#define SPI_TRACE_K(slot)                                                                                  \
+    do {                                                                                                   \
+        if (p.trace != nullptr)                                                                            \
+            p.trace[(size_t)kTraceCtas * kTraceTiles * kTraceEv + blockIdx.x * 4 + (slot)] = globaltimer_ns(); \
+    } while (0)
+#define SPI_TRACE(ev)                                                                               \
+    do {                                                                                            \
+        if (p.trace != nullptr && blockIdx.x < kTraceCtas && lt < kTraceTiles)                      \
+            p.trace[((size_t)blockIdx.x * kTraceTiles + lt) * kTraceEv + (ev)] = clock64();         \
+    } while (0)
 
 constexpr int kSlotBytes = kKeyTile * kHeadDim * 2;  // 32 KB: one K or V tile
 constexpr int kHalfBytes = kSlotBytes / 2;            // 16 KB: 128 keys x 64 dims
-constexpr int kTailRows = 16;                          // row granularity of partial tiles
+// the last tile of a request is loaded row-exactly (boxes of 16, 4 and 1 rows) so that no cache
+// slot at or beyond P_b + n_b is ever read; the rest of the slot keeps stale finite data
 constexpr float kRescaleThreshold = 8.0f;              // log2 units: stale max tolerance
+constexpr int kCombineBatch = 8;                       // split pieces merged per round
+constexpr int kSegRing = 16;                           // segment descriptors in flight
+constexpr int kMaxSlots = 8;
 
 template <int NT>
 struct SmemPlan {
@@ -53,49 +84,30 @@ struct SmemPlan {
     static constexpr int kTmemCols = (3 * NT <= 32) ? 32 : (3 * NT <= 64 ? 64 : (3 * NT <= 128 ? 128 : 256));
 };
 
+struct SegDesc {
+    int x, begin, end, ib, ie, b, g, c, P, n;
+};
+
 struct SmemMisc {
-    uint64_t slot_full[16];
-    uint64_t slot_empty[16];
+    uint64_t k_full[kMaxSlots], k_empty[kMaxSlots];
+    uint64_t v_full[kMaxSlots], v_empty[kMaxSlots];
     uint64_t q_full[2], q_empty[2];
     uint64_t s_full[2], s_empty[2];
-    uint64_t p_full[2], p_empty[2];
+    uint64_t p_full, p_empty;  // single P^T buffer: written by softmax(t) after PV(t-1) read it
+    uint64_t seg_full[kSegRing];
+    SegDesc seg[kSegRing];
     uint32_t tmem_base;
     int32_t flags[2][4];
     int32_t bcast;
-    alignas(16) float m_run[64];
+    alignas(16) float m_thr[64];   // running row max + threshold (-inf: no key seen yet)
+    alignas(16) float m_ref[64];   // running row max used as exp2 reference (0 if none yet)
     alignas(16) float alpha[64];
     alignas(16) float l_part[4][64];
     alignas(16) float wred[4][64];
-};
-
-// Iterates the (item, tile-range) segments of this CTA's contiguous tile range [t0, t1).
-struct SegIter {
-    const int32_t *item_start;
-    int t0, t1, x;
-    int begin, end, ib, ie;
-    __device__ void init(const int32_t *is, int n_items, int t0_, int t1_) {
-        item_start = is;
-        t0 = t0_;
-        t1 = t1_;
-        // last item with start <= t0
-        int lo = 0, hi = n_items;  // answer in [0, n_items)
-        while (hi - lo > 1) {
-            const int mid = (lo + hi) >> 1;
-            if (item_start[mid] <= t0) lo = mid; else hi = mid;
-        }
-        x = lo - 1;
-    }
-    __device__ bool next() {
-        for (;;) {
-            ++x;
-            ib = item_start[x];
-            if (ib >= t1) return false;
-            ie = item_start[x + 1];
-            begin = max(t0, ib);
-            end = min(t1, ie);
-            if (end > begin) return true;
-        }
-    }
+    // split-combine state (the per-piece staging arrays live in the idle P^T buffer)
+    alignas(16) float run_m[64];
+    alignas(16) float run_l[64];
+    size_t piece_off[kCombineBatch];
 };
 
 __device__ __forceinline__ int cta_start(long long c, long long T, long long NC) {
@@ -110,6 +122,8 @@ __device__ __forceinline__ int cta_of_tile(int t, int T, int NC) {
     return c;
 }
 
+// Cross-lane "transpose reduction": on entry each lane holds N values (one per row); on exit
+// lane l holds in v[0] the reduction over the 32 lanes of row (l mod N) (N <= 32).
 template <int N, bool kIsMax>
 __device__ __forceinline__ void transpose_reduce(float *v) {
     const int lane = threadIdx.x & 31;
@@ -131,44 +145,68 @@ __device__ __forceinline__ void transpose_reduce(float *v) {
     }
 }
 
+// Loads rows [row0, row0 + nv) of a K or V tile (nv < 128) with boxes of 16, 4 and 1 rows.
+__device__ __forceinline__ void tma_load_rows(uint8_t *dst, uint64_t *bar, int nv, int row0, uint64_t pol,
+                                              const CUtensorMap *m16, const CUtensorMap *m4,
+                                              const CUtensorMap *m1) {
+    mbar_arrive_expect_tx(bar, (uint32_t)nv * 256u);
+    int r = 0;
+    for (; r + 16 <= nv; r += 16) {
+        tma_load_2d(dst + r * 128, m16, bar, 0, row0 + r, pol);
+        tma_load_2d(dst + kHalfBytes + r * 128, m16, bar, 64, row0 + r, pol);
+    }
+    for (; r + 4 <= nv; r += 4) {
+        tma_load_2d(dst + r * 128, m4, bar, 0, row0 + r, pol);
+        tma_load_2d(dst + kHalfBytes + r * 128, m4, bar, 64, row0 + r, pol);
+    }
+    for (; r < nv; ++r) {
+        tma_load_2d(dst + r * 128, m1, bar, 0, row0 + r, pol);
+        tma_load_2d(dst + kHalfBytes + r * 128, m1, bar, 64, row0 + r, pol);
+    }
+}
+
 template <int NT>
-__global__ void __launch_bounds__(192, 1)
+__global__ void __launch_bounds__(224, 1)
     tree_attn_kernel(const __grid_constant__ CUtensorMap tm_q, const __grid_constant__ CUtensorMap tm_k,
                      const __grid_constant__ CUtensorMap tm_v, const __grid_constant__ CUtensorMap tm_k16,
-                     const __grid_constant__ CUtensorMap tm_v16, const AttnParams p) {
+                     const __grid_constant__ CUtensorMap tm_v16, const __grid_constant__ CUtensorMap tm_k4,
+                     const __grid_constant__ CUtensorMap tm_v4, const __grid_constant__ CUtensorMap tm_k1,
+                     const __grid_constant__ CUtensorMap tm_v1, const AttnParams p) {
     using Plan = SmemPlan<NT>;
     extern __shared__ __align__(1024) uint8_t smem_raw[];
-    uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-    const int NS = p.num_slots;
-    uint8_t *s_slots = smem;
-    uint8_t *s_q = s_slots + (size_t)NS * kSlotBytes;
+    // keep the pointer derived from smem_raw so the compiler emits LDS/STS, not generic LD/ST
+    uint8_t *smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
+    const int NK = p.nk_slots, NV = p.nv_slots;
+    uint8_t *s_k = smem;
+    uint8_t *s_v = s_k + (size_t)NK * kSlotBytes;
+    uint8_t *s_q = s_v + (size_t)NV * kSlotBytes;
     uint8_t *s_p = s_q + 2 * Plan::kQBuf;
-    SmemMisc *misc = reinterpret_cast<SmemMisc *>(s_p + 2 * Plan::kPBuf);
+    SmemMisc *misc = reinterpret_cast<SmemMisc *>(s_p + Plan::kPBuf);
 
     const int warp = threadIdx.x >> 5;
     const int lane = threadIdx.x & 31;
 
-    const int T = p.item_start[p.n_items];
+    if (threadIdx.x == 0) SPI_TRACE_K(0);
     const int NC = gridDim.x;
-    const int t0 = cta_start(blockIdx.x, T, NC);
-    const int t1 = cta_start(blockIdx.x + 1, T, NC);
-    if (t1 <= t0) return;  // uniform across the CTA
-
     if (threadIdx.x == 0) {
-        for (int i = 0; i < NS; ++i) {
-            mbar_init(&misc->slot_full[i], 1);
-            mbar_init(&misc->slot_empty[i], 1);
+        for (int i = 0; i < NK; ++i) {
+            mbar_init(&misc->k_full[i], 1);
+            mbar_init(&misc->k_empty[i], 1);
+        }
+        for (int i = 0; i < NV; ++i) {
+            mbar_init(&misc->v_full[i], 1);
+            mbar_init(&misc->v_empty[i], 1);
         }
         for (int i = 0; i < 2; ++i) {
             mbar_init(&misc->q_full[i], 1);
             mbar_init(&misc->q_empty[i], 1);
             mbar_init(&misc->s_full[i], 1);
-            mbar_init(&misc->s_empty[i], 128);
-            mbar_init(&misc->p_full[i], 4);
-            mbar_init(&misc->p_empty[i], 1);
+            mbar_init(&misc->s_empty[i], 4);
         }
+        mbar_init(&misc->p_full, 4);
+        mbar_init(&misc->p_empty, 1);
+        for (int i = 0; i < kSegRing; ++i) mbar_init(&misc->seg_full[i], 1);
         fence_barrier_init();
-        fence_proxy_async_smem();
     }
     if (warp == 0 && lane == 0) {
         tma_prefetch_desc(&tm_q);
@@ -176,6 +214,19 @@ __global__ void __launch_bounds__(192, 1)
         tma_prefetch_desc(&tm_v);
         tma_prefetch_desc(&tm_k16);
         tma_prefetch_desc(&tm_v16);
+        tma_prefetch_desc(&tm_k4);
+        tma_prefetch_desc(&tm_v4);
+        tma_prefetch_desc(&tm_k1);
+        tma_prefetch_desc(&tm_v1);
+    }
+    if (warp >= 3) {
+        // Q rows beyond a chunk's G*npc rows are never written by TMA: keep them zero
+        for (int i = threadIdx.x - 96; i < 2 * Plan::kQBuf / 16; i += 128)
+            reinterpret_cast<uint4 *>(s_q)[i] = make_uint4(0, 0, 0, 0);
+        // V rows past a request's last key are never loaded: they must hold finite data (0 * NaN)
+        for (int i = threadIdx.x - 96; i < NV * kSlotBytes / 16; i += 128)
+            reinterpret_cast<uint4 *>(s_v)[i] = make_uint4(0, 0, 0, 0);
+        fence_proxy_async_smem();
     }
     if (warp == 1) tmem_alloc<Plan::kTmemCols>(&misc->tmem_base);
     tc_fence_before();
@@ -184,100 +235,124 @@ __global__ void __launch_bounds__(192, 1)
     const uint32_t tmem = misc->tmem_base;
     const uint32_t tm_S0 = tmem, tm_O = tmem + 2 * NT;
 
-    SegIter it;
-    it.init(p.item_start, p.n_items, t0, t1);
+    // Programmatic dependent launch: everything above overlapped the previous kernel's tail;
+    // from here on we read inputs it may have produced.
+    grid_dependency_wait();
+    // this CTA's slice of the tile sequence (precomputed by tree_prepare for this grid)
+    const int4 ci = __ldg(p.cta_info + 2 * blockIdx.x);
+    const int4 first_info = __ldg(p.cta_info + 2 * blockIdx.x + 1);
+    const int t0 = ci.x, t1 = ci.y, x_first = ci.z, T = ci.w;
+    const int ntiles = t1 - t0;
 
-    if (warp == 0) {
-        // ============================ TMA producer ============================
+    if (ntiles <= 0) {
+        // no work for this CTA (fewer tiles than CTAs)
+    } else if (warp == 0) {
+        // ============================ TMA producers ============================
+        const uint64_t pol = l2_evict_first_policy();
         if (lane == 0) {
-            const uint64_t pol = l2_evict_first_policy();
+            // segment descriptors for every role, Q, and the K tiles
             int lt = 0, ls = 0;
-            while (it.next()) {
-                const int x = it.x;
-                const int c = x % p.chunks;
-                const int g = (x / p.chunks) % p.Hkv;
-                const int b = x / (p.chunks * p.Hkv);
-                const int Kend = p.prefix_len[b] + p.n_nodes[b];
+            int4 next_info = first_info;
+            for (int x = x_first; lt < ntiles; ++x) {
+                const int4 info = next_info;  // {first tile, end tile, P, n}
+                next_info = __ldg(p.item_info + x + 1);  // prefetched a segment ahead (sentinel-safe)
+                const int begin = max(t0, info.x), end = min(t1, info.y);
+                if (end <= begin) continue;
+                SegDesc d;
+                d.x = x;
+                d.begin = begin;
+                d.end = end;
+                d.ib = info.x;
+                d.ie = info.y;
+                d.c = x % p.chunks;
+                d.g = (x / p.chunks) % p.Hkv;
+                d.b = x / (p.chunks * p.Hkv);
+                d.P = info.z;
+                d.n = info.w;
+                misc->seg[ls % kSegRing] = d;
+                mbar_arrive(&misc->seg_full[ls % kSegRing]);  // release: descriptor visible
+                const int Kend = d.P + d.n;
                 const int qb = ls & 1;
                 if (ls >= 2) mbar_wait(&misc->q_empty[qb], ((ls >> 1) - 1) & 1);
-                const uint32_t qbytes = 2u * (uint32_t)(p.G * p.npc) * 128u;
-                mbar_arrive_expect_tx(&misc->q_full[qb], qbytes);
+                mbar_arrive_expect_tx(&misc->q_full[qb], 2u * (uint32_t)(p.G * p.npc) * 128u);
                 uint8_t *qdst = s_q + qb * Plan::kQBuf;
-                const int node0 = b * p.Nmax + c * p.npc;
-                tma_load_3d(qdst, &tm_q, &misc->q_full[qb], 0, g * p.G, node0);
-                tma_load_3d(qdst + NT * 128, &tm_q, &misc->q_full[qb], 64, g * p.G, node0);
-                const long long rowbase = (long long)(b * p.Hkv + g) * p.Smax;
-                for (int t = it.begin; t < it.end; ++t, ++lt) {
-                    const int key0 = (t - it.ib) * kKeyTile;
+                const int node0 = d.b * p.Nmax + d.c * p.npc;
+                tma_load_3d(qdst, &tm_q, &misc->q_full[qb], 0, d.g * p.G, node0);
+                tma_load_3d(qdst + NT * 128, &tm_q, &misc->q_full[qb], 64, d.g * p.G, node0);
+                const long long rowbase = (long long)(d.b * p.Hkv + d.g) * p.Smax;
+                for (int t = d.begin; t < d.end; ++t, ++lt) {
+                    const int key0 = (t - d.ib) * kKeyTile;
                     const int nv = min(kKeyTile, Kend - key0);
                     const int row0 = (int)(rowbase + key0);
-#pragma unroll
-                    for (int which = 0; which < 2; ++which) {
-                        const int seq = 2 * lt + which;
-                        const int slot = seq % NS;
-                        const int f = seq / NS;
-                        if (f >= 1) mbar_wait(&misc->slot_empty[slot], (f - 1) & 1);
-                        uint8_t *dst = s_slots + (size_t)slot * kSlotBytes;
-                        uint64_t *bar = &misc->slot_full[slot];
-                        if (nv == kKeyTile) {
-                            mbar_arrive_expect_tx(bar, kSlotBytes);
-                            const CUtensorMap *m = which ? &tm_v : &tm_k;
-                            tma_load_2d(dst, m, bar, 0, row0, pol);
-                            tma_load_2d(dst + kHalfBytes, m, bar, 64, row0, pol);
-                        } else {
-                            const int nb = (nv + kTailRows - 1) / kTailRows;
-                            mbar_arrive_expect_tx(bar, (uint32_t)nb * kTailRows * 128u * 2u);
-                            const CUtensorMap *m = which ? &tm_v16 : &tm_k16;
-                            for (int i = 0; i < nb; ++i) {
-                                tma_load_2d(dst + i * kTailRows * 128, m, bar, 0, row0 + i * kTailRows, pol);
-                                tma_load_2d(dst + kHalfBytes + i * kTailRows * 128, m, bar, 64,
-                                            row0 + i * kTailRows, pol);
-                            }
-                        }
+                    const int slot = lt % NK, f = lt / NK;
+                    if (f >= 1) mbar_wait(&misc->k_empty[slot], (f - 1) & 1);
+                    SPI_TRACE(0);
+                    if (lt == 0) SPI_TRACE_K(2);
+                    uint8_t *dst = s_k + (size_t)slot * kSlotBytes;
+                    uint64_t *bar = &misc->k_full[slot];
+                    if (p.debug_flags & 1) {
+                        mbar_arrive(bar);
+                    } else if (nv == kKeyTile) {
+                        mbar_arrive_expect_tx(bar, kSlotBytes);
+                        tma_load_2d(dst, &tm_k, bar, 0, row0, pol);
+                        tma_load_2d(dst + kHalfBytes, &tm_k, bar, 64, row0, pol);
+                    } else {
+                        tma_load_rows(dst, bar, nv, row0, pol, &tm_k16, &tm_k4, &tm_k1);
+                    }
+                }
+                ++ls;
+            }
+            grid_launch_dependents();  // all of this CTA's K loads are issued
+        } else if (lane == 1) {
+            // V tiles, following the segment ring written by lane 0
+            int lt = 0, ls = 0;
+            while (lt < ntiles) {
+                mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
+                const SegDesc d = misc->seg[ls % kSegRing];
+                const int Kend = d.P + d.n;
+                const long long rowbase = (long long)(d.b * p.Hkv + d.g) * p.Smax;
+                for (int t = d.begin; t < d.end; ++t, ++lt) {
+                    const int key0 = (t - d.ib) * kKeyTile;
+                    const int nv = min(kKeyTile, Kend - key0);
+                    const int row0 = (int)(rowbase + key0);
+                    const int slot = lt % NV, f = lt / NV;
+                    if (f >= 1) mbar_wait(&misc->v_empty[slot], (f - 1) & 1);
+                    SPI_TRACE(1);
+                    uint8_t *dst = s_v + (size_t)slot * kSlotBytes;
+                    uint64_t *bar = &misc->v_full[slot];
+                    if (p.debug_flags & 1) {
+                        mbar_arrive(bar);
+                    } else if (nv == kKeyTile) {
+                        mbar_arrive_expect_tx(bar, kSlotBytes);
+                        tma_load_2d(dst, &tm_v, bar, 0, row0, pol);
+                        tma_load_2d(dst + kHalfBytes, &tm_v, bar, 64, row0, pol);
+                    } else {
+                        tma_load_rows(dst, bar, nv, row0, pol, &tm_v16, &tm_v4, &tm_v1);
                     }
                 }
                 ++ls;
             }
         }
     } else if (warp == 1) {
-        // ============================ MMA issuer ==============================
+        // ===================== S issuer: S^T = K Q^T per tile =====================
+        // (its own warp so that S(t+1) never queues behind PV(t) in one thread's program order)
         if (lane == 0) {
             const uint32_t idesc_s = make_idesc_bf16(128, NT, false, false);
-            const uint32_t idesc_o = make_idesc_bf16(128, NT, true, true);
-            const uint32_t slots_addr = smem_u32(s_slots);
-            const uint32_t q_addr = smem_u32(s_q);
-            const uint32_t p_addr = smem_u32(s_p);
+            const uint32_t k_addr = smem_u32(s_k), q_addr = smem_u32(s_q);
             int lt = 0, ls = 0;
-            bool prev_first = false;  // tile lt-1 was the first of its segment
-            auto issue_pv = [&](int u, bool first) {
-                mbar_wait(&misc->p_full[u & 1], (u >> 1) & 1);
-                const int seq = 2 * u + 1;
-                const int slot = seq % NS;
-                mbar_wait(&misc->slot_full[slot], (seq / NS) & 1);
-                tc_fence_after();
-                const uint32_t vbase = slots_addr + slot * kSlotBytes;
-                const uint32_t pbase = p_addr + (u & 1) * Plan::kPBuf;
-#pragma unroll
-                for (int kk = 0; kk < kKeyTile / 16; ++kk) {
-                    const uint64_t adesc = make_smem_desc(vbase + kk * 16 * 128, kHalfBytes, 1024, kSw128);
-                    const uint64_t bdesc = make_smem_desc(pbase + kk * 16 * (NT * 2), Plan::kPBuf,
-                                                          8 * NT * 2, Plan::kPSwizzle);
-                    umma_bf16_ss(tm_O, adesc, bdesc, idesc_o, (first && kk == 0) ? 0u : 1u);
-                }
-                umma_commit(&misc->p_empty[u & 1]);
-                umma_commit(&misc->slot_empty[slot]);
-            };
-            while (it.next()) {
+            while (lt < ntiles) {
+                mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
+                const SegDesc d = misc->seg[ls % kSegRing];
                 const int qb = ls & 1;
                 mbar_wait(&misc->q_full[qb], (ls >> 1) & 1);
-                for (int t = it.begin; t < it.end; ++t, ++lt) {
-                    const int seq = 2 * lt;
-                    const int slot = seq % NS;
-                    mbar_wait(&misc->slot_full[slot], (seq / NS) & 1);
+                for (int t = d.begin; t < d.end; ++t, ++lt) {
+                    const int slot = lt % NK;
+                    mbar_wait(&misc->k_full[slot], (lt / NK) & 1);
                     const int sb = lt & 1;
                     if (lt >= 2) mbar_wait(&misc->s_empty[sb], ((lt - 2) >> 1) & 1);
                     tc_fence_after();
-                    const uint32_t kbase = slots_addr + slot * kSlotBytes;
+                    SPI_TRACE(2);
+                    const uint32_t kbase = k_addr + slot * kSlotBytes;
                     const uint32_t qbase = q_addr + qb * Plan::kQBuf;
 #pragma unroll
                     for (int kk = 0; kk < kHeadDim / 16; ++kk) {
@@ -285,134 +360,162 @@ __global__ void __launch_bounds__(192, 1)
                         const uint32_t qoff = (kk >> 2) * (NT * 128) + (kk & 3) * 32;
                         const uint64_t adesc = make_smem_desc(kbase + koff, 16, 1024, kSw128);
                         const uint64_t bdesc = make_smem_desc(qbase + qoff, 16, 1024, kSw128);
-                        umma_bf16_ss(tm_S0 + sb * NT, adesc, bdesc, idesc_s, kk > 0 ? 1u : 0u);
+                        if (!(p.debug_flags & 2)) umma_bf16_ss(tm_S0 + sb * NT, adesc, bdesc, idesc_s, kk > 0 ? 1u : 0u);
                     }
                     umma_commit(&misc->s_full[sb]);
-                    umma_commit(&misc->slot_empty[slot]);
-                    if (t == it.end - 1) umma_commit(&misc->q_empty[qb]);
-                    if (lt >= 1) issue_pv(lt - 1, prev_first);
-                    prev_first = (t == it.begin);
+                    umma_commit(&misc->k_empty[slot]);
+                    if (t == d.end - 1) umma_commit(&misc->q_empty[qb]);
                 }
                 ++ls;
             }
-            if (lt >= 1) issue_pv(lt - 1, prev_first);
+        }
+    } else if (warp == 2) {
+        // ===================== PV issuer: O^T += V^T P^T per tile ==================
+        if (lane == 0) {
+            const uint32_t idesc_o = make_idesc_bf16(128, NT, true, true);
+            const uint32_t v_addr = smem_u32(s_v), p_addr = smem_u32(s_p);
+            int lt = 0, ls = 0;
+            while (lt < ntiles) {
+                mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
+                const SegDesc d = misc->seg[ls % kSegRing];
+                for (int t = d.begin; t < d.end; ++t, ++lt) {
+                    mbar_wait(&misc->p_full, lt & 1);
+                    const int slot = lt % NV;
+                    mbar_wait(&misc->v_full[slot], (lt / NV) & 1);
+                    tc_fence_after();
+                    SPI_TRACE(3);
+                    const uint32_t vbase = v_addr + slot * kSlotBytes;
+                    const bool first = (t == d.begin);
+#pragma unroll
+                    for (int kk = 0; kk < kKeyTile / 16; ++kk) {
+                        const uint64_t adesc = make_smem_desc(vbase + kk * 16 * 128, kHalfBytes, 1024, kSw128);
+                        const uint64_t bdesc = make_smem_desc(p_addr + kk * 16 * (NT * 2), Plan::kPBuf,
+                                                              8 * NT * 2, Plan::kPSwizzle);
+                        if (!(p.debug_flags & 2)) umma_bf16_ss(tm_O, adesc, bdesc, idesc_o, (first && kk == 0) ? 0u : 1u);
+                    }
+                    umma_commit(&misc->p_empty);
+                    umma_commit(&misc->v_empty[slot]);
+                }
+                ++ls;
+            }
         }
     } else {
         // ======================= softmax / epilogue warps =======================
-        const int st = threadIdx.x - 64;       // 0..127
+        const int st = threadIdx.x - 96;       // 0..127
         const int qd = warp & 3;               // TMEM lane quarter of this warp
         const int kt = qd * 32 + lane;         // key within tile (S^T lane) / head dim (O^T lane)
+        const int d = kt;
         const uint32_t lane_off = (uint32_t)(qd * 32) << 16;
-        int lt = 0;
-        while (it.next()) {
-            const int x = it.x;
-            const int c = x % p.chunks;
-            const int g = (x / p.chunks) % p.Hkv;
-            const int b = x / (p.chunks * p.Hkv);
-            const int P = p.prefix_len[b];
-            const int n = p.n_nodes[b];
+        int lt = 0, ls = 0;
+        while (lt < ntiles) {
+            mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
+            const SegDesc sd = misc->seg[ls % kSegRing];
+            const int b = sd.b, g = sd.g, c = sd.c, P = sd.P, n = sd.n;
             const int Kend = P + n;
             const int node0 = c * p.npc;
             const int G = p.G;
-            const int rc = G * p.npc;               // rows used in this chunk
-            // rows whose node exists
-            uint64_t row_valid = 0;
-            for (int r = 0; r < rc; ++r)
-                if (node0 + r / G < n) row_valid |= 1ull << r;
+            // prefetch the tree row masks this thread needs in this segment (<= 3 tiles carry
+            // tree keys): latency is hidden behind the prefix tiles
+            const int tt_tree0 = P / kKeyTile;  // first item tile holding a tree key
+            unsigned long long rm[3] = {0ull, 0ull, 0ull};
+#pragma unroll
+            for (int i = 0; i < 3; ++i) {
+                const int tt = tt_tree0 + i;
+                const int kk = tt * kKeyTile + kt;
+                if (tt >= sd.begin - sd.ib && tt < sd.end - sd.ib && kk >= P && kk < Kend)
+                    rm[i] = __ldg(p.rowmask + ((size_t)b * p.chunks + c) * p.Nmax + (kk - P));
+            }
             // reset row statistics
             if (qd == 0) {
-                for (int r = lane; r < NT; r += 32) misc->m_run[r] = -INFINITY;
+                for (int r = lane; r < NT; r += 32) {
+                    misc->m_thr[r] = -INFINITY;
+                    misc->m_ref[r] = 0.f;
+                }
             }
-            for (int r = lane; r < NT; r += 32) misc->l_part[qd][r] = 0.f;
+            float lsum[NT];
+#pragma unroll
+            for (int r = 0; r < NT; ++r) lsum[r] = 0.f;
             named_bar_sync(1, 128);
+            if (st == 0) SPI_TRACE(10);
 
-            for (int t = it.begin; t < it.end; ++t, ++lt) {
-                const int key0 = (t - it.ib) * kKeyTile;
-                const int kk = key0 + kt;
+            for (int t = sd.begin; t < sd.end; ++t, ++lt) {
+                const int tt = t - sd.ib;
+                const int kk = tt * kKeyTile + kt;
                 const int sb = lt & 1;
                 // ---- S^T row of this key ----
                 mbar_wait(&misc->s_full[sb], (lt >> 1) & 1);
                 tc_fence_after();
+                if (st == 0) SPI_TRACE(4);
                 float xv[NT];
                 {
-                    uint32_t r16[16];
+                    uint32_t r16[NT / 16][16];
 #pragma unroll
-                    for (int c16 = 0; c16 < NT / 16; ++c16) {
-                        tmem_ld16(tm_S0 + sb * NT + c16 * 16 + lane_off, r16);
-                        tmem_ld_wait();
+                    for (int c16 = 0; c16 < NT / 16; ++c16) tmem_ld16(tm_S0 + sb * NT + c16 * 16 + lane_off, r16[c16]);
+                    tmem_ld_wait();
 #pragma unroll
-                        for (int i = 0; i < 16; ++i) xv[c16 * 16 + i] = __uint_as_float(r16[i]);
-                    }
+                    for (int c16 = 0; c16 < NT / 16; ++c16)
+#pragma unroll
+                        for (int i = 0; i < 16; ++i) xv[c16 * 16 + i] = __uint_as_float(r16[c16][i]) * p.scale_log2;
                 }
                 tc_fence_before();
-                mbar_arrive(&misc->s_empty[sb]);
-                // ---- mask + scale ----
-                uint64_t vis;
-                if (kk < P) {
-                    vis = row_valid;
-                } else if (kk < Kend) {
-                    const int j = kk - P;
-                    const uint4 *dp = reinterpret_cast<const uint4 *>(p.desc + ((size_t)b * p.Nmax + j) * kBitWords);
-                    const uint4 d0 = __ldg(dp), d1 = __ldg(dp + 1);
-                    const uint32_t dw[8] = {d0.x, d0.y, d0.z, d0.w, d1.x, d1.y, d1.z, d1.w};
-                    uint64_t m = 0;
-                    for (int nd = 0; nd < p.npc; ++nd) {
-                        const int node = node0 + nd;
-                        if (node < kMaxNodes && ((dw[node >> 5] >> (node & 31)) & 1u)) {
-                            const uint64_t run = (G >= 64) ? ~0ull : ((1ull << G) - 1ull);
-                            m |= run << (nd * G);
-                        }
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&misc->s_empty[sb]);
+                // ---- mask: committed keys are visible to every row (padded rows are harmless:
+                // their Q rows are zero or belong to no output); tree keys use the row mask;
+                // keys past the request's end are invisible ----
+                if (kk >= P) {
+                    unsigned long long vis = 0ull;
+                    if (kk < Kend) {
+                        const int i = tt - tt_tree0;
+                        vis = i == 0 ? rm[0] : (i == 1 ? rm[1] : rm[2]);
                     }
-                    vis = m & row_valid;
-                } else {
-                    vis = 0;
-                }
 #pragma unroll
-                for (int r = 0; r < NT; ++r)
-                    xv[r] = ((vis >> r) & 1ull) ? xv[r] * p.scale_log2 : -INFINITY;
-                // ---- does this tile raise some row max beyond the stale tolerance? ----
+                    for (int r = 0; r < NT; ++r)
+                        if (!((vis >> r) & 1ull)) xv[r] = -INFINITY;
+                }
+                // ---- does this tile raise a row max beyond the stale tolerance? ----
                 bool need = false;
 #pragma unroll
                 for (int r = 0; r < NT; r += 4) {
-                    const float4 m4 = *reinterpret_cast<const float4 *>(&misc->m_run[r]);
-                    need |= xv[r] > m4.x + kRescaleThreshold;
-                    need |= xv[r + 1] > m4.y + kRescaleThreshold;
-                    need |= xv[r + 2] > m4.z + kRescaleThreshold;
-                    need |= xv[r + 3] > m4.w + kRescaleThreshold;
+                    const float4 m4 = *reinterpret_cast<const float4 *>(&misc->m_thr[r]);
+                    need |= (xv[r] > m4.x) | (xv[r + 1] > m4.y) | (xv[r + 2] > m4.z) | (xv[r + 3] > m4.w);
                 }
                 const unsigned ballot = __ballot_sync(0xffffffffu, need);
                 if (lane == 0) misc->flags[sb][qd] = ballot != 0u;
+                bulk_wait_read_all();  // output staging (P^T buffer) read by the bulk stores
                 named_bar_sync(1, 128);
                 const bool rescale = (misc->flags[sb][0] | misc->flags[sb][1] | misc->flags[sb][2] |
                                       misc->flags[sb][3]) != 0;
                 if (rescale) {
                     // exact tile max per row: transpose-reduce within the warp, combine 4 warps
-                    float mx[NT];
-#pragma unroll
-                    for (int r = 0; r < NT; ++r) mx[r] = xv[r];
 #pragma unroll
                     for (int blk = 0; blk < (NT + 31) / 32; ++blk) {
                         constexpr int W = NT < 32 ? NT : 32;
-                        transpose_reduce<W, true>(mx + blk * 32);
+                        float mx[W];
+#pragma unroll
+                        for (int r = 0; r < W; ++r) mx[r] = xv[blk * 32 + r];
+                        transpose_reduce<W, true>(mx);
                         const int row = blk * 32 + (lane & (W - 1));
-                        if (lane < W) misc->wred[qd][row] = mx[blk * 32];
+                        if (lane < W) misc->wred[qd][row] = mx[0];
                     }
                     named_bar_sync(1, 128);
                     if (qd == 0) {
                         for (int r = lane; r < NT; r += 32) {
-                            const float tm = fmaxf(fmaxf(misc->wred[0][r], misc->wred[1][r]),
-                                                   fmaxf(misc->wred[2][r], misc->wred[3][r]));
-                            const float mo = misc->m_run[r];
-                            const float mn = fmaxf(mo, tm);
+                            const float tmx = fmaxf(fmaxf(misc->wred[0][r], misc->wred[1][r]),
+                                                    fmaxf(misc->wred[2][r], misc->wred[3][r]));
+                            const float mo = misc->m_thr[r] - kRescaleThreshold;  // -inf stays -inf
+                            const float mn = fmaxf(mo, tmx);
                             misc->alpha[r] = (mo == -INFINITY) ? 0.f : ex2(mo - mn);
-                            misc->m_run[r] = mn;
+                            misc->m_thr[r] = mn + kRescaleThreshold;
+                            misc->m_ref[r] = (mn == -INFINITY) ? 0.f : mn;
                         }
                     }
                     named_bar_sync(1, 128);
-                    for (int r = lane; r < NT; r += 32) misc->l_part[qd][r] *= misc->alpha[r];
-                    if (t != it.begin) {
-                        // O^T columns (rows of Q) scaled by alpha: wait for PV of tile lt-1
-                        mbar_wait(&misc->p_empty[(lt - 1) & 1], ((lt - 1) >> 1) & 1);
+#pragma unroll
+                    for (int r = 0; r < NT; ++r) lsum[r] *= misc->alpha[r];
+                    if (t != sd.begin) {
+                        // O^T columns (query rows) scaled by alpha: wait for PV of tile lt-1
+                        mbar_wait(&misc->p_empty, (lt - 1) & 1);
                         tc_fence_after();
                         uint32_t r16[16];
 #pragma unroll
@@ -427,154 +530,226 @@ __global__ void __launch_bounds__(192, 1)
                         tmem_st_wait();
                     }
                 }
-                // ---- probabilities (bf16) ----
+                // ---- probabilities, row sums ----
 #pragma unroll
                 for (int r = 0; r < NT; r += 4) {
-                    const float4 m4 = *reinterpret_cast<const float4 *>(&misc->m_run[r]);
-                    const float mr[4] = {m4.x, m4.y, m4.z, m4.w};
-#pragma unroll
-                    for (int i = 0; i < 4; ++i) {
-                        const float ref = (mr[i] == -INFINITY) ? 0.f : mr[i];
-                        const float e = ex2(xv[r + i] - ref);
-                        xv[r + i] = __bfloat162float(__float2bfloat16_rn(e));
-                    }
+                    const float4 m4 = *reinterpret_cast<const float4 *>(&misc->m_ref[r]);
+                    xv[r] = ex2(xv[r] - m4.x);
+                    xv[r + 1] = ex2(xv[r + 1] - m4.y);
+                    xv[r + 2] = ex2(xv[r + 2] - m4.z);
+                    xv[r + 3] = ex2(xv[r + 3] - m4.w);
                 }
-                // V rows of keys beyond the request's last key must be finite zeros (0 * NaN)
-                if (kk >= Kend) {
-                    const int seq = 2 * lt + 1;
-                    const int slot = seq % NS;
-                    mbar_wait(&misc->slot_full[slot], (seq / NS) & 1);
-                    uint4 *v0 = reinterpret_cast<uint4 *>(s_slots + (size_t)slot * kSlotBytes + kt * 128);
-                    uint4 *v1 = reinterpret_cast<uint4 *>(s_slots + (size_t)slot * kSlotBytes + kHalfBytes + kt * 128);
+                // P rounded to bf16 once; the row sums use the rounded values so that the
+                // normalisation matches the numerator the PV MMA computes
+                uint32_t pk[NT / 2];
 #pragma unroll
-                    for (int i = 0; i < 8; ++i) {
-                        v0[i] = make_uint4(0, 0, 0, 0);
-                        v1[i] = make_uint4(0, 0, 0, 0);
-                    }
+                for (int i = 0; i < NT / 2; ++i) {
+                    pk[i] = pack_bf16x2(xv[2 * i], xv[2 * i + 1]);
+                    lsum[2 * i] += __uint_as_float(pk[i] << 16);
+                    lsum[2 * i + 1] += __uint_as_float(pk[i] & 0xFFFF0000u);
                 }
-                // ---- P^T row (this key) into smem, MN-major + swizzle ----
-                if (lt >= 2) mbar_wait(&misc->p_empty[sb], ((lt - 2) >> 1) & 1);
+                // ---- P^T row (this key) into smem as bf16, MN-major + swizzle ----
+                if (lt >= 1) mbar_wait(&misc->p_empty, (lt - 1) & 1);  // PV(t-1) has read P^T
                 {
-                    uint8_t *pb = s_p + sb * Plan::kPBuf;
+                    uint8_t *pb = s_p;
 #pragma unroll
                     for (int c8 = 0; c8 < NT / 8; ++c8) {
                         const uint32_t o = (uint32_t)kt * (NT * 2) + c8 * 16;
                         const uint32_t phys = o ^ (((o >> 7) & Plan::kPMask) << 4);
-                        uint4 v;
-                        v.x = pack_bf16x2(xv[c8 * 8 + 0], xv[c8 * 8 + 1]);
-                        v.y = pack_bf16x2(xv[c8 * 8 + 2], xv[c8 * 8 + 3]);
-                        v.z = pack_bf16x2(xv[c8 * 8 + 4], xv[c8 * 8 + 5]);
-                        v.w = pack_bf16x2(xv[c8 * 8 + 6], xv[c8 * 8 + 7]);
-                        *reinterpret_cast<uint4 *>(pb + phys) = v;
+                        *reinterpret_cast<uint4 *>(pb + phys) =
+                            make_uint4(pk[c8 * 4], pk[c8 * 4 + 1], pk[c8 * 4 + 2], pk[c8 * 4 + 3]);
                     }
                 }
                 fence_proxy_async_smem();
                 tc_fence_before();
                 __syncwarp();
-                if (lane == 0) mbar_arrive(&misc->p_full[sb]);
-                // ---- row sums of this tile (in key order over the 4 warps) ----
-#pragma unroll
-                for (int blk = 0; blk < (NT + 31) / 32; ++blk) {
-                    constexpr int W = NT < 32 ? NT : 32;
-                    transpose_reduce<W, false>(xv + blk * 32);
-                    const int row = blk * 32 + (lane & (W - 1));
-                    if (lane < W) misc->l_part[qd][row] += xv[blk * 32];
-                }
+                if (lane == 0) mbar_arrive(&misc->p_full);
+                if (st == 0) SPI_TRACE(5);
 
-                if (t == it.end - 1) {
+                if (t == sd.end - 1) {
                     // ============ epilogue of this segment ============
-                    mbar_wait(&misc->p_empty[sb], (lt >> 1) & 1);  // last PV done
+                    // row sums over the 128 keys of every tile: reduce the per-thread partials
+#pragma unroll
+                    for (int blk = 0; blk < (NT + 31) / 32; ++blk) {
+                        constexpr int W = NT < 32 ? NT : 32;
+                        transpose_reduce<W, false>(lsum + blk * 32);
+                        const int row = blk * 32 + (lane & (W - 1));
+                        if (lane < W) misc->l_part[qd][row] = lsum[blk * 32];
+                    }
+                    mbar_wait(&misc->p_empty, lt & 1);  // last PV done
                     tc_fence_after();
+                    if (st == 0) SPI_TRACE(6);
                     float o[NT];
                     {
-                        uint32_t r16[16];
+                        uint32_t r16[NT / 16][16];
 #pragma unroll
-                        for (int c16 = 0; c16 < NT / 16; ++c16) {
-                            tmem_ld16(tm_O + c16 * 16 + lane_off, r16);
-                            tmem_ld_wait();
+                        for (int c16 = 0; c16 < NT / 16; ++c16) tmem_ld16(tm_O + c16 * 16 + lane_off, r16[c16]);
+                        tmem_ld_wait();
 #pragma unroll
-                            for (int i = 0; i < 16; ++i) o[c16 * 16 + i] = __uint_as_float(r16[i]);
-                        }
+                        for (int c16 = 0; c16 < NT / 16; ++c16)
+#pragma unroll
+                            for (int i = 0; i < 16; ++i) o[c16 * 16 + i] = __uint_as_float(r16[c16][i]);
                     }
                     tc_fence_before();
-                    named_bar_sync(1, 128);  // all l_part updates visible
-                    const int d = kt;
-                    const bool full = (it.begin == it.ib) && (it.end == it.ie);
+                    named_bar_sync(1, 128);  // all l_part visible
+                    if (st < NT) {
+                        const float l = misc->l_part[0][st] + misc->l_part[1][st] + misc->l_part[2][st] + misc->l_part[3][st];
+                        misc->run_l[st] = l;           // row sum of this segment
+                        misc->alpha[st] = 1.0f / l;    // its reciprocal (inf for rows with no key)
+                    }
+                    named_bar_sync(1, 128);
+                    if (st == 0) SPI_TRACE(9);
+                    const bool full = (sd.begin == sd.ib) && (sd.end == sd.ie);
+                    const int rc = G * p.npc;
                     if (full) {
+                        // stage the bf16 rows in the idle P^T buffer (row r at r*256 B, rows of a
+                        // node contiguous) and write each node's G rows with one bulk async copy
+                        __nv_bfloat16 *stg = reinterpret_cast<__nv_bfloat16 *>(s_p);
 #pragma unroll
-                        for (int r = 0; r < NT; ++r) {
-                            if (!((row_valid >> r) & 1ull)) continue;
-                            const float l = misc->l_part[0][r] + misc->l_part[1][r] + misc->l_part[2][r] + misc->l_part[3][r];
-                            const int node = node0 + r / G, hl = r % G;
-                            p.out[(((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim + d] =
-                                __float2bfloat16_rn(o[r] / l);
+                        for (int r = 0; r < NT; r += 4) {
+                            const float4 inv = *reinterpret_cast<const float4 *>(&misc->alpha[r]);
+                            stg[(r + 0) * kHeadDim + d] = __float2bfloat16_rn(o[r + 0] * inv.x);
+                            stg[(r + 1) * kHeadDim + d] = __float2bfloat16_rn(o[r + 1] * inv.y);
+                            stg[(r + 2) * kHeadDim + d] = __float2bfloat16_rn(o[r + 2] * inv.z);
+                            stg[(r + 3) * kHeadDim + d] = __float2bfloat16_rn(o[r + 3] * inv.w);
                         }
+                        fence_proxy_async_smem();
+                        named_bar_sync(1, 128);
+                        const int nodes_here = min(p.npc, n - node0);
+                        if (st < nodes_here) {
+                            bulk_store_s2g(p.out + (((size_t)b * p.Nmax + node0 + st) * p.Hq + g * G) * kHeadDim,
+                                           s_p + st * G * kHeadDim * 2, (uint32_t)(G * kHeadDim * 2));
+                            bulk_commit();
+                        }
+                        if (st == 0) SPI_TRACE(8);
                     } else {
-                        const int slot = (it.begin == t0) ? 0 : 1;
+                        const int slot = (sd.begin == t0) ? 0 : 1;
                         float *po = p.part_o + (((size_t)blockIdx.x * 2 + slot) * NT) * kHeadDim;
 #pragma unroll
                         for (int r = 0; r < NT; ++r) po[(size_t)r * kHeadDim + d] = o[r];
                         float *pml = p.part_ml + ((size_t)blockIdx.x * 2 + slot) * 2 * NT;
                         if (st < NT) {
-                            pml[st] = misc->m_run[st];
-                            pml[NT + st] = misc->l_part[0][st] + misc->l_part[1][st] + misc->l_part[2][st] + misc->l_part[3][st];
+                            const float mt = misc->m_thr[st];
+                            pml[st] = mt == -INFINITY ? -INFINITY : mt - kRescaleThreshold;
+                            pml[NT + st] = misc->run_l[st];
                         }
                         __threadfence();
                         named_bar_sync(1, 128);
                         if (st == 0) {
-                            const int c_first = cta_of_tile(it.ib, T, NC);
-                            const int c_last = cta_of_tile(it.ie - 1, T, NC);
+                            const int c_first = cta_of_tile(sd.ib, T, NC);
+                            const int c_last = cta_of_tile(sd.ie - 1, T, NC);
                             int npieces = 0;
                             for (int cc = c_first; cc <= c_last; ++cc)
                                 npieces += cta_start(cc + 1, T, NC) > cta_start(cc, T, NC);
-                            const unsigned old = atomicAdd(&p.item_cnt[x], 1u);
+                            const unsigned old = atomicAdd(&p.item_cnt[sd.x], 1u);
                             misc->bcast = (old == (unsigned)(npieces - 1)) ? 1 : 0;
-                            if (misc->bcast) p.item_cnt[x] = 0u;  // ready for the next launch
+                            if (misc->bcast) p.item_cnt[sd.x] = 0u;  // ready for the next launch
                         }
                         named_bar_sync(1, 128);
                         if (misc->bcast) {
+                            // last piece: merge all pieces' (m, l, O) by log-sum-exp, pieces staged
+                            // kCombineBatch at a time so every global load of a batch is in flight
                             __threadfence();
-                            const int c_first = cta_of_tile(it.ib, T, NC);
-                            const int c_last = cta_of_tile(it.ie - 1, T, NC);
+                            if (st < NT) {
+                                misc->run_m[st] = -INFINITY;
+                                misc->run_l[st] = 0.f;
+                            }
+                            float acc[NT];
+#pragma unroll
+                            for (int r = 0; r < NT; ++r) acc[r] = 0.f;
+                            // the P^T buffer is idle during an epilogue (last PV done, next P not yet written)
+                            float *cmb_m = reinterpret_cast<float *>(s_p);
+                            float *cmb_l = cmb_m + kCombineBatch * NT;
+                            float *cmb_w = cmb_l + kCombineBatch * NT;
+                            int cc = 0, c_last = 0;
+                            if (st == 0) {
+                                cc = cta_of_tile(sd.ib, T, NC);
+                                c_last = cta_of_tile(sd.ie - 1, T, NC);
+                            }
+                            for (;;) {
+                                named_bar_sync(1, 128);
+                                if (st == 0) {
+                                    int nb = 0;
+                                    while (cc <= c_last && nb < kCombineBatch) {
+                                        const int s0 = cta_start(cc, T, NC);
+                                        if (cta_start(cc + 1, T, NC) > s0) {
+                                            misc->piece_off[nb] = ((size_t)cc * 2 + ((s0 >= sd.ib) ? 0 : 1));
+                                            ++nb;
+                                        }
+                                        ++cc;
+                                    }
+                                    misc->bcast = nb;
+                                }
+                                named_bar_sync(1, 128);
+                                const int nb = misc->bcast;
+                                if (nb == 0) break;
+                                for (int idx = st; idx < nb * NT; idx += 128) {
+                                    const int pc = idx / NT, r = idx - pc * NT;
+                                    const float *pm = p.part_ml + misc->piece_off[pc] * 2 * NT;
+                                    cmb_m[pc * NT + r] = ldcg_f32(pm + r);
+                                    cmb_l[pc * NT + r] = ldcg_f32(pm + NT + r);
+                                }
+                                named_bar_sync(1, 128);
+                                if (st < NT) {
+                                    const int r = st;
+                                    float bm = -INFINITY;
+                                    for (int pc = 0; pc < nb; ++pc) bm = fmaxf(bm, cmb_m[pc * NT + r]);
+                                    const float mo = misc->run_m[r];
+                                    const float mn = fmaxf(mo, bm);
+                                    const float sc = (mo == -INFINITY) ? 0.f : ex2(mo - mn);
+                                    float L = misc->run_l[r] * sc;
+                                    for (int pc = 0; pc < nb; ++pc) {
+                                        const float mp = cmb_m[pc * NT + r];
+                                        const float w = (mp == -INFINITY) ? 0.f : ex2(mp - mn);
+                                        cmb_w[pc * NT + r] = w;
+                                        L += w * cmb_l[pc * NT + r];
+                                    }
+                                    misc->run_m[r] = mn;
+                                    misc->run_l[r] = L;
+                                    misc->alpha[r] = sc;
+                                }
+                                named_bar_sync(1, 128);
+#pragma unroll
+                                for (int r = 0; r < NT; ++r) acc[r] *= misc->alpha[r];
+                                for (int pc = 0; pc < nb; ++pc) {
+                                    const float *po2 = p.part_o + misc->piece_off[pc] * NT * kHeadDim + d;
+                                    float v[NT];
+#pragma unroll
+                                    for (int r = 0; r < NT; ++r) v[r] = ldcg_f32(po2 + (size_t)r * kHeadDim);
+#pragma unroll
+                                    for (int r = 0; r < NT; ++r) acc[r] += cmb_w[pc * NT + r] * v[r];
+                                }
+                            }
+                            int node = node0, hl = 0;
+#pragma unroll
                             for (int r = 0; r < NT; ++r) {
-                                if (!((row_valid >> r) & 1ull)) continue;
-                                float M = -INFINITY;
-                                for (int cc = c_first; cc <= c_last; ++cc) {
-                                    const int s0 = cta_start(cc, T, NC);
-                                    if (cta_start(cc + 1, T, NC) <= s0) continue;
-                                    const int sl = (s0 >= it.ib) ? 0 : 1;
-                                    M = fmaxf(M, ldcg_f32(p.part_ml + ((size_t)cc * 2 + sl) * 2 * NT + r));
+                                if (r < rc && node < n) {
+                                    p.out[(((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim + d] =
+                                        __float2bfloat16_rn(__fdividef(acc[r], misc->run_l[r]));
                                 }
-                                float L = 0.f, O = 0.f;
-                                for (int cc = c_first; cc <= c_last; ++cc) {
-                                    const int s0 = cta_start(cc, T, NC);
-                                    if (cta_start(cc + 1, T, NC) <= s0) continue;
-                                    const int sl = (s0 >= it.ib) ? 0 : 1;
-                                    const float *pm = p.part_ml + ((size_t)cc * 2 + sl) * 2 * NT;
-                                    const float mp = ldcg_f32(pm + r);
-                                    if (mp == -INFINITY) continue;
-                                    const float w = ex2(mp - M);
-                                    L += w * ldcg_f32(pm + NT + r);
-                                    O += w * ldcg_f32(p.part_o + (((size_t)cc * 2 + sl) * NT + r) * kHeadDim + d);
+                                if (++hl == G) {
+                                    hl = 0;
+                                    ++node;
                                 }
-                                const int node = node0 + r / G, hl = r % G;
-                                p.out[(((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim + d] =
-                                    __float2bfloat16_rn(O / L);
                             }
                         }
                     }
                     named_bar_sync(1, 128);  // stats read by everyone before the next reset
+                    if (st == 0) SPI_TRACE(7);
                 }
             }
+            ++ls;
         }
     }
 
+    if (warp >= 3) bulk_wait_all();  // output bulk stores complete before smem goes away
     tc_fence_before();
     __syncthreads();
     if (warp == 1) {
         tc_fence_after();
         tmem_dealloc<Plan::kTmemCols>(tmem);
     }
+    if (threadIdx.x == 0) SPI_TRACE_K(1);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -624,28 +799,28 @@ static bool encode_q(CUtensorMap *m, const void *base, int Hq, uint64_t nodes, i
 template <int NT>
 static size_t attn_smem_bytes(int num_slots) {
     using Plan = SmemPlan<NT>;
-    return 1024 + (size_t)num_slots * kSlotBytes + 2 * Plan::kQBuf + 2 * Plan::kPBuf + sizeof(SmemMisc);
-}
-
-template <int NT>
-static int pick_slots(size_t max_smem) {
-    int ns = 16;
-    while (ns > 2 && attn_smem_bytes<NT>(ns) > max_smem) --ns;
-    return ns;
+    static_assert(3 * kCombineBatch * NT * 4 <= Plan::kPBuf, "combine staging must fit the P buffer");
+    return 1024 + (size_t)num_slots * kSlotBytes + 2 * Plan::kQBuf + Plan::kPBuf + sizeof(SmemMisc);
 }
 
 template <int NT>
 static cudaError_t launch_nt(const AttnParams &prm0, const void *q, const void *k, const void *v,
                              int num_sms, size_t max_smem, cudaStream_t stream) {
     AttnParams prm = prm0;
-    CUtensorMap tq, tk, tv, tk16, tv16;
+    CUtensorMap tq, tk, tv, tk16, tv16, tk4, tv4, tk1, tv1;
     const uint64_t rows = (uint64_t)prm.B * prm.Hkv * prm.Smax;
     if (!encode_q(&tq, q, prm.Hq, (uint64_t)prm.B * prm.Nmax, prm.G, prm.npc) ||
         !encode_2d(&tk, k, rows, kKeyTile) || !encode_2d(&tv, v, rows, kKeyTile) ||
-        !encode_2d(&tk16, k, rows, kTailRows) || !encode_2d(&tv16, v, rows, kTailRows))
+        !encode_2d(&tk16, k, rows, 16) || !encode_2d(&tv16, v, rows, 16) || !encode_2d(&tk4, k, rows, 4) ||
+        !encode_2d(&tv4, v, rows, 4) || !encode_2d(&tk1, k, rows, 1) || !encode_2d(&tv1, v, rows, 1))
         return cudaErrorInvalidValue;
-    prm.num_slots = pick_slots<NT>(max_smem);
-    const size_t smem = attn_smem_bytes<NT>(prm.num_slots);
+    int ns = 2 * kMaxSlots;
+    while (ns > 2 && attn_smem_bytes<NT>(ns) > max_smem) --ns;
+    // K tiles are released right after S = K Q^T; V tiles are held until PV: give V the extra slot
+    ns = min(ns, 6);
+    prm.nk_slots = ns / 2;
+    prm.nv_slots = ns - ns / 2;
+    const size_t smem = attn_smem_bytes<NT>(ns);
     static bool attr_set = false;
     if (!attr_set) {
         cudaError_t e = cudaFuncSetAttribute(tree_attn_kernel<NT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -653,9 +828,23 @@ static cudaError_t launch_nt(const AttnParams &prm0, const void *q, const void *
         if (e != cudaSuccess) return e;
         attr_set = true;
     }
-    tree_attn_kernel<NT><<<num_sms, 192, smem, stream>>>(tq, tk, tv, tk16, tv16, prm);
-    return cudaGetLastError();
+    // programmatic dependent launch: the prologue (barrier init, TMEM alloc, smem zeroing) of
+    // this grid overlaps the tail of the previous kernel on the stream
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(num_sms);
+    cfg.blockDim = dim3(224);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = stream;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, tree_attn_kernel<NT>, tq, tk, tv, tk16, tv16, tk4, tv4, tk1, tv1, prm);
 }
+
+unsigned long long *g_attn_trace = nullptr;  // debug only (specinfer_debug_set_trace)
+int g_attn_debug_flags = 0;                   // debug only (SPECINFER_DEBUG_FLAGS, experiments)
 
 cudaError_t launch_tree_attention(const specinfer_shape_t &s, const WsLayout &w, const void *q,
                                   const void *k, const void *v, const int32_t *prefix_len,
@@ -666,7 +855,9 @@ cudaError_t launch_tree_attention(const specinfer_shape_t &s, const WsLayout &w,
     prm.n_nodes = n_nodes;
     prm.item_start = reinterpret_cast<const int32_t *>(ws + w.item_start);
     prm.item_cnt = reinterpret_cast<uint32_t *>(ws + w.item_cnt);
-    prm.desc = reinterpret_cast<const uint32_t *>(ws + w.desc);
+    prm.item_info = reinterpret_cast<const int4 *>(ws + w.item_info);
+    prm.cta_info = reinterpret_cast<const int4 *>(ws + w.cta_info);
+    prm.rowmask = reinterpret_cast<const unsigned long long *>(ws + w.rowmask);
     prm.part_o = reinterpret_cast<float *>(ws + w.part_o);
     prm.part_ml = reinterpret_cast<float *>(ws + w.part_ml);
     prm.out = reinterpret_cast<__nv_bfloat16 *>(out);
@@ -681,6 +872,8 @@ cudaError_t launch_tree_attention(const specinfer_shape_t &s, const WsLayout &w,
     prm.n_items = w.n_items;
     const float sm_scale = s.sm_scale > 0.f ? s.sm_scale : 1.0f / sqrtf((float)s.head_dim);
     prm.scale_log2 = sm_scale * 1.4426950408889634f;
+    prm.trace = g_attn_trace;
+    prm.debug_flags = g_attn_debug_flags;
     const int grid = num_sms;  // persistent: one CTA per SM
     switch (w.nt) {
         case 16: return launch_nt<16>(prm, q, k, v, grid, max_smem, stream);
