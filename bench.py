@@ -216,13 +216,14 @@ def run_ours(args, ws, rank, local):
         ("mss" in wl.verify) * spi.specinfer_launches_per_call("verify_mss") +
         spi.specinfer_launches_per_call("kv_commit"))
 
+    from paper_conf_asplos_miaoozcwzwzyssc24_b200 import dist as D
+
     def gather():
+        # a7: the tokens-only exchange after verification, NCCL over NVLink
         if ws > 1:
-            src_n, src_a = (na, at) if "greedy" in wl.verify else (na2, at2)
-            gather_in[:, 0] = src_n
-            gather_in[:, 1:1 + Lp] = src_a
-            gather_in[:, 1 + Lp:] = (an if "greedy" in wl.verify else an2)
-            torch.distributed.all_gather_into_tensor(gather_out, gather_in)
+            src = (na, at, an) if "greedy" in wl.verify else (na2, at2, an2)
+            gather_in.copy_(D.pack_accepted(*src))
+            D.gather_accepted(gather_in, gather_out)
 
     # ---- capture the three segments as CUDA graphs (one launch each per step) ----
     s = torch.cuda.Stream(device)

@@ -31,6 +31,7 @@ cudaError_t launch_kv_commit(const specinfer_shape_t &s, void *k_all, void *v_al
 cudaError_t launch_philox_debug(const uint32_t *ck, uint32_t *out, int n, cudaStream_t stream);
 extern unsigned long long *g_attn_trace;
 extern int g_attn_debug_flags;
+extern unsigned long long *g_mss_trace;
 }  // namespace specinfer
 
 using namespace specinfer;
@@ -220,6 +221,8 @@ specinfer_status_t specinfer_philox_debug(const uint32_t *ctr_key, uint32_t *out
 
 void specinfer_debug_set_trace(void *trace) {
     g_attn_trace = reinterpret_cast<unsigned long long *>(trace);
+    g_mss_trace = getenv("SPECINFER_TRACE_MSS") ? reinterpret_cast<unsigned long long *>(trace) : nullptr;
+    if (g_mss_trace) g_attn_trace = nullptr;
     // experiment switches for pipeline studies (results invalid when set); never set in production
     const char *f = getenv("SPECINFER_DEBUG_FLAGS");
     g_attn_debug_flags = f ? atoi(f) : 0;

@@ -152,7 +152,7 @@ __global__ void __launch_bounds__(1024) schedule_kernel(
         status[1] = run;
         s_total = run;
     }
-    for (int b = threadIdx.x; b < B; b += blockDim.x) verify_cnt[b] = 0u;
+    for (int b = threadIdx.x; b < 2 * B; b += blockDim.x) verify_cnt[b] = 0u;
     __syncthreads();
     // per-CTA slice [t0, t1) of the tile sequence for the attention grid, and its first item
     const long long T = s_total;

@@ -1,0 +1,55 @@
+"""Multi-GPU plumbing of the verification step.
+
+The hot path partitions by request: every (request, kv-head) is independent for tree attention and
+KV commit, every request for verification.  Ranks own disjoint request ranges; the only exchange is
+the tokens-only gather after verification (the request manager and GPU workers
+"only communicate tokens").  MSS counters use global request ids, so results are identical at any
+world size.  NCCL (over NVLink/NVSwitch) on GPUs; gloo is accepted for the CPU tests.
+"""
+from __future__ import annotations
+
+from typing import Tuple
+
+import torch
+
+
+def shard_requests(batch_global: int, world: int, rank: int) -> Tuple[int, int]:
+    """Contiguous request range [start, start + count) of `rank` (strong scaling split)."""
+    base, rem = divmod(batch_global, world)
+    start = rank * base + min(rank, rem)
+    return start, base + (1 if rank < rem else 0)
+
+
+def global_request_ids(start: int, count: int, device) -> torch.Tensor:
+    return torch.arange(start, start + count, dtype=torch.int32, device=device)
+
+
+def pack_accepted(n_accepted: torch.Tensor, accepted_tokens: torch.Tensor,
+                  accepted_nodes: torch.Tensor) -> torch.Tensor:
+    """int32 [B][2 Lp + 1] = [n | tokens | nodes] (one contiguous row per request)."""
+    B, Lp = accepted_tokens.shape
+    out = torch.empty((B, 2 * Lp + 1), dtype=torch.int32, device=accepted_tokens.device)
+    out[:, 0] = n_accepted
+    out[:, 1:1 + Lp] = accepted_tokens
+    out[:, 1 + Lp:] = accepted_nodes
+    return out
+
+
+def unpack_accepted(buf: torch.Tensor):
+    Lp = (buf.shape[1] - 1) // 2
+    return buf[:, 0], buf[:, 1:1 + Lp], buf[:, 1 + Lp:]
+
+
+def gather_accepted(packed: torch.Tensor, out: torch.Tensor = None) -> torch.Tensor:
+    """All-gather the per-rank packed rows (equal request counts per rank) into [world·B][2Lp+1]."""
+    world = torch.distributed.get_world_size()
+    if out is None:
+        out = torch.empty((world * packed.shape[0], packed.shape[1]), dtype=packed.dtype, device=packed.device)
+    if torch.distributed.get_backend() == "nccl":
+        torch.distributed.all_gather_into_tensor(out, packed)
+    else:
+        parts = list(out.chunk(world, dim=0))
+        torch.distributed.all_gather(parts, packed)
+        if parts[0].data_ptr() != out.data_ptr():
+            out.copy_(torch.cat(parts, 0))
+    return out

@@ -1,0 +1,81 @@
+"""World-size-2 gloo test of the multi-GPU host logic (request sharding, global request ids, the
+tokens-only all-gather).  The per-rank "device" work is the oracle, so this runs on CPU; the
+invariant checked is that the gathered results equal a single-process run on the whole batch
+(integer outputs bit-identical across world sizes)."""
+import os
+import socket
+
+import numpy as np
+import torch
+import torch.multiprocessing as mp
+
+import oracle
+import workloads as W
+from paper_conf_asplos_miaoozcwzwzyssc24_b200 import dist as D
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _inputs():
+    rng = np.random.default_rng(0)
+    B, N, V = 10, 24, 40
+    trees = [W.random_tree(int(rng.integers(1, N + 1)), 8, 4, rng) for _ in range(B)]
+    tb = W.make_tree_batch(trees, [3] * B, max_nodes=N, max_depth=8)
+    vi = W.make_verify_inputs(tb, V, seed=3, mode="mss")
+    return tb, vi
+
+
+def _verify(tb, vi, lo, cnt):
+    sl = slice(lo, lo + cnt)
+    an, at, na, _ = oracle.verify_mss(vi.logits[sl].numpy(), vi.tree_tokens[sl].numpy(), tb.parent[sl].numpy(),
+                                      tb.n_nodes[sl].numpy(), vi.draft_probs[sl].numpy(), seed=9, offset=2,
+                                      request_ids=np.arange(lo, lo + cnt, dtype=np.int32), path_len=9)
+    return torch.from_numpy(na), torch.from_numpy(at), torch.from_numpy(an)
+
+
+def _worker(rank, world, port, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    torch.distributed.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        tb, vi = _inputs()
+        B = tb.parent.shape[0]
+        lo, cnt = D.shard_requests(B, world, rank)
+        assert cnt == B // world  # equal shards for the gather
+        na, at, an = _verify(tb, vi, lo, cnt)
+        packed = D.pack_accepted(na, at, an)
+        gathered = D.gather_accepted(packed)
+        if rank == 0:
+            q.put(gathered.numpy())
+    finally:
+        torch.distributed.destroy_process_group()
+
+
+def test_sharding_math():
+    assert D.shard_requests(10, 3, 0) == (0, 4)
+    assert D.shard_requests(10, 3, 1) == (4, 3)
+    assert D.shard_requests(10, 3, 2) == (7, 3)
+    assert sum(D.shard_requests(17, 4, r)[1] for r in range(4)) == 17
+
+
+def test_two_rank_gather_equals_single_process():
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    gathered = q.get(timeout=120)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    tb, vi = _inputs()
+    na, at, an = _verify(tb, vi, 0, tb.parent.shape[0])
+    ref = D.pack_accepted(na, at, an).numpy()
+    assert np.array_equal(gathered, ref)
