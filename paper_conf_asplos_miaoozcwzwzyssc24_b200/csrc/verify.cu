@@ -250,14 +250,16 @@ __global__ void __launch_bounds__(kGreedyThreads) verify_greedy_kernel(
 }
 
 // ------------------------------------------------------------------------------------------
-// K5 verify_mss
+// K5 verify_mss: one thread-block cluster per request walks Alg. 2; every V-wide pass (softmax
+// statistics, residual, exponential race) is split over the cluster's CTAs and reduced through
+// distributed shared memory, so a pass costs ~1/CS of a single SM's time.
+// Arithmetic: V-wide work runs on the MUFU fast path in base 2 (ex2/lg2/rcp .approx, relative
+// error ~1e-7); the fp64 oracle differs only at decisions whose margin is below that
+// (boundary-excused in the parity tests).  p_k = 2^(l_k c - m c) / z, c = log2(e)/T.
 // ------------------------------------------------------------------------------------------
-// Arithmetic: everything V-wide runs on the MUFU fast path in base 2 (ex2/lg2/rcp .approx,
-// relative error ~1e-7); the fp64 oracle differs only at decisions whose margin is below that
-// (boundary-excused in the parity tests).  p_k = 2^(l_k c - m c) / z with
-// c = log2(e) / T.
-constexpr int kMssThreads = 512;
+constexpr int kMssThreads = 256;
 constexpr int kMssUnroll = 4;
+constexpr int kMssCluster = 8;
 
 __device__ __forceinline__ float lg2f(float x) {
     float y;
@@ -269,6 +271,34 @@ __device__ __forceinline__ float rcpf(float x) {
     asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
     return y;
 }
+__device__ __forceinline__ uint32_t cluster_ctarank() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
+__device__ __forceinline__ uint32_t cluster_nctarank() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_nctarank;" : "=r"(r));
+    return r;
+}
+__device__ __forceinline__ void cluster_sync_all() {
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+__device__ __forceinline__ uint32_t map_to_rank(const void *p, uint32_t rank) {
+    uint32_t r;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(smem_u32(p)), "r"(rank));
+    return r;
+}
+__device__ __forceinline__ float ld_dsmem_f32(uint32_t a) {
+    float v;
+    asm volatile("ld.shared::cluster.f32 %0, [%1];" : "=f"(v) : "r"(a) : "memory");
+    return v;
+}
+__device__ __forceinline__ int ld_dsmem_s32(uint32_t a) {
+    int v;
+    asm volatile("ld.shared::cluster.s32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+    return v;
+}
 
 // E'_k = -log2 U_k = E_k / ln 2 with U_k = ((w >> 9) + 0.5) 2^-23 (c4 step 4); the race argmax of
 // p_k / E_k equals that of p_k / E'_k and of log2 p_k - log2 E'_k.
@@ -277,25 +307,84 @@ __device__ __forceinline__ float race_E2(uint32_t w) {
     return -lg2f(U);
 }
 
-struct MssState {
-    int mode;      // 0: p = 2^(l c - mc) * invZ (softmax of node u); 1: p = buf[cur] * inv
-    int cur;       // which residual buffer holds p (mode 1)
-    float mc;      // max logit * c (mode 0)
-    float invZ;    // 1 / sum_k 2^(l_k c - mc) (mode 0)
-    float inv;     // 1 / sum of the residual buffer (mode 1)
+// Per-CTA partial results exchanged through DSMEM (double-buffered by reduction parity).
+struct MssPart {
+    float a, b;  // (max, sum) pair or (sum, -)
+    float v;     // race key
+    int i;       // race index
 };
 
-__device__ __forceinline__ float mss_p(const MssState &s, const float *lrow, const float *buf, float c, int k) {
-    return s.mode == 0 ? ex2(fmaf(__ldcg(lrow + k), c, -s.mc)) * s.invZ : __ldcg(buf + k) * s.inv;
+struct MssCluster {
+    MssPart *slot;    // smem [2], this CTA's contribution per reduction parity
+    MssPart *result;  // smem [1], the merged value broadcast to the CTA
+    uint32_t rank, size;
+    int parity;
+    // every CTA contributes `mine` (already reduced over the block); returns the merged result
+    // identically on every CTA.  Warp 0 gathers the cluster's slots through DSMEM.
+    template <class Merge>
+    __device__ MssPart reduce(const MssPart &mine, Merge merge) {
+        if (threadIdx.x == 0) slot[parity] = mine;
+        cluster_sync_all();
+        if (threadIdx.x < 32) {
+            const int lane = threadIdx.x;
+            MssPart o = mine;
+            bool have = false;
+            if (lane < (int)size) {
+                const uint32_t base = map_to_rank(&slot[parity], lane);
+                o.a = ld_dsmem_f32(base);
+                o.b = ld_dsmem_f32(base + 4);
+                o.v = ld_dsmem_f32(base + 8);
+                o.i = ld_dsmem_s32(base + 12);
+                have = true;
+            }
+#pragma unroll
+            for (int off = 16; off >= 1; off >>= 1) {
+                MssPart t;
+                t.a = __shfl_xor_sync(0xffffffffu, o.a, off);
+                t.b = __shfl_xor_sync(0xffffffffu, o.b, off);
+                t.v = __shfl_xor_sync(0xffffffffu, o.v, off);
+                t.i = __shfl_xor_sync(0xffffffffu, o.i, off);
+                const bool th = __shfl_xor_sync(0xffffffffu, have, off);
+                if (th) o = have ? merge(o, t) : t;
+                have = have || th;
+            }
+            if (lane == 0) *result = o;
+        }
+        __syncthreads();
+        const MssPart r = *result;
+        __syncthreads();
+        parity ^= 1;
+        return r;
+    }
+};
+
+__device__ __forceinline__ MssPart merge_maxsum(MssPart x, MssPart y) {
+    // (max, sum 2^(l c - max c)) in the log2 domain: a = max*c, b = sum
+    if (y.a == -INFINITY) return x;
+    if (x.a == -INFINITY) return y;
+    const float m = fmaxf(x.a, y.a);
+    MssPart r = x;
+    r.a = m;
+    r.b = x.b * ex2(x.a - m) + y.b * ex2(y.a - m);
+    return r;
+}
+__device__ __forceinline__ MssPart merge_sum_race(MssPart x, MssPart y) {
+    MssPart r;
+    r.a = x.a + y.a;
+    r.b = 0.f;
+    const ArgMax m = argmax_merge(ArgMax{x.v, x.i}, ArgMax{y.v, y.i});
+    r.v = m.v;
+    r.i = m.i;
+    return r;
 }
 
-// Loads kMssUnroll float4 groups of a row (k4 = k4b + j * kMssThreads) with all loads in flight.
-__device__ __forceinline__ void load_groups(const float *row, int k4b, int nk4, int V, float (&v)[kMssUnroll][4],
+// Loads kMssUnroll float4 groups of a row slice (k4 = k4b + j * kMssThreads < k4end).
+__device__ __forceinline__ void load_groups(const float *row, int k4b, int k4end, int V, float (&v)[kMssUnroll][4],
                                             bool streaming) {
 #pragma unroll
     for (int j = 0; j < kMssUnroll; ++j) {
         const int k4 = k4b + j * kMssThreads;
-        if (k4 >= nk4) continue;
+        if (k4 >= k4end) continue;
         if ((V & 3) == 0) {
             const float4 x = streaming ? __ldcs(reinterpret_cast<const float4 *>(row) + k4)
                                        : __ldcg(reinterpret_cast<const float4 *>(row) + k4);
@@ -310,197 +399,62 @@ __device__ __forceinline__ void load_groups(const float *row, int k4b, int nk4, 
     }
 }
 
-// One V-wide pass of the walk: residual r = max(0, p - q) into dst (returns sum r); when
-// `race` is set also the exponential race over r (the sample that follows the last rejection).
-__device__ void mss_residual_pass(const MssState &S, const float *lrow, const float *src, const float *qrow,
-                                  float *dst, float c, int V, bool race, uint32_t rid, uint32_t c1, uint32_t off,
-                                  uint2 key, float *tot_out, ArgMax *best_out, float *s_red, ArgMax *s_am) {
-    const int tid = threadIdx.x;
-    float part = 0.f;
-    ArgMax best{-INFINITY, -1};
-    const int nk4 = (V + 3) >> 2;
-    for (int k4b = tid; k4b < nk4; k4b += kMssUnroll * kMssThreads) {
-        float pv[kMssUnroll][4], qv[kMssUnroll][4];
-        load_groups(qrow, k4b, nk4, V, qv, true);
-        load_groups(S.mode == 0 ? lrow : src, k4b, nk4, V, pv, false);
-#pragma unroll
-        for (int j = 0; j < kMssUnroll; ++j) {
-            const int k4 = k4b + j * kMssThreads;
-            if (k4 >= nk4) continue;
-            uint4 w = make_uint4(0, 0, 0, 0);
-            if (race) w = philox4x32_10(make_uint4(rid, c1, (2u << 28) | (uint32_t)k4, off), key);
-            const uint32_t ws[4] = {w.x, w.y, w.z, w.w};
-            float rr[4];
-#pragma unroll
-            for (int i = 0; i < 4; ++i) {
-                const float pk = S.mode == 0 ? ex2(fmaf(pv[j][i], c, -S.mc)) * S.invZ : pv[j][i] * S.inv;
-                rr[i] = (4 * k4 + i < V) ? fmaxf(pk - qv[j][i], 0.f) : 0.f;
-                part += rr[i];
-                if (race && rr[i] > 0.f) best = argmax_merge(best, ArgMax{rr[i] * rcpf(race_E2(ws[i])), 4 * k4 + i});
-            }
-            if ((V & 3) == 0) {
-                __stcg(reinterpret_cast<float4 *>(dst) + k4, make_float4(rr[0], rr[1], rr[2], rr[3]));
-            } else {
-#pragma unroll
-                for (int i = 0; i < 4; ++i)
-                    if (4 * k4 + i < V) __stcg(dst + 4 * k4 + i, rr[i]);
-            }
-        }
-    }
-    *tot_out = block_sum<kMssThreads>(part, s_red);
-    if (race) *best_out = block_argmax<kMssThreads>(best, s_am);
-}
-
-// The race over the current p (fallback for an all-zero residual, reading R11).
-__device__ ArgMax mss_race_pass(const MssState &S, const float *lrow, const float *src, float c, int V,
-                                uint32_t rid, uint32_t c1, uint32_t off, uint2 key, ArgMax *s_am) {
-    ArgMax best{-INFINITY, -1};
-    for (int k4 = threadIdx.x; 4 * k4 < V; k4 += kMssThreads) {
-        const uint4 w = philox4x32_10(make_uint4(rid, c1, (2u << 28) | (uint32_t)k4, off), key);
-        const uint32_t ws[4] = {w.x, w.y, w.z, w.w};
-#pragma unroll
-        for (int i = 0; i < 4; ++i) {
-            const int k = 4 * k4 + i;
-            if (k >= V) continue;
-            const float pk = mss_p(S, lrow, src, c, k);
-            if (pk > 0.f) best = argmax_merge(best, ArgMax{pk * rcpf(race_E2(ws[i])), k});
-        }
-    }
-    return block_argmax<kMssThreads>(best, s_am);
-}
-
-__global__ void __launch_bounds__(kMssThreads, 2) verify_mss_kernel(
+__global__ void __launch_bounds__(kMssThreads) verify_mss_kernel(
     const float *__restrict__ logits, const int32_t *__restrict__ tree_tokens,
     const int32_t *__restrict__ parent, const int32_t *__restrict__ n_nodes,
     const float *__restrict__ draft_probs, const int32_t *__restrict__ req_ok, float temperature,
     uint32_t seed_lo, uint32_t seed_hi, uint32_t off, const int32_t *__restrict__ request_ids,
-    float2 *__restrict__ stats, int32_t *__restrict__ leaf_sample, uint32_t *__restrict__ counter,
     float *__restrict__ pbuf_all, int32_t *__restrict__ acc_nodes, int32_t *__restrict__ acc_tokens,
     int32_t *__restrict__ n_acc, int Nmax, int V, int path_len, unsigned long long *__restrict__ trace) {
-    const int u0 = blockIdx.x, b = blockIdx.y;
+    const int b = blockIdx.y;
     const int tid = threadIdx.x;
-    const int n = n_nodes[b];
-    const float c = 1.4426950408889634f / temperature;
+    __shared__ MssPart s_slot[2], s_result;
+    __shared__ float s_red[32];
+    __shared__ ArgMax s_am[32];
+    __shared__ int32_t s_par[kMaxNodes], s_tok[kMaxNodes], s_H[kMaxNodes];
+    __shared__ int s_nh;
+    MssCluster cl{s_slot, &s_result, cluster_ctarank(), cluster_nctarank(), 0};
+    const bool leader = (cl.rank == 0);
     int tev = 0;
     auto TR = [&](int ev) {
-        if (trace != nullptr && tid == 0 && b < 16 && ev < 64) {
+        if (trace != nullptr && tid == 0 && leader && b < 16 && ev < 64) {
             unsigned long long t;
             asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
             trace[b * 64 + ev] = t;
         }
     };
-    if (u0 == 0) TR(0);
-    __shared__ float s_red[32];
-    __shared__ ArgMax s_am[32];
-    __shared__ int32_t s_par[kMaxNodes], s_tok[kMaxNodes], s_H[kMaxNodes];
-    __shared__ int s_last, s_nh;
-    if (!req_ok[b]) {
-        if (u0 == 0) {
-            for (int j = tid; j < path_len; j += kMssThreads) {
-                acc_nodes[(size_t)b * path_len + j] = -1;
-                acc_tokens[(size_t)b * path_len + j] = -1;
-            }
-            if (tid == 0) n_acc[b] = 0;
-        }
-        return;
-    }
-    if (u0 >= n) return;
-    const uint32_t rid = request_ids ? (uint32_t)request_ids[b] : (uint32_t)b;
-    const uint2 key = make_uint2(seed_lo, seed_hi);
-    const int nk4 = (V + 3) >> 2;
-    // ---------------- phase 1 (one CTA per node): softmax statistics of node u0, and for a
-    // leaf its final sample (c4 step 4 at round 0 on p = softmax(logits[u0]/T)) ----------------
-    {
-        bool has_child = false;
-        for (int ch = u0 + 1 + tid; ch < n; ch += kMssThreads) has_child |= (parent[(size_t)b * Nmax + ch] == u0);
-        const bool leaf = !__syncthreads_or(has_child);
-        const float *lrow = logits + ((size_t)b * Nmax + u0) * V;
-        // pass A: row max (and, for a leaf, the race in log2 domain: l c - log2 E')
-        float mx = -INFINITY;
-        ArgMax best{-INFINITY, -1};
-        const uint32_t c1 = (uint32_t)u0 << 8;  // round 0
-        for (int k4b = tid; k4b < nk4; k4b += kMssUnroll * kMssThreads) {
-            float xv[kMssUnroll][4];
-            load_groups(lrow, k4b, nk4, V, xv, false);
-#pragma unroll
-            for (int j = 0; j < kMssUnroll; ++j) {
-                const int k4 = k4b + j * kMssThreads;
-                if (k4 >= nk4) continue;
-#pragma unroll
-                for (int i = 0; i < 4; ++i) mx = fmaxf(mx, xv[j][i]);
-                if (leaf) {
-                    const uint4 w = philox4x32_10(make_uint4(rid, c1, (2u << 28) | (uint32_t)k4, off), key);
-                    const uint32_t ws[4] = {w.x, w.y, w.z, w.w};
-#pragma unroll
-                    for (int i = 0; i < 4; ++i)
-                        if (4 * k4 + i < V) best = argmax_merge(best, ArgMax{xv[j][i] * c - lg2f(race_E2(ws[i])), 4 * k4 + i});
-                }
-            }
-        }
-        // block max
-#pragma unroll
-        for (int o = 16; o >= 1; o >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, o));
-        if ((tid & 31) == 0) s_red[tid >> 5] = mx;
-        __syncthreads();
-        if (tid < 32) {
-            float m2 = tid < kMssThreads / 32 ? s_red[tid] : -INFINITY;
-#pragma unroll
-            for (int o = 16; o >= 1; o >>= 1) m2 = fmaxf(m2, __shfl_xor_sync(0xffffffffu, m2, o));
-            if (tid == 0) s_red[0] = m2;
-        }
-        __syncthreads();
-        const float mc = s_red[0] * c;
-        __syncthreads();
-        if (leaf) best = block_argmax<kMssThreads>(best, s_am);
-        // pass B: z = sum 2^(l c - m c)  (the row is L2-resident after pass A)
-        float z = 0.f;
-        for (int k4b = tid; k4b < nk4; k4b += kMssUnroll * kMssThreads) {
-            float xv[kMssUnroll][4];
-            load_groups(lrow, k4b, nk4, V, xv, false);
-#pragma unroll
-            for (int j = 0; j < kMssUnroll; ++j)
-#pragma unroll
-                for (int i = 0; i < 4; ++i) z += (k4b + j * kMssThreads < nk4) ? ex2(fmaf(xv[j][i], c, -mc)) : 0.f;
-        }
-        z = block_sum<kMssThreads>(z, s_red);
-        if (tid == 0) {
-            stats[(size_t)b * Nmax + u0] = make_float2(mc, z);
-            leaf_sample[(size_t)b * Nmax + u0] = leaf ? best.i : -1;
-            __threadfence();
-            const unsigned old = atomicAdd(&counter[b], 1u);
-            s_last = (old == (unsigned)(n - 1));
-        }
-        __syncthreads();
-        if (!s_last) return;
-        __threadfence();
-    }
-    TR(1);
-    tev = 2;
-    // ---------------- phase 2 (last CTA of the request): the walk of Alg. 2 ----------------
+    TR(tev++);
     int32_t *an = acc_nodes + (size_t)b * path_len;
     int32_t *at = acc_tokens + (size_t)b * path_len;
-    for (int j = tid; j < path_len; j += kMssThreads) {
-        an[j] = -1;
-        at[j] = -1;
+    if (leader)
+        for (int j = tid; j < path_len; j += kMssThreads) {
+            an[j] = -1;
+            at[j] = -1;
+        }
+    if (!req_ok[b]) {  // uniform over the cluster
+        if (leader && tid == 0) n_acc[b] = 0;
+        return;
     }
+    const int n = n_nodes[b];
     for (int i = tid; i < n; i += kMssThreads) {
         s_par[i] = parent[(size_t)b * Nmax + i];
         s_tok[i] = tree_tokens[(size_t)b * Nmax + i];
     }
+    const float c = 1.4426950408889634f / temperature;
+    const uint32_t rid = request_ids ? (uint32_t)request_ids[b] : (uint32_t)b;
+    const uint2 key = make_uint2(seed_lo, seed_hi);
+    // this CTA's slice of the vocabulary, in float4 groups
+    const int nk4 = (V + 3) >> 2;
+    const int k4lo = (int)((long long)nk4 * cl.rank / cl.size);
+    const int k4hi = (int)((long long)nk4 * (cl.rank + 1) / cl.size);
     float *bufs = pbuf_all + (size_t)b * 2 * V;
     __syncthreads();
-    if (tid == 0) {
-        an[0] = 0;
-        counter[b] = 0u;  // reusable by the next call on this workspace
-    }
+    if (leader && tid == 0) an[0] = 0;
+
     int u = 0, cnt = 0;
     for (;;) {
         const float *lrow = logits + ((size_t)b * Nmax + u) * V;
-        // step 1: p = softmax(logits[u] / T), implicit through the phase-1 statistics
-        const float2 su = __ldcg(stats + (size_t)b * Nmax + u);
-        MssState S{0, 0, su.x, 1.0f / su.y, 0.f};
-        uint32_t round = 0;
-        // step 2: children of u in ascending order
+        // children of u in ascending order (step 2)
         if (tid == 0) {
             int nh = 0;
             for (int ch = u + 1; ch < n; ++ch)
@@ -510,12 +464,74 @@ __global__ void __launch_bounds__(kMssThreads, 2) verify_mss_kernel(
         __syncthreads();
         int nh = s_nh;
         if (nh == 0) {
-            // a leaf: its round-0 sample was drawn in phase 1
-            if (tid == 0) at[cnt] = __ldcg(leaf_sample + (size_t)b * Nmax + u);
+            // a leaf: x_next ~ softmax(logits[u]/T) at round 0 (steps 1 and 4); race in log2 domain
+            ArgMax best{-INFINITY, -1};
+            const uint32_t c1 = (uint32_t)u << 8;
+            for (int k4b = k4lo + tid; k4b < k4hi; k4b += kMssUnroll * kMssThreads) {
+                float xv[kMssUnroll][4];
+                load_groups(lrow, k4b, k4hi, V, xv, true);
+#pragma unroll
+                for (int j = 0; j < kMssUnroll; ++j) {
+                    const int k4 = k4b + j * kMssThreads;
+                    if (k4 >= k4hi) continue;
+                    const uint4 w = philox4x32_10(make_uint4(rid, c1, (2u << 28) | (uint32_t)k4, off), key);
+                    const uint32_t ws[4] = {w.x, w.y, w.z, w.w};
+#pragma unroll
+                    for (int i = 0; i < 4; ++i)
+                        if (4 * k4 + i < V) best = argmax_merge(best, ArgMax{xv[j][i] * c - lg2f(race_E2(ws[i])), 4 * k4 + i});
+                }
+            }
+            best = block_argmax<kMssThreads>(best, s_am);
+            const MssPart r = cl.reduce(MssPart{0.f, 0.f, best.v, best.i}, merge_sum_race);
+            if (leader && tid == 0) at[cnt] = r.i;
             break;
         }
-        int accepted = -1;
-        int final_tok = -1;
+        // step 1: softmax statistics of logits[u] / T (one pass, online max/sum)
+        float mc = -INFINITY, z = 0.f;
+        for (int k4b = k4lo + tid; k4b < k4hi; k4b += kMssUnroll * kMssThreads) {
+            float xv[kMssUnroll][4];
+            load_groups(lrow, k4b, k4hi, V, xv, false);
+#pragma unroll
+            for (int j = 0; j < kMssUnroll; ++j) {
+                if (k4b + j * kMssThreads >= k4hi) continue;
+                float lm = -INFINITY;
+#pragma unroll
+                for (int i = 0; i < 4; ++i) lm = fmaxf(lm, xv[j][i] * c);
+                if (lm > mc) {
+                    z = (mc == -INFINITY) ? 0.f : z * ex2(mc - lm);
+                    mc = lm;
+                }
+#pragma unroll
+                for (int i = 0; i < 4; ++i) z += ex2(fmaf(xv[j][i], c, -mc));
+            }
+        }
+        {
+            // block merge of (mc, z)
+#pragma unroll
+            for (int o = 16; o >= 1; o >>= 1) {
+                const float om = __shfl_xor_sync(0xffffffffu, mc, o), oz = __shfl_xor_sync(0xffffffffu, z, o);
+                const MssPart m = merge_maxsum(MssPart{mc, z, 0.f, 0}, MssPart{om, oz, 0.f, 0});
+                mc = m.a;
+                z = m.b;
+            }
+            __shared__ float s_m[32], s_z[32];
+            if ((tid & 31) == 0) {
+                s_m[tid >> 5] = mc;
+                s_z[tid >> 5] = z;
+            }
+            __syncthreads();
+            MssPart acc{-INFINITY, 0.f, 0.f, 0};
+            for (int w = 0; w < kMssThreads / 32; ++w) acc = merge_maxsum(acc, MssPart{s_m[w], s_z[w], 0.f, 0});
+            __syncthreads();
+            const MssPart r = cl.reduce(acc, merge_maxsum);
+            mc = r.a;
+            z = r.b;
+        }
+        int mode = 0, cur = 0;    // p = 2^(l c - mc)/z (mode 0) or buf[cur] * inv (mode 1)
+        const float invZ = 1.0f / z;
+        float inv = 0.f;
+        uint32_t round = 0;
+        int accepted = -1, final_tok = -1;
         // step 3: try children in Philox-uniform order
         while (nh > 0) {
             const uint4 w = philox4x32_10(make_uint4(rid, ((uint32_t)u << 8) | round, 0u, off), key);
@@ -524,29 +540,76 @@ __global__ void __launch_bounds__(kMssThreads, 2) verify_mss_kernel(
             const int s = s_H[idx];
             const int x = s_tok[s];
             const float *qrow = draft_probs + ((size_t)b * Nmax + s) * V;
-            const float px = mss_p(S, lrow, bufs + (size_t)S.cur * V, c, x);
+            const float px = mode == 0 ? ex2(fmaf(__ldcg(lrow + x), c, -mc)) * invZ
+                                       : __ldcg(bufs + (size_t)cur * V + x) * inv;
             const float rq = r * __ldg(qrow + x);
             if (px > 0.f && rq <= px) {
                 accepted = s;
                 break;
             }
-            // reject: residual max(0, p - q) into the other buffer (and, after the last child,
-            // the exponential race over it with the next round's counters)
+            // reject: residual max(0, p - q) of this CTA's slice into the other buffer, and after
+            // the last child the exponential race over it (next round's counters)
             const bool last = (nh == 1);
-            const int dsti = (S.mode == 0) ? 0 : (S.cur ^ 1);
-            float tot;
-            ArgMax best;
-            mss_residual_pass(S, lrow, bufs + (size_t)S.cur * V, qrow, bufs + (size_t)dsti * V, c, V, last, rid,
-                              ((uint32_t)u << 8) | (round + 1), off, key, &tot, &best, s_red, s_am);
-            if (tot > 0.f) {
-                S.cur = dsti;
-                S.mode = 1;
-                S.inv = 1.0f / tot;
-                if (last) final_tok = best.i;
+            const int dsti = (mode == 0) ? 0 : (cur ^ 1);
+            const float *src = mode == 0 ? lrow : bufs + (size_t)cur * V;
+            float *dst = bufs + (size_t)dsti * V;
+            const uint32_t c1 = ((uint32_t)u << 8) | (round + 1);
+            float part = 0.f;
+            ArgMax best{-INFINITY, -1};
+            for (int k4b = k4lo + tid; k4b < k4hi; k4b += kMssUnroll * kMssThreads) {
+                float pv[kMssUnroll][4], qv[kMssUnroll][4];
+                load_groups(qrow, k4b, k4hi, V, qv, true);
+                load_groups(src, k4b, k4hi, V, pv, false);
+#pragma unroll
+                for (int j = 0; j < kMssUnroll; ++j) {
+                    const int k4 = k4b + j * kMssThreads;
+                    if (k4 >= k4hi) continue;
+                    uint4 wr = make_uint4(0, 0, 0, 0);
+                    if (last) wr = philox4x32_10(make_uint4(rid, c1, (2u << 28) | (uint32_t)k4, off), key);
+                    const uint32_t ws[4] = {wr.x, wr.y, wr.z, wr.w};
+                    float rr[4];
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) {
+                        const float pk = mode == 0 ? ex2(fmaf(pv[j][i], c, -mc)) * invZ : pv[j][i] * inv;
+                        rr[i] = (4 * k4 + i < V) ? fmaxf(pk - qv[j][i], 0.f) : 0.f;
+                        part += rr[i];
+                        if (last && rr[i] > 0.f) best = argmax_merge(best, ArgMax{rr[i] * rcpf(race_E2(ws[i])), 4 * k4 + i});
+                    }
+                    if ((V & 3) == 0) {
+                        __stcg(reinterpret_cast<float4 *>(dst) + k4, make_float4(rr[0], rr[1], rr[2], rr[3]));
+                    } else {
+#pragma unroll
+                        for (int i = 0; i < 4; ++i)
+                            if (4 * k4 + i < V) __stcg(dst + 4 * k4 + i, rr[i]);
+                    }
+                }
+            }
+            part = block_sum<kMssThreads>(part, s_red);
+            if (last) best = block_argmax<kMssThreads>(best, s_am);
+            // the reduction's cluster barrier also publishes this CTA's residual slice
+            const MssPart red = cl.reduce(MssPart{part, 0.f, best.v, best.i}, merge_sum_race);
+            if (red.a > 0.f) {
+                mode = 1;
+                cur = dsti;
+                inv = 1.0f / red.a;
+                if (last) final_tok = red.i;
             } else if (last) {
-                // R11: the residual is all zero, p is kept; sample from it
-                final_tok = mss_race_pass(S, lrow, bufs + (size_t)S.cur * V, c, V, rid,
-                                          ((uint32_t)u << 8) | (round + 1), off, key, s_am).i;
+                // R11: the residual is all zero, p is kept; sample from it with the same counters
+                ArgMax b2{-INFINITY, -1};
+                const float *src2 = mode == 0 ? lrow : bufs + (size_t)cur * V;
+                for (int k4 = k4lo + tid; k4 < k4hi; k4 += kMssThreads) {
+                    const uint4 w2 = philox4x32_10(make_uint4(rid, c1, (2u << 28) | (uint32_t)k4, off), key);
+                    const uint32_t ws[4] = {w2.x, w2.y, w2.z, w2.w};
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) {
+                        const int k = 4 * k4 + i;
+                        if (k >= V) continue;
+                        const float pk = mode == 0 ? ex2(fmaf(__ldcg(src2 + k), c, -mc)) * invZ : __ldcg(src2 + k) * inv;
+                        if (pk > 0.f) b2 = argmax_merge(b2, ArgMax{pk * rcpf(race_E2(ws[i])), k});
+                    }
+                }
+                b2 = block_argmax<kMssThreads>(b2, s_am);
+                final_tok = cl.reduce(MssPart{0.f, 0.f, b2.v, b2.i}, merge_sum_race).i;
             }
             if (tid == 0) {
                 for (int j = idx; j + 1 < nh; ++j) s_H[j] = s_H[j + 1];
@@ -558,7 +621,7 @@ __global__ void __launch_bounds__(kMssThreads, 2) verify_mss_kernel(
         }
         if (accepted >= 0) {
             ++cnt;
-            if (tid == 0) {
+            if (leader && tid == 0) {
                 an[cnt] = accepted;
                 at[cnt - 1] = s_tok[accepted];
             }
@@ -567,11 +630,12 @@ __global__ void __launch_bounds__(kMssThreads, 2) verify_mss_kernel(
             continue;
         }
         // step 4: every child was rejected; x_next was drawn during the last residual pass
-        if (tid == 0) at[cnt] = final_tok;
+        if (leader && tid == 0) at[cnt] = final_tok;
         break;
     }
-    if (tid == 0) n_acc[b] = cnt + 1;
+    if (leader && tid == 0) n_acc[b] = cnt + 1;
     TR(63);
+    cluster_sync_all();  // no CTA leaves while others may still read its DSMEM slots
 }
 
 unsigned long long *g_mss_trace = nullptr;  // debug only (specinfer_debug_set_trace with SPECINFER_TRACE_MSS)
@@ -593,15 +657,23 @@ cudaError_t launch_verify_mss(const specinfer_shape_t &s, const WsLayout &w, con
                               const float *draft_probs, float temperature, uint64_t seed, uint64_t offset,
                               const int32_t *request_ids, int32_t *acc_nodes, int32_t *acc_tokens,
                               int32_t *n_acc, char *ws, cudaStream_t stream) {
-    dim3 grid(s.max_nodes, s.batch);
-    verify_mss_kernel<<<grid, kMssThreads, 0, stream>>>(
-        logits, tree_tokens, parent, n_nodes, draft_probs, reinterpret_cast<const int32_t *>(ws + w.req_ok),
-        temperature, (uint32_t)seed, (uint32_t)(seed >> 32), (uint32_t)offset, request_ids,
-        reinterpret_cast<float2 *>(ws + w.mss_stats), reinterpret_cast<int32_t *>(ws + w.mss_leaf),
-        reinterpret_cast<uint32_t *>(ws + w.verify_cnt) + s.batch,
-        reinterpret_cast<float *>(ws + w.mss_p), acc_nodes, acc_tokens, n_acc, s.max_nodes, s.vocab,
-        s.max_depth + 1, g_mss_trace);
-    return cudaGetLastError();
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(kMssCluster, s.batch);
+    cfg.blockDim = dim3(kMssThreads);
+    cfg.dynamicSmemBytes = 0;
+    cfg.stream = stream;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = kMssCluster;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, verify_mss_kernel, logits, tree_tokens, parent, n_nodes, draft_probs,
+                              reinterpret_cast<const int32_t *>(ws + w.req_ok), temperature, (uint32_t)seed,
+                              (uint32_t)(seed >> 32), (uint32_t)offset, request_ids,
+                              reinterpret_cast<float *>(ws + w.mss_p), acc_nodes, acc_tokens, n_acc, s.max_nodes,
+                              s.vocab, s.max_depth + 1, g_mss_trace);
 }
 
 cudaError_t launch_philox_debug(const uint32_t *ck, uint32_t *out, int n, cudaStream_t stream) {
