@@ -325,34 +325,77 @@ def run_ours(args, ws, rank, local):
             sum(t.numel() * 4 for t in h_tree)
         d2h = h_res_a.numel() * 4 + h_res_n.numel() * 4
 
+        # One CUDA graph per step: the H2D copies run on a copy stream (pinned memory, the copy
+        # engines) and each layer's attention waits only for its own q, so the PCIe transfer of
+        # layer l+1's q and of the logits / draft probabilities overlaps the attention of layer l.
+        copy_s = torch.cuda.Stream(device)
+        ev_fork = torch.cuda.Event()
+        ev_tree = torch.cuda.Event()
+        ev_q = [torch.cuda.Event() for _ in range(L)]
+        ev_lg = torch.cuda.Event()
+
         def e2e_step():
-            for d, h in zip(dsts, h_tree):
-                d.copy_(h, non_blocking=True)
-            wl.ai.q.copy_(h_q, non_blocking=True)
-            wl.vi.logits.copy_(h_logits, non_blocking=True)
-            if h_draft is not None:
-                wl.vi.draft_probs.copy_(h_draft, non_blocking=True)
-            step()
+            ev_fork.record(s)
+            copy_s.wait_event(ev_fork)
+            with torch.cuda.stream(copy_s):
+                for d, h in zip(dsts, h_tree):
+                    d.copy_(h, non_blocking=True)
+                ev_tree.record(copy_s)
+                for l in range(L):
+                    wl.ai.q[l].copy_(h_q[l], non_blocking=True)
+                    ev_q[l].record(copy_s)
+                wl.vi.logits.copy_(h_logits, non_blocking=True)
+                if h_draft is not None:
+                    wl.vi.draft_probs.copy_(h_draft, non_blocking=True)
+                ev_lg.record(copy_s)
+            s.wait_event(ev_tree)
+            seg_prepare()
+            for l in range(L):
+                s.wait_event(ev_q[l])
+                st.attention(wl.ai.q[l], wl.ai.k_cache[l], wl.ai.v_cache[l], out[l])
+            s.wait_event(ev_lg)
+            seg_verify_commit()
+            gather()
             h_res_a.copy_(res_a, non_blocking=True)
             h_res_n.copy_(res_n, non_blocking=True)
 
         with torch.cuda.stream(s):
-            for _ in range(max(1, args.warmup // 2)):
+            e2e_step()  # eager warm-up of the multi-stream step
+        torch.cuda.synchronize(device)
+        g_e2e = None
+        if ws == 1:
+            g_e2e = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g_e2e, stream=s):
                 e2e_step()
+            torch.cuda.synchronize(device)
+
+        def e2e_run():
+            if g_e2e is not None:
+                g_e2e.replay()
+            else:
+                e2e_step()
+
+        with torch.cuda.stream(s):
+            for _ in range(max(1, args.warmup // 2)):
+                e2e_run()
         torch.cuda.synchronize(device)
         barrier(ws)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         with torch.cuda.stream(s):
             e0.record(s)
             for _ in range(K):
-                e2e_step()
+                e2e_run()
             e1.record(s)
         torch.cuda.synchronize(device)
         barrier(ws)
         e2e_ms = max_over_ranks(e0.elapsed_time(e1), ws, device)
         e2e = {"value": round(tokens_step * ws * K / (e2e_ms / 1e3), 1), "unit": UNIT,
                "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
-               "ms_per_step": round(e2e_ms / K, 4)}
+               "ms_per_step": round(e2e_ms / K, 4),
+               "inputs": "per step from pinned host memory: tree arrays, q of every layer, logits"
+                         + (", draft probabilities" if h_draft is not None else "")
+                         + "; result read back: accepted tokens + counts; H2D on a copy stream "
+                           "overlapping the attention of earlier layers"}
 
     cpu = None
     if rank == 0 and ws == 1 and not args.no_cpu:
@@ -386,44 +429,51 @@ def run_ours(args, ws, rank, local):
 # ------------------------------------------------------------------------------------------
 # CPU baseline: the fp64 oracle as it stands, on a bounded sample of the same workload
 # ------------------------------------------------------------------------------------------
-def _oracle_sample(wl: Workload, n_req: int):
+def _oracle_sample(wl: Workload, n_req: int, layers=(0,)):
+    """Times the fp64 oracle (as it stands) on `n_req` requests of the workload: tree attention of the
+    given layers, then greedy / MSS verification of those requests."""
     import oracle
     cores = len(os.sched_getaffinity(0))
     os.environ["OMP_NUM_THREADS"] = str(cores)
-    q = wl.ai.q[0, :n_req].cpu()
-    k = wl.ai.k_cache[0, :n_req].cpu()
-    v = wl.ai.v_cache[0, :n_req].cpu()
     tb = wl.tb
     par, dep = tb.parent[:n_req].cpu(), tb.depth[:n_req].cpu()
     pl, nn_ = tb.prefix_len[:n_req].cpu(), tb.n_nodes[:n_req].cpu()
     lg = wl.vi.logits[:n_req].cpu().numpy()
     toks = wl.vi.tree_tokens[:n_req].cpu().numpy()
     dr = wl.vi.draft_probs[:n_req].cpu().numpy() if "mss" in wl.verify else None
-    t0 = time.perf_counter()
-    oracle.tree_attention(q, k, v, par, dep, pl, nn_)
+    ta = 0.0
+    for l in layers:
+        q = wl.ai.q[l, :n_req].cpu()
+        k = wl.ai.k_cache[l, :n_req].cpu()
+        v = wl.ai.v_cache[l, :n_req].cpu()
+        t0 = time.perf_counter()
+        oracle.tree_attention(q, k, v, par, dep, pl, nn_)
+        ta += time.perf_counter() - t0
     t1 = time.perf_counter()
     if "greedy" in wl.verify:
         oracle.verify_greedy(lg, toks, par.numpy(), nn_.numpy(), path_len=wl.Dmax + 1)
     if "mss" in wl.verify:
         oracle.verify_mss(lg, toks, par.numpy(), nn_.numpy(), dr, seed=1, path_len=wl.Dmax + 1)
-    t2 = time.perf_counter()
-    return t1 - t0, t2 - t1, cores
+    tv = time.perf_counter() - t1
+    return ta, tv, cores
 
 
-def cpu_baseline(wl: Workload, budget_s: float = 15.0):
+def cpu_baseline(wl: Workload, budget_s: float = 12.0):
+    """The oracle timed on the host cores on a bounded sample (~10-20 s): every request of the
+    step, as many layers as fit the budget (extrapolated linearly to all layers when fewer)."""
     import oracle  # noqa: F401  (test infrastructure; only this leg and --impl reference use it)
-    # calibrate with one request, then size the sample to ~budget_s
-    ta, tv, cores = _oracle_sample(wl, 1)
-    n_req = int(max(1, min(wl.B, budget_s / max(ta + tv, 1e-3))))
-    if n_req > 1:
-        ta, tv, cores = _oracle_sample(wl, n_req)
-    # extrapolate: attention for all L layers, verification once, for n_req requests
-    t_step = ta * wl.L + tv
-    tokens = int(wl.tb.n_nodes[:n_req].sum().item())
+    ta1, tv, cores = _oracle_sample(wl, wl.B, layers=(0,))
+    n_layers = int(max(1, min(wl.L, budget_s // max(ta1, 1e-3))))
+    if n_layers > 1:
+        ta, tv, cores = _oracle_sample(wl, wl.B, layers=tuple(range(n_layers)))
+    else:
+        ta = ta1
+    t_step = ta * wl.L / n_layers + tv
+    tokens = wl.tree_tokens_per_step()
+    extra = "" if n_layers == wl.L else f", x{wl.L / n_layers:.1f} extrapolated to {wl.L} layers"
     return {"value": round(tokens / t_step, 3), "unit": UNIT, "cores": cores, "kind": "oracle",
-            "sample": f"{n_req} request(s) x 1 layer of {wl.cfg.name} tree attention (fp64, measured "
-                      f"{ta:.2f} s, x{wl.L} layers extrapolated) + verification of those requests "
-                      f"({tv:.2f} s)"}
+            "sample": f"all {wl.B} requests, tree attention of {n_layers} of {wl.L} layers "
+                      f"({ta:.1f} s fp64{extra}) + greedy/MSS verification ({tv:.2f} s)"}
 
 
 def run_reference(args, ws, rank, local):
@@ -441,8 +491,8 @@ def run_reference(args, ws, rank, local):
     t_tot = 0.0
     tokens = 0
     cores = 1
-    for _ in range(args.steps):
-        ta, tv, cores = _oracle_sample(wl, 1)
+    for it in range(args.steps):
+        ta, tv, cores = _oracle_sample(wl, 1, layers=(it % wl.L,))
         t_tot += ta * wl.L + tv
         tokens += int(wl.tb.n_nodes[:1].sum().item())
     value = tokens / t_tot
