@@ -1,0 +1,161 @@
+// attn_shared.cuh — pieces shared by the two tree-attention kernels (tree_attention.cu:
+// swapped keys-as-M kernel for <= 64 query rows per kv-head; tree_attention_rows.cu: rows-as-M
+// kernel for wider trees / GQA groups): launch parameters, schedule helpers, TMA helpers,
+// tensor-map encoding, debug tracing.
+#pragma once
+#include "common.cuh"
+
+namespace specinfer {
+
+struct AttnParams {
+    const int32_t *prefix_len;
+    const int32_t *n_nodes;
+    const int32_t *item_start;
+    const int4 *item_info;
+    const int4 *cta_info;
+    uint32_t *item_cnt;
+    const unsigned long long *rowmask;
+    const uint32_t *anc;
+    float *part_o;
+    float *part_ml;
+    __nv_bfloat16 *out;
+    int B, Nmax, Hq, Hkv, G, Smax, chunks, npc, n_items, nk_slots, nv_slots;
+    float scale_log2;
+    unsigned long long *trace;  // optional per-tile timestamps (debug), nullptr in production
+    int debug_flags;            // experiments only: 1 = skip K/V TMA, 2 = skip MMAs (results invalid)
+};
+
+// debug timestamps: trace[cta][tile][event], CTAs < kTraceCtas, tiles < kTraceTiles
+constexpr int kTraceCtas = 8, kTraceTiles = 64, kTraceEv = 12;
+__device__ __forceinline__ unsigned long long globaltimer_ns() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+// kernel-level timestamps of every CTA (ns): [entry, exit, first K issue, 0]
+#define SPI_TRACE_K(slot)                                                                                  \
+    do {                                                                                                   \
+        if (p.trace != nullptr)                                                                            \
+            p.trace[(size_t)kTraceCtas * kTraceTiles * kTraceEv + blockIdx.x * 4 + (slot)] = globaltimer_ns(); \
+    } while (0)
+#define SPI_TRACE(ev)                                                                               \
+    do {                                                                                            \
+        if (p.trace != nullptr && blockIdx.x < kTraceCtas && lt < kTraceTiles)                      \
+            p.trace[((size_t)blockIdx.x * kTraceTiles + lt) * kTraceEv + (ev)] = clock64();         \
+    } while (0)
+
+constexpr int kSlotBytes = kKeyTile * kHeadDim * 2;  // 32 KB: one K or V tile
+constexpr int kHalfBytes = kSlotBytes / 2;            // 16 KB: 128 keys x 64 dims
+// the last tile of a request is loaded row-exactly (boxes of 16, 4 and 1 rows) so that no cache
+// slot at or beyond P_b + n_b is ever read; the rest of the slot keeps stale finite data
+constexpr float kRescaleThreshold = 8.0f;              // log2 units: stale max tolerance
+constexpr int kCombineBatch = 8;                       // split pieces merged per round
+constexpr int kSegRing = 16;                           // segment descriptors in flight
+constexpr int kMaxSlots = 8;
+
+
+struct SegDesc {
+    int x, begin, end, ib, ie, b, g, c, P, n;
+};
+
+__device__ __forceinline__ int cta_start(long long c, long long T, long long NC) {
+    return (int)((c * T) / NC);
+}
+
+__device__ __forceinline__ int cta_of_tile(int t, int T, int NC) {
+    int c = (int)(((long long)t * NC) / T);
+    if (c >= NC) c = NC - 1;
+    while (c + 1 < NC && cta_start(c + 1, T, NC) <= t) ++c;
+    while (c > 0 && cta_start(c, T, NC) > t) --c;
+    return c;
+}
+
+// Cross-lane "transpose reduction": on entry each lane holds N values (one per row); on exit
+// lane l holds in v[0] the reduction over the 32 lanes of row (l mod N) (N <= 32).
+template <int N, bool kIsMax>
+__device__ __forceinline__ void transpose_reduce(float *v) {
+    const int lane = threadIdx.x & 31;
+#pragma unroll
+    for (int off = N / 2; off >= 1; off >>= 1) {
+        const bool upper = (lane & off) != 0;
+#pragma unroll
+        for (int i = 0; i < off; ++i) {
+            const float send = upper ? v[i] : v[i + off];
+            const float keep = upper ? v[i + off] : v[i];
+            const float got = __shfl_xor_sync(0xffffffffu, send, off);
+            v[i] = kIsMax ? fmaxf(keep, got) : keep + got;
+        }
+    }
+#pragma unroll
+    for (int off = N; off < 32; off <<= 1) {
+        const float got = __shfl_xor_sync(0xffffffffu, v[0], off);
+        v[0] = kIsMax ? fmaxf(v[0], got) : v[0] + got;
+    }
+}
+
+// Loads rows [row0, row0 + nv) of a K or V tile (nv < 128) with boxes of 16, 4 and 1 rows.
+__device__ __forceinline__ void tma_load_rows(uint8_t *dst, uint64_t *bar, int nv, int row0, uint64_t pol,
+                                              const CUtensorMap *m16, const CUtensorMap *m4,
+                                              const CUtensorMap *m1) {
+    mbar_arrive_expect_tx(bar, (uint32_t)nv * 256u);
+    int r = 0;
+    for (; r + 16 <= nv; r += 16) {
+        tma_load_2d(dst + r * 128, m16, bar, 0, row0 + r, pol);
+        tma_load_2d(dst + kHalfBytes + r * 128, m16, bar, 64, row0 + r, pol);
+    }
+    for (; r + 4 <= nv; r += 4) {
+        tma_load_2d(dst + r * 128, m4, bar, 0, row0 + r, pol);
+        tma_load_2d(dst + kHalfBytes + r * 128, m4, bar, 64, row0 + r, pol);
+    }
+    for (; r < nv; ++r) {
+        tma_load_2d(dst + r * 128, m1, bar, 0, row0 + r, pol);
+        tma_load_2d(dst + kHalfBytes + r * 128, m1, bar, 64, row0 + r, pol);
+    }
+}
+
+// ------------------------------------------------------------------------------------------
+// host side
+// ------------------------------------------------------------------------------------------
+typedef CUresult (*PFN_encodeTiled_t)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *,
+                                      const cuuint64_t *, const cuuint64_t *, const cuuint32_t *,
+                                      const cuuint32_t *, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                      CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+static PFN_encodeTiled_t get_encode_fn() {
+    static PFN_encodeTiled_t fn = nullptr;
+    if (!fn) {
+        void *ptr = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &ptr, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<PFN_encodeTiled_t>(ptr);
+    }
+    return fn;
+}
+
+static bool encode_2d(CUtensorMap *m, const void *base, uint64_t rows, uint32_t box_rows) {
+    PFN_encodeTiled_t enc = get_encode_fn();
+    if (!enc) return false;
+    const cuuint64_t dims[2] = {128, rows};
+    const cuuint64_t strides[1] = {256};
+    const cuuint32_t box[2] = {64, box_rows};
+    const cuuint32_t estr[2] = {1, 1};
+    return enc(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void *>(base), dims, strides, box, estr,
+               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+static bool encode_q(CUtensorMap *m, const void *base, int Hq, uint64_t nodes, int G, int npc) {
+    PFN_encodeTiled_t enc = get_encode_fn();
+    if (!enc) return false;
+    const cuuint64_t dims[3] = {128, (cuuint64_t)Hq, nodes};
+    const cuuint64_t strides[2] = {256, (cuuint64_t)Hq * 256};
+    const cuuint32_t box[3] = {64, (cuuint32_t)G, (cuuint32_t)npc};
+    const cuuint32_t estr[3] = {1, 1, 1};
+    return enc(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, const_cast<void *>(base), dims, strides, box, estr,
+               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+
+}  // namespace specinfer

@@ -48,11 +48,16 @@ struct WsLayout {
 
 inline size_t align256(size_t x) { return (x + 255) & ~size_t(255); }
 
+// Query rows per work item.  Up to 64 rows (G * Nmax <= 64): the "swapped" kernel (keys as the
+// UMMA M dimension, NT = 16/32/64 rows as N).  Wider trees / GQA groups: the rows-as-M kernel with
+// 128-row blocks (kRowsBlock), one TMEM lane per query row.
+constexpr int kRowsBlock = 128;
 inline int choose_nt(int G, int nmax) {
     const int r = G * nmax;
     if (r <= 16 && G <= 16) return 16;
     if (r <= 32 && G <= 32) return 32;
-    return 64;
+    if (r <= 64) return 64;
+    return kRowsBlock;
 }
 
 inline WsLayout ws_layout(const specinfer_shape_t &s, int num_sms) {

@@ -77,8 +77,8 @@ __global__ void __launch_bounds__(256) tree_validate_bitsets_kernel(
     }
     // row masks of the tree part for the attention kernel: bit r of rowmask[b][c][j] is set iff
     // query row r of chunk c (node c*npc + r/G) exists and has tree node j on its root path
-    const int rc = G * npc;
-    for (int idx = threadIdx.x; idx < chunks * Nmax; idx += blockDim.x) {
+    const int rc = G * npc;  // the row masks serve the swapped kernel (<= 64 rows per chunk)
+    for (int idx = threadIdx.x; rc <= 64 && idx < chunks * Nmax; idx += blockDim.x) {
         const int c = idx / Nmax, j = idx - c * Nmax;
         unsigned long long m = 0ull;
         if (ok && j < n) {

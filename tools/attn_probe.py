@@ -68,8 +68,8 @@ def main():
         t = allt[:8 * 64 * 12].reshape(8, 64, 12)
         kt = allt[8 * 64 * 12:].reshape(-1, 4)
         kt = kt[kt[:, 0] > 0]
-        t0 = kt[:, 0].min()
-        print(f"kernel-level (us from first CTA entry) over {len(kt)} CTAs: entry max {(kt[:,0].max()-t0)/1e3:.2f}; "
+        t0 = kt[:, 0].min() if len(kt) else 0
+        if len(kt): print(f"kernel-level (us from first CTA entry) over {len(kt)} CTAs: entry max {(kt[:,0].max()-t0)/1e3:.2f}; "
               f"first K issue median {np.median(kt[:,2]-t0)/1e3:.2f} max {(kt[:,2].max()-t0)/1e3:.2f}; "
               f"exit min {(kt[:,1].min()-t0)/1e3:.2f} median {np.median(kt[:,1]-t0)/1e3:.2f} max {(kt[:,1].max()-t0)/1e3:.2f}")
         names = ["K-iss", "V-iss", "S-mma", "PV-mma", "sm-beg", "P-rdy", "epi-PV", "epi-end", "epi-st", "epi-ld", "seg-beg"]
