@@ -92,9 +92,6 @@ specinfer_status_t check_ws(const void *ws) {
     return SPECINFER_OK;
 }
 
-// the persistent tree-attention grid: one CTA per SM (tree_prepare builds its schedule)
-int attention_grid(int num_sms) { return num_sms; }
-
 specinfer_status_t from_cuda(cudaError_t e) { return e == cudaSuccess ? SPECINFER_OK : SPECINFER_ERR_CUDA; }
 
 #define SPI_TRY(x)                                 \
@@ -124,7 +121,7 @@ specinfer_status_t specinfer_tree_prepare(const specinfer_shape_t *shape, const 
     SPI_TRY(check_device(&d));
     const WsLayout w = ws_layout(*shape, d.num_sms);
     return from_cuda(launch_tree_prepare(*shape, w, parent, depth, prefix_len, n_nodes,
-                                         reinterpret_cast<char *>(workspace), attention_grid(d.num_sms),
+                                         reinterpret_cast<char *>(workspace), w.grid,
                                          (cudaStream_t)stream));
 }
 
@@ -143,7 +140,7 @@ specinfer_status_t specinfer_tree_attention(const specinfer_shape_t *shape, cons
     SPI_TRY(check_device(&d));
     const WsLayout w = ws_layout(*shape, d.num_sms);
     return from_cuda(launch_tree_attention(*shape, w, q, k_cache, v_cache, prefix_len, n_nodes, out,
-                                           reinterpret_cast<char *>(workspace), attention_grid(d.num_sms), d.max_smem,
+                                           reinterpret_cast<char *>(workspace), w.grid, d.max_smem,
                                            (cudaStream_t)stream));
 }
 

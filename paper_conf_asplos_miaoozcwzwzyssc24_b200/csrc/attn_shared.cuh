@@ -20,6 +20,7 @@ struct AttnParams {
     float *part_ml;
     __nv_bfloat16 *out;
     int B, Nmax, Hq, Hkv, G, Smax, chunks, npc, n_items, nk_slots, nv_slots;
+    int lanes;  // CTAs per lock-step group (schedule_kernel); 1 = plain stream-K over items
     float scale_log2;
     unsigned long long *trace;  // optional per-tile timestamps (debug), nullptr in production
     int debug_flags;            // experiments only: 1 = skip K/V TMA, 2 = skip MMAs (results invalid)

@@ -43,6 +43,8 @@ struct WsLayout {
     int npc;            // tree nodes per chunk = nt / G
     int chunks;         // chunks per (b, kv-head) item = ceil(Nmax / npc)
     int n_items;        // B * Hkv * chunks
+    int lanes;          // CTAs sharing one KV stream in lock-step (rows kernel: chunks; else 1)
+    int grid;           // attention CTAs: the largest multiple of `lanes` <= the SM count
     int max_ctas;
 };
 
@@ -68,6 +70,8 @@ inline WsLayout ws_layout(const specinfer_shape_t &s, int num_sms) {
     w.npc = w.nt / G;
     w.chunks = (N + w.npc - 1) / w.npc;
     w.n_items = B * s.num_kv_heads * w.chunks;
+    w.lanes = (w.nt == kRowsBlock && w.chunks > 1 && 2 * w.chunks <= num_sms) ? w.chunks : 1;
+    w.grid = (num_sms / w.lanes) * w.lanes;
     w.max_ctas = num_sms * kMaxCtasPerSm;
     size_t o = 0;
     auto take = [&](size_t bytes) { size_t r = o; o = align256(o + bytes); return r; };
@@ -161,6 +165,12 @@ __device__ __forceinline__ void named_bar_sync(uint32_t id, uint32_t nthreads) {
 // ---- TMA ---------------------------------------------------------------------------------
 __device__ __forceinline__ void tma_prefetch_desc(const CUtensorMap *map) {
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(map)) : "memory");
+}
+
+__device__ __forceinline__ uint64_t l2_evict_normal_policy() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
 }
 
 __device__ __forceinline__ uint64_t l2_evict_first_policy() {

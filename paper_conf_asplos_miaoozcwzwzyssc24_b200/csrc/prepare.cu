@@ -95,17 +95,25 @@ __global__ void __launch_bounds__(256) tree_validate_bitsets_kernel(
     }
 }
 
-// Single block: tiles per item, exclusive scan, total; zero the split/verify counters.
+// Single block: tiles per schedule unit, exclusive scan, total; zero the split/verify counters.
+// A unit is one item (lanes == 1) or the `lanes` row chunks of one (b, kv-head) (lanes == chunks,
+// the rows-as-M kernel).  In lane mode CTA c runs chunk c % lanes of every unit in its tile range
+// [t0, t1) of the unit stream, so the `lanes` CTAs of a group read the same KV tile at about the
+// same time: one HBM read, the other chunks hit L2.
 __global__ void __launch_bounds__(1024) schedule_kernel(
     const int32_t *__restrict__ prefix_len, const int32_t *__restrict__ n_nodes,
-    const int32_t *__restrict__ req_ok, int B, int Hkv, int chunks, int npc,
+    const int32_t *__restrict__ req_ok, int B, int Hkv, int chunks, int npc, int lanes,
     int32_t *__restrict__ item_start, uint32_t *__restrict__ item_cnt, int4 *__restrict__ item_info,
     int4 *__restrict__ cta_info, int num_ctas, uint32_t *__restrict__ verify_cnt, int32_t *__restrict__ status) {
     const int n_items = B * Hkv * chunks;
-    const int per = (n_items + blockDim.x - 1) / blockDim.x;
+    const int n_units = n_items / lanes;
+    const int per = (n_units + blockDim.x - 1) / blockDim.x;
     const int lo = threadIdx.x * per;
-    const int hi = min(n_items, lo + per);
-    auto tiles_of = [&](int x) -> int {
+    const int hi = min(n_units, lo + per);
+    // tiles of unit u: a unit's chunks share its KV stream; an empty chunk (c * npc >= n) of a
+    // lane-mode unit keeps the unit's tile range and is skipped by its CTAs (n field 0)
+    auto tiles_of = [&](int u) -> int {
+        const int x = u * lanes;
         const int c = x % chunks;
         const int b = x / (chunks * Hkv);
         if (!req_ok[b]) return 0;
@@ -114,7 +122,7 @@ __global__ void __launch_bounds__(1024) schedule_kernel(
         return (prefix_len[b] + n + kKeyTile - 1) / kKeyTile;
     };
     int local = 0;
-    for (int x = lo; x < hi; ++x) local += tiles_of(x);
+    for (int u = lo; u < hi; ++u) local += tiles_of(u);
     // block exclusive scan of per-thread sums
     __shared__ int s_warp[32];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -137,35 +145,43 @@ __global__ void __launch_bounds__(1024) schedule_kernel(
     }
     __syncthreads();
     int run = v - local + (wid > 0 ? s_warp[wid - 1] : 0);
-    for (int x = lo; x < hi; ++x) {
-        const int tl = tiles_of(x);
-        const int b = x / (chunks * Hkv);
-        item_start[x] = run;
-        item_info[x] = make_int4(run, run + tl, prefix_len[b], n_nodes[b]);
+    for (int u = lo; u < hi; ++u) {
+        const int tl = tiles_of(u);
+        item_start[u] = run;
+        for (int x = u * lanes; x < (u + 1) * lanes; ++x) {
+            const int b = x / (chunks * Hkv);
+            const int c = x % chunks;
+            const int n = n_nodes[b];
+            const bool empty = lanes > 1 && c * npc >= n;
+            item_info[x] = make_int4(run, run + tl, prefix_len[b], empty ? 0 : n);
+            item_cnt[x] = 0u;
+        }
         run += tl;
-        item_cnt[x] = 0u;
     }
     __shared__ int s_total;
     if (threadIdx.x == blockDim.x - 1) {
-        item_start[n_items] = run;
+        item_start[n_units] = run;
         item_info[n_items] = make_int4(run, run, 0, 0);
         status[1] = run;
         s_total = run;
     }
     for (int b = threadIdx.x; b < 2 * B; b += blockDim.x) verify_cnt[b] = 0u;
     __syncthreads();
-    // per-CTA slice [t0, t1) of the tile sequence for the attention grid, and its first item
+    // per-CTA slice [t0, t1) of the unit tile sequence, and its first item
     const long long T = s_total;
+    const int NCv = num_ctas / lanes;
     for (int c = threadIdx.x; c < num_ctas; c += blockDim.x) {
-        const int t0 = (int)((long long)c * T / num_ctas);
-        const int t1 = (int)((long long)(c + 1) * T / num_ctas);
-        int lo2 = 0, hi2 = n_items;  // last item with start <= t0
+        const int vc = c / lanes, cl = c % lanes;
+        const int t0 = (int)((long long)vc * T / NCv);
+        const int t1 = (int)((long long)(vc + 1) * T / NCv);
+        int lo2 = 0, hi2 = n_units;  // last unit with start <= t0
         while (hi2 - lo2 > 1) {
             const int mid = (lo2 + hi2) >> 1;
             if (item_start[mid] <= t0) lo2 = mid; else hi2 = mid;
         }
-        cta_info[2 * c] = make_int4(t0, t1, lo2, (int)T);
-        cta_info[2 * c + 1] = lo2 < n_items ? item_info[lo2] : make_int4(0, 0, 0, 0);
+        const int x0 = lo2 * lanes + cl;
+        cta_info[2 * c] = make_int4(t0, t1, x0, (int)T);
+        cta_info[2 * c + 1] = x0 < n_items ? item_info[x0] : make_int4(0, 0, 0, 0);
     }
 }
 
@@ -185,7 +201,7 @@ cudaError_t launch_tree_prepare(const specinfer_shape_t &s, const WsLayout &w,
     if (e != cudaSuccess) return e;
     schedule_kernel<<<1, 1024, 0, stream>>>(
         prefix_len, n_nodes, reinterpret_cast<int32_t *>(ws + w.req_ok), s.batch,
-        s.num_kv_heads, w.chunks, w.npc, reinterpret_cast<int32_t *>(ws + w.item_start),
+        s.num_kv_heads, w.chunks, w.npc, w.lanes, reinterpret_cast<int32_t *>(ws + w.item_start),
         reinterpret_cast<uint32_t *>(ws + w.item_cnt), reinterpret_cast<int4 *>(ws + w.item_info),
         reinterpret_cast<int4 *>(ws + w.cta_info), num_ctas, reinterpret_cast<uint32_t *>(ws + w.verify_cnt), status);
     return cudaGetLastError();

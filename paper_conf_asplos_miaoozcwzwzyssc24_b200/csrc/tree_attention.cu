@@ -726,6 +726,7 @@ cudaError_t launch_tree_attention(const specinfer_shape_t &s, const WsLayout &w,
     prm.chunks = w.chunks;
     prm.npc = w.npc;
     prm.n_items = w.n_items;
+    prm.lanes = w.lanes;
     const float sm_scale = s.sm_scale > 0.f ? s.sm_scale : 1.0f / sqrtf((float)s.head_dim);
     prm.scale_log2 = sm_scale * 1.4426950408889634f;
     prm.trace = g_attn_trace;

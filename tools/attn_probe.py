@@ -25,8 +25,12 @@ def main():
     ap.add_argument("--prefix", type=int, default=None)
     ap.add_argument("--iters", type=int, default=20)
     ap.add_argument("--trace", action="store_true")
+    ap.add_argument("--raw", action="store_true", help="with --trace: print the raw per-tile events")
+    ap.add_argument("--lib", default=None, help="load this libspecinfer build instead (A/B experiments)")
     ap.add_argument("--flags", type=int, default=0, help="debug flags: 1 skip TMA, 2 skip MMA (timing only)")
     a = ap.parse_args()
+    if a.lib:
+        spi.load_library(a.lib)
     cfg = W.CONFIGS[a.config]
     dev = torch.device("cuda:0")
     B = a.batch or cfg.batch
@@ -73,6 +77,14 @@ def main():
               f"first K issue median {np.median(kt[:,2]-t0)/1e3:.2f} max {(kt[:,2].max()-t0)/1e3:.2f}; "
               f"exit min {(kt[:,1].min()-t0)/1e3:.2f} median {np.median(kt[:,1]-t0)/1e3:.2f} max {(kt[:,1].max()-t0)/1e3:.2f}")
         names = ["K-iss", "V-iss", "S-mma", "PV-mma", "sm-beg", "P-rdy", "epi-PV", "epi-end", "epi-st", "epi-ld", "seg-beg"]
+        if a.raw:
+            for c in range(2):
+                x = t[c]
+                base = x[0, 0]
+                print(f"CTA {c} raw events (cycles rel. to first K issue): 0 K-iss 1 V-iss 2 S-mma 3 PV-mma 4/5 sm-beg g0/g1 6/7 P-rdy g0/g1 8 epi 9 epi-end")
+                for i in range(40):
+                    print(f"{i:3d} " + " ".join(f"{(v - base) if v else -1:8d}" for v in x[i, :10]))
+            return
         for c in range(2):
             x = t[c]
             nv = int((x[:, 4] > 0).sum())
