@@ -9,6 +9,9 @@
  *   specinfer_verify_greedy   Alg. 2 VerifyGreedy L395-401; §4.3
  *   specinfer_verify_mss      Alg. 2 VerifyStochastic L403-425; Fig. 5; Thm 4.2
  *   specinfer_kv_commit       depth-first KV-cache update L635-644; tree-topology KV layout L659-661
+ *   specinfer_verify_ns       NEXT-3: naive sampling, the baseline of Theorem 4.3 (L747-765)
+ *   specinfer_leaf_paths,     NEXT-1 baseline: sequence-based parallel decoding (§4.2,
+ *   specinfer_sequence_pack   Fig. 4 left L682, §6.5)
  * Readings of the paper where it is silent or garbled are numbered R1..R23 in DESIGN.md.
  *
  * General conventions
@@ -131,6 +134,53 @@ specinfer_status_t specinfer_verify_mss(const specinfer_shape_t *shape, const fl
                                         const int32_t *request_ids, int32_t *accepted_nodes,
                                         int32_t *accepted_tokens, int32_t *n_accepted,
                                         void *workspace, specinfer_stream_t stream);
+
+/* NEXT-3: naive sampling (NS), the verifier Theorem 4.3 compares MSS with (L747-765): at each
+ * node u on the walk draw x ~ softmax(logits[u]/temperature) by the exponential race of
+ * verify_mss step 4 at round 0 (same Philox counters, so a leaf draws the same token under both
+ * verifiers); if a child of u carries token x (lowest index, R7) append it and continue, else
+ * emit x and stop.  Outputs, workspace and error behaviour as verify_greedy. */
+specinfer_status_t specinfer_verify_ns(const specinfer_shape_t *shape, const float *logits,
+                                       const int32_t *tree_tokens, const int32_t *parent,
+                                       const int32_t *n_nodes, float temperature, uint64_t seed,
+                                       uint64_t offset, const int32_t *request_ids,
+                                       int32_t *accepted_nodes, int32_t *accepted_tokens,
+                                       int32_t *n_accepted, void *workspace,
+                                       specinfer_stream_t stream);
+
+/* NEXT-1: sequence-based parallel decoding, the baseline tree-based decoding replaces (§4.2
+ * L622-632, Fig. 4 left L682, §6.5).  Not part of the hot path; used by the Fig. 11
+ * ablation and by the tests that check tree attention == per-sequence causal attention.
+ *
+ * specinfer_leaf_paths: for each request, its leaves in node-index order (= DFS order for a
+ * DFS-linearised tree) and their root paths: paths[b][r][0..len-1] = root..leaf node ids of
+ * the r-th leaf (-1 padded), path_len[b][r] = depth(leaf) + 1 (0 for r >= n_leaves[b]).
+ * Layouts: paths int32 [B][Nmax][Dmax+1], path_len int32 [B][Nmax], n_leaves int32 [B].
+ * Invalid trees (bad parent / n_nodes, depth > Dmax): n_leaves[b] = 0 and, when `workspace`
+ * is not NULL, the sticky BAD_TREE bit is set in it.  No other state is used. */
+specinfer_status_t specinfer_leaf_paths(const specinfer_shape_t *shape, const int32_t *parent,
+                                        const int32_t *n_nodes, int32_t *paths, int32_t *path_len,
+                                        int32_t *n_leaves, void *workspace, specinfer_stream_t stream);
+
+/* specinfer_sequence_pack: builds the sequence batch of sequence-based decoding for ONE layer.
+ * Sequence s (0 <= s < num_seqs) is leaf seq_map[s][1] of request seq_map[s][0] (int32 [S][2],
+ * host-chosen, e.g. all (b, r) with r < n_leaves[b]).  Writes, for every kv-head g:
+ *   k_seq/v_seq [S][Hkv][seq_max_seq][128]: slots [0, P_b) = the request's committed prefix,
+ *       slot P_b + j = the tree slot P_b + path[j] (its own cache, "a different key-value cache
+ *       for each sequence", L627-628); seq_max_seq >= P_b + path_len;
+ *   q_seq [S][Dmax+1][Hq][128]: row j = q of node path[j];
+ *   seq_parent/seq_depth int32 [S][Dmax+1]: the chain j-1 / j; seq_prefix_len, seq_n_nodes
+ *       int32 [S]: P_b and path_len.
+ * The result is a valid input of specinfer_tree_prepare / specinfer_tree_attention with
+ * shape {batch = S, max_nodes = Dmax+1, max_seq = seq_max_seq, heads as `shape`}. */
+specinfer_status_t specinfer_sequence_pack(const specinfer_shape_t *shape, int32_t num_seqs,
+                                           int32_t seq_max_seq, const int32_t *seq_map,
+                                           const int32_t *paths, const int32_t *path_len,
+                                           const int32_t *prefix_len, const void *q,
+                                           const void *k_cache, const void *v_cache, void *q_seq,
+                                           void *k_seq, void *v_seq, int32_t *seq_parent,
+                                           int32_t *seq_depth, int32_t *seq_prefix_len,
+                                           int32_t *seq_n_nodes, specinfer_stream_t stream);
 
 /* a6 (K6).  Depth-first KV-cache commit (L635-644): for every layer l < L, request b with
  * n = n_accepted[b] > 0 and kv-head g: slot P_b + j <- old slot P_b + accepted_nodes[b][j]

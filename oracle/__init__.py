@@ -47,6 +47,8 @@ def lib():
                                               vp, vp, vp, vp]
         _lib.oracle_verify_mss.argtypes = [i32, i32, i32, i32, i32, i32, vp, vp, vp, vp, vp, vp,
                                            vp, dbl, u64, u64, vp, vp, vp, vp, vp]
+        _lib.oracle_verify_ns.argtypes = [i32, i32, i32, i32, i32, i32, vp, vp, vp, vp, vp, vp,
+                                          dbl, u64, u64, vp, vp, vp, vp, vp]
         _lib.oracle_philox4x32_10.argtypes = [vp, vp, vp]
     return _lib
 
@@ -149,9 +151,58 @@ def verify_mss(logits, tree_tokens, parent, n_nodes, draft_probs, *, temperature
     return an, at, na, mg
 
 
+def verify_ns(logits, tree_tokens, parent, n_nodes, *, temperature=1.0, seed=0, offset=0, request_ids=None,
+              depth=None, prefix_len=None, smax=1 << 30, max_depth=255, path_len=None):
+    """NEXT-3 naive sampling (L747-753, the baseline of Theorem 4.3): x ~ p at each node by the
+    exponential race (c4's counters at round 0); follow the child with token x, else stop.
+    Returns (accepted_nodes, accepted_tokens, n_accepted, margin)."""
+    logits = _c(logits, np.float32)
+    B, Nmax, V = logits.shape
+    path_len = path_len or (max_depth + 1 if max_depth < 255 else Nmax + 1)
+    an = np.empty((B, path_len), np.int32)
+    at = np.empty((B, path_len), np.int32)
+    na = np.empty((B,), np.int32)
+    mg = np.empty((B,), np.float64)
+    rids = None if request_ids is None else _c(request_ids, np.int32)
+    lib().oracle_verify_ns(B, Nmax, V, smax, max_depth, path_len, _p(logits), _p(_c(tree_tokens, np.int32)),
+                           _p(_c(parent, np.int32)), _p(None if depth is None else _c(depth, np.int32)),
+                           _p(None if prefix_len is None else _c(prefix_len, np.int32)),
+                           _p(_c(n_nodes, np.int32)), float(temperature), int(seed) & (2**64 - 1),
+                           int(offset) & (2**64 - 1), _p(rids), _p(an), _p(at), _p(na), _p(mg))
+    return an, at, na, mg
+
+
 def philox4x32_10(ctr, key) -> np.ndarray:
     c = _c(ctr, np.uint32)
     k = _c(key, np.uint32)
     o = np.empty(4, np.uint32)
     lib().oracle_philox4x32_10(_p(c), _p(k), _p(o))
     return o
+
+
+def leaf_paths(parent, n_nodes):
+    """NEXT-1 (sequence-based decoding, §4.2, Fig. 4 left L682): the token
+    tree decomposed into its root-to-leaf token sequences.  For each request: the leaves (nodes
+    without children) in node-index order, each with the node ids of its path root .. leaf.
+    Plain Python, literally the definition (a leaf is a node no other node names as parent;
+    its sequence is the chain of parents up to the root).  Returns a list (per request) of lists
+    of paths; an invalid tree (parent[0] != -1 or parent[i] not in [0, i)) gives None."""
+    parent = np.asarray(parent)
+    out = []
+    for b in range(parent.shape[0]):
+        n = int(n_nodes[b])
+        par = [int(x) for x in parent[b, :n]]
+        if n < 1 or par[0] != -1 or any(not (0 <= par[i] < i) for i in range(1, n)):
+            out.append(None)
+            continue
+        has_child = set(par[1:])
+        paths = []
+        for leaf in range(n):
+            if leaf in has_child:
+                continue
+            path = [leaf]
+            while par[path[-1]] != -1:
+                path.append(par[path[-1]])
+            paths.append(path[::-1])
+        out.append(paths)
+    return out

@@ -30,7 +30,8 @@ EXPORTED_SYMBOLS = (
     "specinfer_verify_greedy", "specinfer_verify_mss", "specinfer_kv_commit",
     "specinfer_read_device_status", "specinfer_philox_debug", "specinfer_debug_set_trace",
     "specinfer_launches_per_call",
-    "specinfer_status_string",
+    "specinfer_status_string", "specinfer_leaf_paths", "specinfer_sequence_pack",
+    "specinfer_verify_ns",
 )
 
 
@@ -79,6 +80,9 @@ def load_library(path: str = LIB_PATH):
     lib.specinfer_kv_commit.argtypes = [sp, vp, vp, vp, vp, vp, vp]
     lib.specinfer_read_device_status.argtypes = [vp, vp, ctypes.POINTER(i32)]
     lib.specinfer_philox_debug.argtypes = [vp, vp, i32, vp]
+    lib.specinfer_verify_ns.argtypes = [sp, vp, vp, vp, vp, f32, u64, u64, vp, vp, vp, vp, vp, vp]
+    lib.specinfer_leaf_paths.argtypes = [sp, vp, vp, vp, vp, vp, vp, vp]
+    lib.specinfer_sequence_pack.argtypes = [sp, i32, i32] + [vp] * 14 + [vp]
     lib.specinfer_debug_set_trace.argtypes = [vp]
     lib.specinfer_debug_set_trace.restype = None
     lib.specinfer_launches_per_call.argtypes = [ctypes.c_char_p]
@@ -87,7 +91,7 @@ def load_library(path: str = LIB_PATH):
     lib.specinfer_status_string.restype = ctypes.c_char_p
     for name in ("specinfer_tree_prepare", "specinfer_tree_attention", "specinfer_verify_greedy",
                  "specinfer_verify_mss", "specinfer_kv_commit", "specinfer_read_device_status",
-                 "specinfer_philox_debug"):
+                 "specinfer_philox_debug", "specinfer_leaf_paths", "specinfer_sequence_pack", "specinfer_verify_ns"):
         getattr(lib, name).restype = i32
     _lib = lib
     return lib
@@ -201,6 +205,27 @@ def specinfer_verify_mss(shape: Shape, logits, tree_tokens, parent, n_nodes, dra
                                                _stream(logits)))
 
 
+def specinfer_verify_ns(shape: Shape, logits, tree_tokens, parent, n_nodes, temperature, seed, offset, request_ids,
+                        accepted_nodes, accepted_tokens, n_accepted, workspace):
+    """NEXT-3 naive sampling (L747-753), see include/specinfer.h."""
+    dev = logits.device
+    B, N, V, Lp = shape.batch, shape.max_nodes, shape.vocab, shape.max_depth + 1
+    if not (temperature > 0):
+        raise ValueError("temperature must be > 0")
+    a = (_req("logits", logits, torch.float32, (B, N, V), dev),
+         _req("tree_tokens", tree_tokens, torch.int32, (B, N), dev),
+         _req("parent", parent, torch.int32, (B, N), dev), _req("n_nodes", n_nodes, torch.int32, (B,), dev))
+    rid = _opt("request_ids", request_ids, torch.int32, (B,), dev)
+    o = (_req("accepted_nodes", accepted_nodes, torch.int32, (B, Lp), dev),
+         _req("accepted_tokens", accepted_tokens, torch.int32, (B, Lp), dev),
+         _req("n_accepted", n_accepted, torch.int32, (B,), dev),
+         _req("workspace", workspace, torch.uint8, None, dev))
+    _check("specinfer_verify_ns",
+           load_library().specinfer_verify_ns(ctypes.byref(shape), *a, ctypes.c_float(temperature),
+                                              ctypes.c_uint64(int(seed) & (2**64 - 1)),
+                                              ctypes.c_uint64(int(offset) & (2**64 - 1)), rid, *o, _stream(logits)))
+
+
 def specinfer_kv_commit(shape: Shape, k_cache_all, v_cache_all, prefix_len, accepted_nodes, n_accepted):
     dev = k_cache_all.device
     B, Lp = shape.batch, shape.max_depth + 1
@@ -236,6 +261,43 @@ def specinfer_philox_debug(ctr_key: torch.Tensor) -> torch.Tensor:
     return out.to(torch.int64).bitwise_and(0xFFFFFFFF)
 
 
+def specinfer_leaf_paths(shape: Shape, parent, n_nodes, paths, path_len, n_leaves, workspace=None):
+    """NEXT-1: leaves (node-index order) and their root paths, see include/specinfer.h."""
+    dev = parent.device
+    B, N, Lp = shape.batch, shape.max_nodes, shape.max_depth + 1
+    args = (_req("parent", parent, torch.int32, (B, N), dev), _req("n_nodes", n_nodes, torch.int32, (B,), dev),
+            _req("paths", paths, torch.int32, (B, N, Lp), dev), _req("path_len", path_len, torch.int32, (B, N), dev),
+            _req("n_leaves", n_leaves, torch.int32, (B,), dev),
+            _opt("workspace", workspace, torch.uint8, None, dev))
+    _check("specinfer_leaf_paths", load_library().specinfer_leaf_paths(ctypes.byref(shape), *args, _stream(parent)))
+
+
+def specinfer_sequence_pack(shape: Shape, seq_map, paths, path_len, prefix_len, q, k_cache, v_cache, q_seq, k_seq,
+                            v_seq, seq_parent, seq_depth, seq_prefix_len, seq_n_nodes):
+    """NEXT-1: the per-sequence caches / queries / chain trees of sequence-based decoding (one
+    layer), see include/specinfer.h."""
+    dev = q.device
+    B, N, Hq, Hkv, S, Lp = (shape.batch, shape.max_nodes, shape.num_q_heads, shape.num_kv_heads, shape.max_seq,
+                            shape.max_depth + 1)
+    ns = int(seq_map.shape[0])
+    sms = int(k_seq.shape[2])
+    args = (_req("seq_map", seq_map, torch.int32, (ns, 2), dev), _req("paths", paths, torch.int32, (B, N, Lp), dev),
+            _req("path_len", path_len, torch.int32, (B, N), dev),
+            _req("prefix_len", prefix_len, torch.int32, (B,), dev),
+            _req("q", q, torch.bfloat16, (B, N, Hq, 128), dev),
+            _req("k_cache", k_cache, torch.bfloat16, (B, Hkv, S, 128), dev),
+            _req("v_cache", v_cache, torch.bfloat16, (B, Hkv, S, 128), dev),
+            _req("q_seq", q_seq, torch.bfloat16, (ns, Lp, Hq, 128), dev),
+            _req("k_seq", k_seq, torch.bfloat16, (ns, Hkv, sms, 128), dev),
+            _req("v_seq", v_seq, torch.bfloat16, (ns, Hkv, sms, 128), dev),
+            _req("seq_parent", seq_parent, torch.int32, (ns, Lp), dev),
+            _req("seq_depth", seq_depth, torch.int32, (ns, Lp), dev),
+            _req("seq_prefix_len", seq_prefix_len, torch.int32, (ns,), dev),
+            _req("seq_n_nodes", seq_n_nodes, torch.int32, (ns,), dev))
+    _check("specinfer_sequence_pack", load_library().specinfer_sequence_pack(
+        ctypes.byref(shape), ns, sms, *args, _stream(q)))
+
+
 def specinfer_debug_set_trace(trace: Optional[torch.Tensor]):
     """Debug only: per-tile timestamps of tree_attention CTAs 0-7 into `trace` (int64 [8][64][8])."""
     load_library().specinfer_debug_set_trace(None if trace is None else ctypes.c_void_p(trace.data_ptr()))
@@ -269,3 +331,71 @@ class TreeState:
     def attention(self, q, k, v, out):
         specinfer_tree_attention(self.shape, q, k, v, self.parent, self.depth, self.prefix_len, self.n_nodes,
                                  out, self.workspace)
+
+
+# ------------------------------------------------------------------------------------------
+# NEXT-1: sequence-based parallel decoding (the baseline of PAPER.md §4.2 / Fig. 4 left)
+# ------------------------------------------------------------------------------------------
+
+class SequenceBaseline:
+    """Sequence-based parallel decoding of a tree batch (Fig. 4 left, §6.5):
+    every root-to-leaf sequence gets its own KV cache (committed prefix + its own tokens) and is
+    decoded as a causal chain.  `build()` decomposes the trees and packs one layer's caches
+    (specinfer_leaf_paths + specinfer_sequence_pack); `attention()` runs all sequences in one
+    tree_attention launch over chain trees, or one launch per sequence (`per_sequence=True`,
+    Fig. 4's Kernel 1/2/3).  Only the host reads n_leaves (once, to size the sequence batch)."""
+
+    def __init__(self, shape: Shape, parent, depth, prefix_len, n_nodes):
+        dev = parent.device
+        B, N, Lp = shape.batch, shape.max_nodes, shape.max_depth + 1
+        self.tree_shape = shape
+        self.prefix_len = prefix_len
+        self.paths = torch.empty((B, N, Lp), dtype=torch.int32, device=dev)
+        self.path_len = torch.empty((B, N), dtype=torch.int32, device=dev)
+        self.n_leaves = torch.empty((B,), dtype=torch.int32, device=dev)
+        specinfer_leaf_paths(shape, parent, n_nodes, self.paths, self.path_len, self.n_leaves)
+        nl = self.n_leaves.cpu().tolist()
+        self.seq_map = torch.tensor([(b, r) for b in range(B) for r in range(nl[b])], dtype=torch.int32,
+                                    device=dev).reshape(-1, 2)
+        ns = int(self.seq_map.shape[0])
+        self.num_seqs = ns
+        pmax = int(prefix_len.max().item())
+        self.seq_max_seq = pmax + Lp
+        Hq, Hkv = shape.num_q_heads, shape.num_kv_heads
+        self.shape = make_shape(ns, Lp, Hq, Hkv, self.seq_max_seq, max_depth=shape.max_depth,
+                                sm_scale=shape.sm_scale)
+        self.q = torch.empty((ns, Lp, Hq, 128), dtype=torch.bfloat16, device=dev)
+        self.k = torch.empty((ns, Hkv, self.seq_max_seq, 128), dtype=torch.bfloat16, device=dev)
+        self.v = torch.empty_like(self.k)
+        self.out = torch.empty_like(self.q)
+        self.parent = torch.empty((ns, Lp), dtype=torch.int32, device=dev)
+        self.depth = torch.empty_like(self.parent)
+        self.seq_prefix = torch.empty((ns,), dtype=torch.int32, device=dev)
+        self.seq_n = torch.empty_like(self.seq_prefix)
+        self.state = None
+        self.singles = None  # per-sequence states (per_sequence=True), prepared once
+
+    def build(self, q, k_cache, v_cache):
+        specinfer_sequence_pack(self.tree_shape, self.seq_map, self.paths, self.path_len, self.prefix_len, q,
+                                k_cache, v_cache, self.q, self.k, self.v, self.parent, self.depth, self.seq_prefix,
+                                self.seq_n)
+        if self.state is None:
+            self.state = TreeState.create(self.shape, self.parent, self.depth, self.seq_prefix, self.seq_n)
+        self.state.prepare()
+
+    def attention(self, per_sequence: bool = False):
+        if not per_sequence:
+            self.state.attention(self.q, self.k, self.v, self.out)
+            return self.out
+        if self.singles is None:
+            s1 = make_shape(1, self.shape.max_nodes, self.shape.num_q_heads, self.shape.num_kv_heads,
+                            self.seq_max_seq, max_depth=self.shape.max_depth, sm_scale=self.shape.sm_scale)
+            self.singles = []
+            for s in range(self.num_seqs):
+                st = TreeState.create(s1, self.parent[s:s + 1], self.depth[s:s + 1], self.seq_prefix[s:s + 1],
+                                      self.seq_n[s:s + 1])
+                st.prepare()
+                self.singles.append(st)
+        for s, st in enumerate(self.singles):
+            st.attention(self.q[s:s + 1], self.k[s:s + 1], self.v[s:s + 1], self.out[s:s + 1])
+        return self.out

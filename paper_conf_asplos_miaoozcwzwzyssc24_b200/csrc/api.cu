@@ -26,8 +26,20 @@ cudaError_t launch_verify_mss(const specinfer_shape_t &s, const WsLayout &w, con
                               const float *draft_probs, float temperature, uint64_t seed, uint64_t offset,
                               const int32_t *request_ids, int32_t *acc_nodes, int32_t *acc_tokens,
                               int32_t *n_acc, char *ws, cudaStream_t stream);
+cudaError_t launch_verify_ns(const specinfer_shape_t &s, const WsLayout &w, const float *logits,
+                             const int32_t *tree_tokens, const int32_t *parent, const int32_t *n_nodes,
+                             float temperature, uint64_t seed, uint64_t offset, const int32_t *request_ids,
+                             int32_t *acc_nodes, int32_t *acc_tokens, int32_t *n_acc, char *ws, cudaStream_t stream);
 cudaError_t launch_kv_commit(const specinfer_shape_t &s, void *k_all, void *v_all, int32_t *prefix_len,
                              const int32_t *acc_nodes, const int32_t *n_acc, cudaStream_t stream);
+cudaError_t launch_leaf_paths(const specinfer_shape_t &s, const int32_t *parent, const int32_t *n_nodes,
+                              int32_t *paths, int32_t *path_len, int32_t *n_leaves, int32_t *status,
+                              cudaStream_t stream);
+cudaError_t launch_sequence_pack(const specinfer_shape_t &s, int num_seqs, int seq_max_seq, const int32_t *seq_map,
+                                 const int32_t *paths, const int32_t *path_len, const int32_t *prefix_len,
+                                 const void *q, const void *k, const void *v, void *q_seq, void *k_seq, void *v_seq,
+                                 int32_t *seq_parent, int32_t *seq_depth, int32_t *seq_prefix, int32_t *seq_n,
+                                 cudaStream_t stream);
 cudaError_t launch_philox_debug(const uint32_t *ck, uint32_t *out, int n, cudaStream_t stream);
 extern unsigned long long *g_attn_trace;
 extern int g_attn_debug_flags;
@@ -181,6 +193,25 @@ specinfer_status_t specinfer_verify_mss(const specinfer_shape_t *shape, const fl
                                        reinterpret_cast<char *>(workspace), (cudaStream_t)stream));
 }
 
+specinfer_status_t specinfer_verify_ns(const specinfer_shape_t *shape, const float *logits,
+                                       const int32_t *tree_tokens, const int32_t *parent, const int32_t *n_nodes,
+                                       float temperature, uint64_t seed, uint64_t offset,
+                                       const int32_t *request_ids, int32_t *accepted_nodes,
+                                       int32_t *accepted_tokens, int32_t *n_accepted, void *workspace,
+                                       specinfer_stream_t stream) {
+    SPI_TRY(check_shape(shape));
+    if (shape->vocab < 1 || !(temperature > 0.f) || !isfinite(temperature)) return SPECINFER_ERR_INVALID_ARG;
+    if (!logits || !tree_tokens || !parent || !n_nodes || !accepted_nodes || !accepted_tokens || !n_accepted)
+        return SPECINFER_ERR_INVALID_ARG;
+    SPI_TRY(check_ws(workspace));
+    DeviceInfo d;
+    SPI_TRY(check_device(&d));
+    const WsLayout w = ws_layout(*shape, d.num_sms);
+    return from_cuda(launch_verify_ns(*shape, w, logits, tree_tokens, parent, n_nodes, temperature, seed, offset,
+                                      request_ids, accepted_nodes, accepted_tokens, n_accepted,
+                                      reinterpret_cast<char *>(workspace), (cudaStream_t)stream));
+}
+
 specinfer_status_t specinfer_kv_commit(const specinfer_shape_t *shape, void *k_cache_all, void *v_cache_all,
                                        int32_t *prefix_len, const int32_t *accepted_nodes, const int32_t *n_accepted,
                                        specinfer_stream_t stream) {
@@ -194,6 +225,40 @@ specinfer_status_t specinfer_kv_commit(const specinfer_shape_t *shape, void *k_c
     SPI_TRY(check_device(&d));
     return from_cuda(launch_kv_commit(*shape, k_cache_all, v_cache_all, prefix_len, accepted_nodes, n_accepted,
                                       (cudaStream_t)stream));
+}
+
+specinfer_status_t specinfer_leaf_paths(const specinfer_shape_t *shape, const int32_t *parent,
+                                        const int32_t *n_nodes, int32_t *paths, int32_t *path_len,
+                                        int32_t *n_leaves, void *workspace, specinfer_stream_t stream) {
+    SPI_TRY(check_shape(shape));
+    if (!parent || !n_nodes || !paths || !path_len || !n_leaves) return SPECINFER_ERR_INVALID_ARG;
+    if (workspace) SPI_TRY(check_ws(workspace));
+    DeviceInfo d;
+    SPI_TRY(check_device(&d));
+    return from_cuda(launch_leaf_paths(*shape, parent, n_nodes, paths, path_len, n_leaves,
+                                       reinterpret_cast<int32_t *>(workspace), (cudaStream_t)stream));
+}
+
+specinfer_status_t specinfer_sequence_pack(const specinfer_shape_t *shape, int32_t num_seqs, int32_t seq_max_seq,
+                                           const int32_t *seq_map, const int32_t *paths, const int32_t *path_len,
+                                           const int32_t *prefix_len, const void *q, const void *k_cache,
+                                           const void *v_cache, void *q_seq, void *k_seq, void *v_seq,
+                                           int32_t *seq_parent, int32_t *seq_depth, int32_t *seq_prefix_len,
+                                           int32_t *seq_n_nodes, specinfer_stream_t stream) {
+    SPI_TRY(check_shape(shape));
+    if (num_seqs < 0 || seq_max_seq < 1) return SPECINFER_ERR_INVALID_ARG;
+    if (num_seqs > 0 && (!seq_map || !paths || !path_len || !prefix_len || !q || !k_cache || !v_cache || !q_seq ||
+                         !k_seq || !v_seq || !seq_parent || !seq_depth || !seq_prefix_len || !seq_n_nodes))
+        return SPECINFER_ERR_INVALID_ARG;
+    if ((reinterpret_cast<uintptr_t>(q) | reinterpret_cast<uintptr_t>(k_cache) | reinterpret_cast<uintptr_t>(v_cache) |
+         reinterpret_cast<uintptr_t>(q_seq) | reinterpret_cast<uintptr_t>(k_seq) | reinterpret_cast<uintptr_t>(v_seq)) &
+        15u)
+        return SPECINFER_ERR_INVALID_ARG;
+    DeviceInfo d;
+    SPI_TRY(check_device(&d));
+    return from_cuda(launch_sequence_pack(*shape, num_seqs, seq_max_seq, seq_map, paths, path_len, prefix_len, q,
+                                          k_cache, v_cache, q_seq, k_seq, v_seq, seq_parent, seq_depth,
+                                          seq_prefix_len, seq_n_nodes, (cudaStream_t)stream));
 }
 
 specinfer_status_t specinfer_read_device_status(const void *workspace, specinfer_stream_t stream,
@@ -232,6 +297,9 @@ int32_t specinfer_launches_per_call(const char *name) {
     if (!strcmp(name, "verify_greedy")) return 1;    // argmax + walk fused (last CTA walks)
     if (!strcmp(name, "verify_mss")) return 1;
     if (!strcmp(name, "kv_commit")) return 2;        // copy, prefix update
+    if (!strcmp(name, "leaf_paths")) return 1;
+    if (!strcmp(name, "verify_ns")) return 1;         // race-argmax + walk fused (last CTA walks)
+    if (!strcmp(name, "sequence_pack")) return 1;
     return -1;
 }
 

@@ -5,6 +5,10 @@
 // argmax with the lowest index on ties, reading R7); the last CTA of a request (counter in the
 // workspace) walks the tree from the root.  One launch.
 //
+// Naive sampling (NEXT-3, L747-753, the baseline of Theorem 4.3) reuses the K4 kernel: the
+// per-node key is the exponential-race key of x ~ softmax(l / T) instead of the logit, and the
+// walk follows the child whose token equals that sample.
+//
 // VerifyStochastic = MSS (Alg. 2 lines 24-44, L403-425; Fig. 5): also one launch.  Phase 1, one
 // CTA per (node, request): the softmax statistics (max, sum of exp) of logits[u]/T for every
 // node, in parallel.  Phase 2, the last CTA of the request: the sequential walk of Alg. 2.  An
@@ -149,12 +153,53 @@ __device__ MaxSum block_maxsum(MaxSum a, float invT, MaxSum *sh) {
 constexpr int kGreedyThreads = 512;
 constexpr int kUnroll = 8;   // 128-bit loads in flight per thread
 
+__device__ __forceinline__ float lg2f(float x) {
+    float y;
+    asm("lg2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+    return y;
+}
+// E'_k = -log2 U_k = E_k / ln 2 with U_k = ((w >> 9) + 0.5) 2^-23 (c4 step 4); the race argmax of
+// p_k / E_k equals that of p_k / E'_k and of log2 p_k - log2 E'_k.
+__device__ __forceinline__ float race_E2(uint32_t w) {
+    const float U = ((float)(w >> 9) + 0.5f) * (1.0f / 8388608.0f);
+    return -lg2f(U);
+}
+
+// Per-node key of the "argmax then walk" verifiers.  Greedy (K4): the logit itself.  Naive
+// sampling (NEXT-3, L747-753): the exponential-race key of x ~ softmax(l / T) at round 0 with the
+// counters of c4 step 4 (rid, u<<8, (2<<28) | (k>>2), offset), in the log2 domain:
+// l_k c - log2 E'_k with c = log2(e) / T (same draw as MSS's leaf sample).
+struct NsParams {
+    float c;
+    uint32_t seed_lo, seed_hi, off;
+    const int32_t *request_ids;
+};
+
+template <bool kNS>
+__device__ __forceinline__ void key4(ArgMax &a, float4 x, int k4, uint32_t rid, uint32_t u, const NsParams &ns) {
+    const int base = k4 << 2;
+    if (kNS) {
+        const uint4 w = philox4x32_10(make_uint4(rid, u << 8, (2u << 28) | (uint32_t)k4, ns.off),
+                                      make_uint2(ns.seed_lo, ns.seed_hi));
+        a = argmax_merge(a, ArgMax{x.x * ns.c - lg2f(race_E2(w.x)), base});
+        a = argmax_merge(a, ArgMax{x.y * ns.c - lg2f(race_E2(w.y)), base + 1});
+        a = argmax_merge(a, ArgMax{x.z * ns.c - lg2f(race_E2(w.z)), base + 2});
+        a = argmax_merge(a, ArgMax{x.w * ns.c - lg2f(race_E2(w.w)), base + 3});
+    } else {
+        a = argmax_merge(a, ArgMax{x.x, base});
+        a = argmax_merge(a, ArgMax{x.y, base + 1});
+        a = argmax_merge(a, ArgMax{x.z, base + 2});
+        a = argmax_merge(a, ArgMax{x.w, base + 3});
+    }
+}
+
+template <bool kNS>
 __global__ void __launch_bounds__(kGreedyThreads) verify_greedy_kernel(
     const float *__restrict__ logits, const int32_t *__restrict__ tree_tokens,
     const int32_t *__restrict__ parent, const int32_t *__restrict__ n_nodes,
     const int32_t *__restrict__ req_ok, int32_t *__restrict__ argmax_ws,
     uint32_t *__restrict__ counter, int32_t *__restrict__ acc_nodes, int32_t *__restrict__ acc_tokens,
-    int32_t *__restrict__ n_acc, int Nmax, int V, int path_len) {
+    int32_t *__restrict__ n_acc, int Nmax, int V, int path_len, NsParams ns) {
     const int u = blockIdx.x, b = blockIdx.y;
     const int n = n_nodes[b];
     __shared__ ArgMax sh[32];
@@ -170,6 +215,7 @@ __global__ void __launch_bounds__(kGreedyThreads) verify_greedy_kernel(
         return;
     }
     if (u >= n) return;
+    const uint32_t rid = kNS ? (ns.request_ids ? (uint32_t)ns.request_ids[b] : (uint32_t)b) : 0u;
     const float *row = logits + ((size_t)b * Nmax + u) * V;
     ArgMax a{-INFINITY, -1};
     if ((V & 3) == 0) {
@@ -181,24 +227,20 @@ __global__ void __launch_bounds__(kGreedyThreads) verify_greedy_kernel(
 #pragma unroll
             for (int j = 0; j < kUnroll; ++j) x[j] = __ldcs(row4 + i + j * kGreedyThreads);
 #pragma unroll
-            for (int j = 0; j < kUnroll; ++j) {
-                const int base = (i + j * kGreedyThreads) << 2;
-                a = argmax_merge(a, ArgMax{x[j].x, base});
-                a = argmax_merge(a, ArgMax{x[j].y, base + 1});
-                a = argmax_merge(a, ArgMax{x[j].z, base + 2});
-                a = argmax_merge(a, ArgMax{x[j].w, base + 3});
-            }
+            for (int j = 0; j < kUnroll; ++j) key4<kNS>(a, x[j], i + j * kGreedyThreads, rid, u, ns);
         }
-        for (; i < V4; i += kGreedyThreads) {
-            const float4 x = __ldcs(row4 + i);
-            const int base = i << 2;
-            a = argmax_merge(a, ArgMax{x.x, base});
-            a = argmax_merge(a, ArgMax{x.y, base + 1});
-            a = argmax_merge(a, ArgMax{x.z, base + 2});
-            a = argmax_merge(a, ArgMax{x.w, base + 3});
-        }
+        for (; i < V4; i += kGreedyThreads) key4<kNS>(a, __ldcs(row4 + i), i, rid, u, ns);
     } else {
-        for (int i = threadIdx.x; i < V; i += kGreedyThreads) a = argmax_merge(a, ArgMax{__ldcs(row + i), i});
+        for (int i = threadIdx.x; i < V; i += kGreedyThreads) {
+            float key = __ldcs(row + i);
+            if (kNS) {
+                const uint4 w = philox4x32_10(make_uint4(rid, (uint32_t)u << 8, (2u << 28) | (uint32_t)(i >> 2), ns.off),
+                                              make_uint2(ns.seed_lo, ns.seed_hi));
+                const uint32_t ws[4] = {w.x, w.y, w.z, w.w};
+                key = key * ns.c - lg2f(race_E2(ws[i & 3]));
+            }
+            a = argmax_merge(a, ArgMax{key, i});
+        }
     }
     a = block_argmax<kGreedyThreads>(a, sh);
     if (threadIdx.x == 0) {
@@ -261,11 +303,6 @@ constexpr int kMssThreads = 256;
 constexpr int kMssUnroll = 4;
 constexpr int kMssCluster = 8;
 
-__device__ __forceinline__ float lg2f(float x) {
-    float y;
-    asm("lg2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
-    return y;
-}
 __device__ __forceinline__ float rcpf(float x) {
     float y;
     asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
@@ -298,13 +335,6 @@ __device__ __forceinline__ int ld_dsmem_s32(uint32_t a) {
     int v;
     asm volatile("ld.shared::cluster.s32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
     return v;
-}
-
-// E'_k = -log2 U_k = E_k / ln 2 with U_k = ((w >> 9) + 0.5) 2^-23 (c4 step 4); the race argmax of
-// p_k / E_k equals that of p_k / E'_k and of log2 p_k - log2 E'_k.
-__device__ __forceinline__ float race_E2(uint32_t w) {
-    const float U = ((float)(w >> 9) + 0.5f) * (1.0f / 8388608.0f);
-    return -lg2f(U);
 }
 
 // Per-CTA partial results exchanged through DSMEM (double-buffered by reduction parity).
@@ -645,10 +675,24 @@ cudaError_t launch_verify_greedy(const specinfer_shape_t &s, const WsLayout &w, 
                                  int32_t *acc_nodes, int32_t *acc_tokens, int32_t *n_acc, char *ws,
                                  cudaStream_t stream) {
     dim3 grid(s.max_nodes, s.batch);
-    verify_greedy_kernel<<<grid, kGreedyThreads, 0, stream>>>(
+    verify_greedy_kernel<false><<<grid, kGreedyThreads, 0, stream>>>(
         logits, tree_tokens, parent, n_nodes, reinterpret_cast<const int32_t *>(ws + w.req_ok),
         reinterpret_cast<int32_t *>(ws + w.argmax), reinterpret_cast<uint32_t *>(ws + w.verify_cnt), acc_nodes,
-        acc_tokens, n_acc, s.max_nodes, s.vocab, s.max_depth + 1);
+        acc_tokens, n_acc, s.max_nodes, s.vocab, s.max_depth + 1, NsParams{});
+    return cudaGetLastError();
+}
+
+cudaError_t launch_verify_ns(const specinfer_shape_t &s, const WsLayout &w, const float *logits,
+                             const int32_t *tree_tokens, const int32_t *parent, const int32_t *n_nodes,
+                             float temperature, uint64_t seed, uint64_t offset, const int32_t *request_ids,
+                             int32_t *acc_nodes, int32_t *acc_tokens, int32_t *n_acc, char *ws, cudaStream_t stream) {
+    dim3 grid(s.max_nodes, s.batch);
+    const NsParams ns{1.4426950408889634f / temperature, (uint32_t)seed, (uint32_t)(seed >> 32), (uint32_t)offset,
+                      request_ids};
+    verify_greedy_kernel<true><<<grid, kGreedyThreads, 0, stream>>>(
+        logits, tree_tokens, parent, n_nodes, reinterpret_cast<const int32_t *>(ws + w.req_ok),
+        reinterpret_cast<int32_t *>(ws + w.argmax), reinterpret_cast<uint32_t *>(ws + w.verify_cnt), acc_nodes,
+        acc_tokens, n_acc, s.max_nodes, s.vocab, s.max_depth + 1, ns);
     return cudaGetLastError();
 }
 
