@@ -9,6 +9,8 @@
  *   specinfer_verify_greedy   Alg. 2 VerifyGreedy L395-401; §4.3
  *   specinfer_verify_mss      Alg. 2 VerifyStochastic L403-425; Fig. 5; Thm 4.2
  *   specinfer_kv_commit       depth-first KV-cache update L635-644; tree-topology KV layout L659-661
+ *   specinfer_expansion_topology, specinfer_expand_step, specinfer_tree_merge
+ *                             NEXT-2: token-tree construction (§3)
  *   specinfer_verify_ns       NEXT-3: naive sampling, the baseline of Theorem 4.3 (L747-765)
  *   specinfer_leaf_paths,     NEXT-1 baseline: sequence-based parallel decoding (§4.2,
  *   specinfer_sequence_pack   Fig. 4 left L682, §6.5)
@@ -147,6 +149,48 @@ specinfer_status_t specinfer_verify_ns(const specinfer_shape_t *shape, const flo
                                        int32_t *accepted_nodes, int32_t *accepted_tokens,
                                        int32_t *n_accepted, void *workspace,
                                        specinfer_stream_t stream);
+
+/* NEXT-2: token-tree construction on the GPU (§3; Fig. 2, Fig. 3).
+ *
+ * specinfer_expansion_topology: the static expansion <k_1..k_m> (L476-483; `expansion` is a
+ * HOST array of m ints, 1 <= k_i <= 8, m <= min(16, Dmax), 1 + sum_i prod_{j<=i} k_j <= Nmax):
+ * every request gets the same tree, node ids in DFS preorder (Fig. 2 "Linearization", L314),
+ * children of a node ordered by SSM rank (child j carries the node's (j+1)-th best token).
+ * Writes parent/depth int32 [B][Nmax] (padding: -1 / 0) and n_nodes int32 [B].
+ *
+ * specinfer_expand_step: expansion step `level` (0-based): the frontier = the nodes of depth
+ * `level` in DFS order, num_frontier of them; ssm_logits fp32 [B][num_frontier][V] holds the
+ * SSM's next-token logits for each frontier node (row f for the f-th frontier node).  Every
+ * frontier node's children (from parent[], in index order, at most 8) get its top tokens
+ * (descending logit, lowest token id on ties, R7) in tree_tokens [B][Nmax].  If draft_probs
+ * (fp32 [B][Nmax][V]) is not NULL, each child's row receives q = softmax(logits / temperature)
+ * of its parent (R12, the distribution the child was drawn from).  More than 8 children: the
+ * step writes nothing for that node and sets BAD_TREE in `workspace` (if not NULL).
+ *
+ * specinfer_tree_merge: token tree merge (Def. 3.2).  Inputs: num_inputs trees per
+ * request, in_parent / in_tokens int32 [B][num_inputs][input_nodes] (topological order, roots
+ * carrying the same token), in_n int32 [B][num_inputs] (0 = no tree).  Output: the tree whose
+ * sequences S_v are exactly the union of the inputs' S_u, node ids in DFS preorder with
+ * children in first-appearance order (inputs in order, nodes in index order): parent, depth,
+ * tree_tokens [B][Nmax], n_nodes [B]; node_map [B][num_inputs][input_nodes] = merged id of each
+ * input node (-1 beyond in_n).  Invalid input, differing roots, more than Nmax merged nodes or
+ * depth > Dmax: n_nodes[b] = 0, node_map -1, BAD_TREE set in `workspace` (if not NULL). */
+specinfer_status_t specinfer_expansion_topology(const specinfer_shape_t *shape,
+                                                const int32_t *expansion, int32_t m,
+                                                int32_t *parent, int32_t *depth, int32_t *n_nodes,
+                                                specinfer_stream_t stream);
+specinfer_status_t specinfer_expand_step(const specinfer_shape_t *shape, int32_t level,
+                                         int32_t num_frontier, const float *ssm_logits,
+                                         float temperature, const int32_t *parent,
+                                         const int32_t *depth, const int32_t *n_nodes,
+                                         int32_t *tree_tokens, float *draft_probs, void *workspace,
+                                         specinfer_stream_t stream);
+specinfer_status_t specinfer_tree_merge(const specinfer_shape_t *shape, int32_t num_inputs,
+                                        int32_t input_nodes, const int32_t *in_parent,
+                                        const int32_t *in_tokens, const int32_t *in_n,
+                                        int32_t *parent, int32_t *depth, int32_t *tree_tokens,
+                                        int32_t *n_nodes, int32_t *node_map, void *workspace,
+                                        specinfer_stream_t stream);
 
 /* NEXT-1: sequence-based parallel decoding, the baseline tree-based decoding replaces (§4.2
  * L622-632, Fig. 4 left L682, §6.5).  Not part of the hot path; used by the Fig. 11

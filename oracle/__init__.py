@@ -206,3 +206,82 @@ def leaf_paths(parent, n_nodes):
             paths.append(path[::-1])
         out.append(paths)
     return out
+
+
+# --------------------------------------------------------------------------------------------
+# NEXT-2: token-tree construction (§3), plain Python by definition
+# --------------------------------------------------------------------------------------------
+
+def expansion_tree_bfs(expansion):
+    """The static expansion <k1..km> (L476-483) built literally step by step: step i gives every
+    node of the current frontier k_i children.  Returns (parent, depth) in BFS (creation) order."""
+    parent, depth = [-1], [0]
+    frontier = [0]
+    for i, k in enumerate(expansion):
+        nxt = []
+        for u in frontier:
+            for _ in range(k):
+                parent.append(u)
+                depth.append(i + 1)
+                nxt.append(len(parent) - 1)
+        frontier = nxt
+    return parent, depth
+
+
+def dfs_linearize(parent, tokens=None):
+    """Depth-first linearisation (Fig. 2 "Linearization", L314): preorder, children in their order
+    of creation.  Returns (new_parent, new_tokens, order) with order[new_id] = old_id."""
+    n = len(parent)
+    kids = [[] for _ in range(n)]
+    for c in range(1, n):
+        kids[parent[c]].append(c)
+    order = []
+
+    def visit(u):
+        order.append(u)
+        for c in kids[u]:
+            visit(c)
+
+    visit(0)
+    new_id = {old: new for new, old in enumerate(order)}
+    new_parent = [-1 if parent[o] < 0 else new_id[parent[o]] for o in order]
+    new_tokens = None if tokens is None else [tokens[o] for o in order]
+    return new_parent, new_tokens, order
+
+
+def expand_topk(ssm_logits_row, k):
+    """The k tokens of an SSM distribution expanded at a node (L455-468: its top-k), by a full
+    sort: descending logit, lowest token id first among equals (reading R7)."""
+    row = np.asarray(ssm_logits_row, np.float64)
+    order = sorted(range(len(row)), key=lambda x: (-row[x], x))
+    return order[:k]
+
+
+def tree_merge(trees):
+    """Token tree merge (Def. 3.2) by its definition: the set of sequences S_u of every
+    input node (Def. 3.1: S_u = S_{p_u} + t_u) becomes one trie whose nodes are those sequences;
+    children ordered by first appearance (inputs in order, nodes in index order); DFS preorder.
+    `trees` = list of (parent, tokens).  Returns (parent, tokens, depth, node_maps) or None when
+    the roots differ (all input roots are the same last verified token, reading R6)."""
+    seqs = []          # distinct sequences in first-appearance order
+    index = {}
+    maps = []
+    for par, tok in trees:
+        S = []
+        m = []
+        for i in range(len(par)):
+            s = (tuple(S[par[i]]) if par[i] >= 0 else ()) + (int(tok[i]),)
+            S.append(list(s))
+            if s not in index:
+                index[s] = len(seqs)
+                seqs.append(s)
+            m.append(index[s])
+        maps.append(m)
+    if len({s[0] for s in seqs}) > 1:
+        return None
+    parent = [-1 if len(s) == 1 else index[s[:-1]] for s in seqs]
+    tokens = [s[-1] for s in seqs]
+    new_parent, new_tokens, order = dfs_linearize(parent, tokens)
+    new_id = {old: new for new, old in enumerate(order)}
+    depth = [len(seqs[o]) - 1 for o in order]
+    return new_parent, new_tokens, depth, [[new_id[x] for x in m] for m in maps]

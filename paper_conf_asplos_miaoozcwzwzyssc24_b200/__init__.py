@@ -31,7 +31,7 @@ EXPORTED_SYMBOLS = (
     "specinfer_read_device_status", "specinfer_philox_debug", "specinfer_debug_set_trace",
     "specinfer_launches_per_call",
     "specinfer_status_string", "specinfer_leaf_paths", "specinfer_sequence_pack",
-    "specinfer_verify_ns",
+    "specinfer_verify_ns", "specinfer_expansion_topology", "specinfer_expand_step", "specinfer_tree_merge",
 )
 
 
@@ -80,6 +80,9 @@ def load_library(path: str = LIB_PATH):
     lib.specinfer_kv_commit.argtypes = [sp, vp, vp, vp, vp, vp, vp]
     lib.specinfer_read_device_status.argtypes = [vp, vp, ctypes.POINTER(i32)]
     lib.specinfer_philox_debug.argtypes = [vp, vp, i32, vp]
+    lib.specinfer_expansion_topology.argtypes = [sp, vp, i32, vp, vp, vp, vp]
+    lib.specinfer_expand_step.argtypes = [sp, i32, i32, vp, f32, vp, vp, vp, vp, vp, vp, vp]
+    lib.specinfer_tree_merge.argtypes = [sp, i32, i32, vp, vp, vp, vp, vp, vp, vp, vp, vp, vp]
     lib.specinfer_verify_ns.argtypes = [sp, vp, vp, vp, vp, f32, u64, u64, vp, vp, vp, vp, vp, vp]
     lib.specinfer_leaf_paths.argtypes = [sp, vp, vp, vp, vp, vp, vp, vp]
     lib.specinfer_sequence_pack.argtypes = [sp, i32, i32] + [vp] * 14 + [vp]
@@ -91,7 +94,8 @@ def load_library(path: str = LIB_PATH):
     lib.specinfer_status_string.restype = ctypes.c_char_p
     for name in ("specinfer_tree_prepare", "specinfer_tree_attention", "specinfer_verify_greedy",
                  "specinfer_verify_mss", "specinfer_kv_commit", "specinfer_read_device_status",
-                 "specinfer_philox_debug", "specinfer_leaf_paths", "specinfer_sequence_pack", "specinfer_verify_ns"):
+                 "specinfer_philox_debug", "specinfer_leaf_paths", "specinfer_sequence_pack", "specinfer_verify_ns",
+                 "specinfer_expansion_topology", "specinfer_expand_step", "specinfer_tree_merge"):
         getattr(lib, name).restype = i32
     _lib = lib
     return lib
@@ -259,6 +263,49 @@ def specinfer_philox_debug(ctr_key: torch.Tensor) -> torch.Tensor:
     _check("specinfer_philox_debug", load_library().specinfer_philox_debug(
         ctypes.c_void_p(ck.data_ptr()), ctypes.c_void_p(out.data_ptr()), ck.shape[0], _stream(ck)))
     return out.to(torch.int64).bitwise_and(0xFFFFFFFF)
+
+
+def specinfer_expansion_topology(shape: Shape, expansion, parent, depth, n_nodes):
+    """NEXT-2: the static expansion tree <k1..km> for every request (DFS preorder)."""
+    dev = parent.device
+    B, N = shape.batch, shape.max_nodes
+    ks = (ctypes.c_int32 * len(expansion))(*[int(k) for k in expansion])
+    _check("specinfer_expansion_topology", load_library().specinfer_expansion_topology(
+        ctypes.byref(shape), ks, len(expansion), _req("parent", parent, torch.int32, (B, N), dev),
+        _req("depth", depth, torch.int32, (B, N), dev), _req("n_nodes", n_nodes, torch.int32, (B,), dev),
+        _stream(parent)))
+
+
+def specinfer_expand_step(shape: Shape, level: int, ssm_logits, temperature, parent, depth, n_nodes, tree_tokens,
+                          draft_probs=None, workspace=None):
+    """NEXT-2: one expansion step (top-k of each frontier node's SSM logits -> its children)."""
+    dev = ssm_logits.device
+    B, N, V = shape.batch, shape.max_nodes, shape.vocab
+    F = int(ssm_logits.shape[1])
+    if not (temperature > 0):
+        raise ValueError("temperature must be > 0")
+    args = (_req("ssm_logits", ssm_logits, torch.float32, (B, F, V), dev),)
+    _check("specinfer_expand_step", load_library().specinfer_expand_step(
+        ctypes.byref(shape), int(level), F, *args, ctypes.c_float(temperature),
+        _req("parent", parent, torch.int32, (B, N), dev), _req("depth", depth, torch.int32, (B, N), dev),
+        _req("n_nodes", n_nodes, torch.int32, (B,), dev), _req("tree_tokens", tree_tokens, torch.int32, (B, N), dev),
+        _opt("draft_probs", draft_probs, torch.float32, (B, N, V), dev),
+        _opt("workspace", workspace, torch.uint8, None, dev), _stream(ssm_logits)))
+
+
+def specinfer_tree_merge(shape: Shape, in_parent, in_tokens, in_n, parent, depth, tree_tokens, n_nodes, node_map,
+                         workspace=None):
+    """NEXT-2: token tree merge (Def. 3.2) of [B][T][Nin] input trees into [B][Nmax] DFS trees."""
+    dev = in_parent.device
+    B, N = shape.batch, shape.max_nodes
+    T, Nin = int(in_parent.shape[1]), int(in_parent.shape[2])
+    _check("specinfer_tree_merge", load_library().specinfer_tree_merge(
+        ctypes.byref(shape), T, Nin, _req("in_parent", in_parent, torch.int32, (B, T, Nin), dev),
+        _req("in_tokens", in_tokens, torch.int32, (B, T, Nin), dev), _req("in_n", in_n, torch.int32, (B, T), dev),
+        _req("parent", parent, torch.int32, (B, N), dev), _req("depth", depth, torch.int32, (B, N), dev),
+        _req("tree_tokens", tree_tokens, torch.int32, (B, N), dev), _req("n_nodes", n_nodes, torch.int32, (B,), dev),
+        _req("node_map", node_map, torch.int32, (B, T, Nin), dev),
+        _opt("workspace", workspace, torch.uint8, None, dev), _stream(in_parent)))
 
 
 def specinfer_leaf_paths(shape: Shape, parent, n_nodes, paths, path_len, n_leaves, workspace=None):

@@ -40,6 +40,15 @@ cudaError_t launch_sequence_pack(const specinfer_shape_t &s, int num_seqs, int s
                                  const void *q, const void *k, const void *v, void *q_seq, void *k_seq, void *v_seq,
                                  int32_t *seq_parent, int32_t *seq_depth, int32_t *seq_prefix, int32_t *seq_n,
                                  cudaStream_t stream);
+cudaError_t launch_expansion_topology(const specinfer_shape_t &s, const int32_t *ks, int m, int32_t *parent,
+                                      int32_t *depth, int32_t *n_nodes, cudaStream_t stream);
+cudaError_t launch_expand_step(const specinfer_shape_t &s, int level, const float *ssm_logits, int F, float temperature,
+                               const int32_t *parent, const int32_t *depth, const int32_t *n_nodes, int32_t *tokens,
+                               float *draft_probs, int32_t *status, cudaStream_t stream);
+cudaError_t launch_tree_merge(const specinfer_shape_t &s, int T, int Nin, const int32_t *in_parent,
+                              const int32_t *in_tokens, const int32_t *in_n, int32_t *parent, int32_t *depth,
+                              int32_t *tokens, int32_t *n_nodes, int32_t *node_map, int32_t *status,
+                              cudaStream_t stream);
 cudaError_t launch_philox_debug(const uint32_t *ck, uint32_t *out, int n, cudaStream_t stream);
 extern unsigned long long *g_attn_trace;
 extern int g_attn_debug_flags;
@@ -261,6 +270,57 @@ specinfer_status_t specinfer_sequence_pack(const specinfer_shape_t *shape, int32
                                           seq_prefix_len, seq_n_nodes, (cudaStream_t)stream));
 }
 
+specinfer_status_t specinfer_expansion_topology(const specinfer_shape_t *shape, const int32_t *expansion,
+                                                int32_t m, int32_t *parent, int32_t *depth, int32_t *n_nodes,
+                                                specinfer_stream_t stream) {
+    SPI_TRY(check_shape(shape));
+    if (!expansion || m < 0 || m > 16 || m > shape->max_depth || !parent || !depth || !n_nodes)
+        return SPECINFER_ERR_INVALID_ARG;
+    long long n = 1, level = 1;
+    for (int i = 0; i < m; ++i) {
+        if (expansion[i] < 1 || expansion[i] > 8) return SPECINFER_ERR_INVALID_ARG;
+        level *= expansion[i];
+        n += level;
+        if (n > shape->max_nodes) return SPECINFER_ERR_INVALID_ARG;
+    }
+    DeviceInfo d;
+    SPI_TRY(check_device(&d));
+    return from_cuda(launch_expansion_topology(*shape, expansion, m, parent, depth, n_nodes, (cudaStream_t)stream));
+}
+
+specinfer_status_t specinfer_expand_step(const specinfer_shape_t *shape, int32_t level, int32_t num_frontier,
+                                         const float *ssm_logits, float temperature, const int32_t *parent,
+                                         const int32_t *depth, const int32_t *n_nodes, int32_t *tree_tokens,
+                                         float *draft_probs, void *workspace, specinfer_stream_t stream) {
+    SPI_TRY(check_shape(shape));
+    if (shape->vocab < 1 || level < 0 || num_frontier < 0 || !(temperature > 0.f) || !isfinite(temperature))
+        return SPECINFER_ERR_INVALID_ARG;
+    if (!ssm_logits || !parent || !depth || !n_nodes || !tree_tokens) return SPECINFER_ERR_INVALID_ARG;
+    if (workspace) SPI_TRY(check_ws(workspace));
+    DeviceInfo d;
+    SPI_TRY(check_device(&d));
+    if (num_frontier == 0) return SPECINFER_OK;
+    return from_cuda(launch_expand_step(*shape, level, ssm_logits, num_frontier, temperature, parent, depth, n_nodes,
+                                        tree_tokens, draft_probs, reinterpret_cast<int32_t *>(workspace),
+                                        (cudaStream_t)stream));
+}
+
+specinfer_status_t specinfer_tree_merge(const specinfer_shape_t *shape, int32_t num_inputs, int32_t input_nodes,
+                                        const int32_t *in_parent, const int32_t *in_tokens, const int32_t *in_n,
+                                        int32_t *parent, int32_t *depth, int32_t *tree_tokens, int32_t *n_nodes,
+                                        int32_t *node_map, void *workspace, specinfer_stream_t stream) {
+    SPI_TRY(check_shape(shape));
+    if (num_inputs < 1 || input_nodes < 1 || input_nodes > kMaxNodes) return SPECINFER_ERR_INVALID_ARG;
+    if (!in_parent || !in_tokens || !in_n || !parent || !depth || !tree_tokens || !n_nodes || !node_map)
+        return SPECINFER_ERR_INVALID_ARG;
+    if (workspace) SPI_TRY(check_ws(workspace));
+    DeviceInfo d;
+    SPI_TRY(check_device(&d));
+    return from_cuda(launch_tree_merge(*shape, num_inputs, input_nodes, in_parent, in_tokens, in_n, parent, depth,
+                                       tree_tokens, n_nodes, node_map, reinterpret_cast<int32_t *>(workspace),
+                                       (cudaStream_t)stream));
+}
+
 specinfer_status_t specinfer_read_device_status(const void *workspace, specinfer_stream_t stream,
                                                 int32_t *status_bits_out) {
     SPI_TRY(check_ws(workspace));
@@ -298,7 +358,10 @@ int32_t specinfer_launches_per_call(const char *name) {
     if (!strcmp(name, "verify_mss")) return 1;
     if (!strcmp(name, "kv_commit")) return 2;        // copy, prefix update
     if (!strcmp(name, "leaf_paths")) return 1;
-    if (!strcmp(name, "verify_ns")) return 1;         // race-argmax + walk fused (last CTA walks)
+    if (!strcmp(name, "verify_ns")) return 1;
+    if (!strcmp(name, "expansion_topology")) return 1;
+    if (!strcmp(name, "expand_step")) return 1;
+    if (!strcmp(name, "tree_merge")) return 1;         // race-argmax + walk fused (last CTA walks)
     if (!strcmp(name, "sequence_pack")) return 1;
     return -1;
 }
