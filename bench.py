@@ -50,6 +50,8 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--verify", default=None, help="comma list overriding the config's verify modes")
+    ap.add_argument("--shard", default="auto", choices=["auto", "request", "kv"],
+                    help="N > 1 layout: request sharding, or kv-head sharding (GQA; auto for G > 1)")
     return ap.parse_args()
 
 
@@ -128,30 +130,44 @@ class ClockSampler:
 # workload
 # ------------------------------------------------------------------------------------------
 class Workload:
-    def __init__(self, cfg: W.Config, args, rank: int, device):
+    """One GPU's share of the step.  Request sharding: this rank's B requests end to end.  kv-head
+    sharding (GQA, N > 1): attention and KV commit over ALL B*N requests for this rank's Hkv/N
+    kv-heads (and their q-heads), verification over this rank's B requests (dist.py)."""
+
+    def __init__(self, cfg: W.Config, args, rank: int, device, ws: int = 1, kv_shard: bool = False):
         self.cfg = cfg
         self.L = args.layers or cfg.layers
         self.B = args.batch or cfg.batch
         self.P = args.prefix or cfg.prefix
+        self.kv_shard = kv_shard
+        self.Batt = self.B * ws if kv_shard else self.B
         self.Hq, self.Hkv, self.V = cfg.num_q_heads, cfg.num_kv_heads, cfg.vocab
+        self.req_lo = rank * self.B if kv_shard else 0
+        if kv_shard:
+            from paper_conf_asplos_miaoozcwzwzyssc24_b200 import dist as D
+            _, self.Hkv, _, self.Hq = D.shard_kv_heads(cfg.num_q_heads, cfg.num_kv_heads, ws, rank)
         self.verify = tuple(args.verify.split(",")) if args.verify else cfg.verify
         parent, depth = cfg.tree
         self.N = int(parent.shape[0])
         self.Dmax = cfg.max_depth
         self.smax = self.P + self.N
         self.device = device
-        self.tb = W.make_tree_batch([(parent, depth)] * self.B, [self.P] * self.B, device=device,
+        self.tb = W.make_tree_batch([(parent, depth)] * self.Batt, [self.P] * self.Batt, device=device,
                                     max_depth=self.Dmax)
         seed = cfg.seed + 1000 * rank
         self.ai = W.make_attention_inputs(self.tb, self.L, self.Hq, self.Hkv, self.smax, seed=seed, device=device)
         mode = "mss" if self.verify == ("mss",) else "greedy"
-        self.vi = W.make_verify_inputs(self.tb, self.V, seed=seed, mode=mode, device=device)
+        lo, hi = self.req_lo, self.req_lo + self.B
+        self.tbv = W.TreeBatch(self.tb.parent[lo:hi], self.tb.depth[lo:hi], self.tb.prefix_len[lo:hi],
+                               self.tb.n_nodes[lo:hi], self.tb.max_nodes, self.tb.max_depth)
+        self.vi = W.make_verify_inputs(self.tbv, self.V, seed=seed, mode=mode, device=device)
         self.rids = torch.arange(rank * self.B, (rank + 1) * self.B, dtype=torch.int32, device=device)
         self.bytes_launch = self.attn_bytes_per_launch()   # before any commit moves prefix_len
         self.flops_launch = self.attn_flops_per_launch()
 
     def tree_tokens_per_step(self) -> int:
-        return int(self.tb.n_nodes.sum().item())
+        """Tree tokens this rank verifies per step (its B requests)."""
+        return int(self.tbv.n_nodes.sum().item())
 
     def attn_bytes_per_launch(self) -> int:
         """Algorithmic bytes of one tree_attention launch: K and V of every
@@ -166,7 +182,7 @@ class Workload:
         pl = self.tb.prefix_len.cpu().numpy().astype(np.int64)
         n = self.tb.n_nodes.cpu().numpy().astype(np.int64)
         dep = self.tb.depth.cpu().numpy()
-        tree_pairs = np.array([int((dep[b, :n[b]] + 1).sum()) for b in range(self.B)])
+        tree_pairs = np.array([int((dep[b, :n[b]] + 1).sum()) for b in range(self.Batt)])
         return int((4 * 128 * (n * pl + tree_pairs) * self.Hq).sum())
 
 
@@ -176,11 +192,21 @@ def run_ours(args, ws, rank, local):
     device = torch.device("cuda", local)
     torch.cuda.set_device(device)
     cfg = W.CONFIGS[args.config]
-    wl = Workload(cfg, args, rank, device)
+    G = cfg.num_q_heads // cfg.num_kv_heads
+    # (--shard kv also runs at N = 1, where the gather degenerates to a copy: exercises the layout)
+    kv_shard = args.shard == "kv" or (ws > 1 and args.shard == "auto" and G > 1 and cfg.num_kv_heads % ws == 0)
+    wl = Workload(cfg, args, rank, device, ws=ws, kv_shard=kv_shard)
     L, B, N, Dmax = wl.L, wl.B, wl.N, wl.Dmax
+    Ba = wl.Batt
     Lp = Dmax + 1
-    shape = spi.make_shape(B, N, wl.Hq, wl.Hkv, wl.smax, num_layers=L, vocab=wl.V, max_depth=Dmax)
+    # attention / commit shape (all B*N requests x local heads when kv-sharded) and verify shape
+    shape = spi.make_shape(Ba, N, wl.Hq, wl.Hkv, wl.smax, num_layers=L, vocab=wl.V, max_depth=Dmax)
     st = spi.TreeState.create(shape, wl.tb.parent, wl.tb.depth, wl.tb.prefix_len, wl.tb.n_nodes)
+    if kv_shard:
+        shape_v = spi.make_shape(B, N, 1, 1, wl.smax, num_layers=L, vocab=wl.V, max_depth=Dmax)
+        st_v = spi.TreeState.create(shape_v, wl.tbv.parent, wl.tbv.depth, wl.tbv.prefix_len, wl.tbv.n_nodes)
+    else:
+        shape_v, st_v = shape, st
     out = torch.empty_like(wl.ai.q)
     prefix0 = wl.tb.prefix_len.clone()
     an = torch.empty((B, Lp), dtype=torch.int32, device=device)
@@ -188,44 +214,63 @@ def run_ours(args, ws, rank, local):
     an2, at2, na2 = torch.empty_like(an), torch.empty_like(an), torch.empty_like(na)
     gather_in = torch.empty((B, 2 * Lp + 1), dtype=torch.int32, device=device)
     gather_out = torch.empty((ws * B, 2 * Lp + 1), dtype=torch.int32, device=device)
+    an_all = torch.empty((Ba, Lp), dtype=torch.int32, device=device)   # kv-sharded commit input
+    na_all = torch.empty((Ba,), dtype=torch.int32, device=device)
     iteration = [0]
 
     def seg_prepare():
         wl.tb.prefix_len.copy_(prefix0)
         st.prepare()
+        if kv_shard:
+            st_v.prepare()
 
     def seg_attention():
         for l in range(L):
             st.attention(wl.ai.q[l], wl.ai.k_cache[l], wl.ai.v_cache[l], out[l])
 
-    def seg_verify_commit():
-        commit_src = None
+    def seg_verify():
         if "greedy" in wl.verify:
-            spi.specinfer_verify_greedy(shape, wl.vi.logits, wl.vi.tree_tokens, wl.tb.parent, wl.tb.n_nodes,
-                                        an, at, na, st.workspace)
-            commit_src = (an, na)
+            spi.specinfer_verify_greedy(shape_v, wl.vi.logits, wl.vi.tree_tokens, wl.tbv.parent, wl.tbv.n_nodes,
+                                        an, at, na, st_v.workspace)
         if "mss" in wl.verify:
-            spi.specinfer_verify_mss(shape, wl.vi.logits, wl.vi.tree_tokens, wl.tb.parent, wl.tb.n_nodes,
-                                     wl.vi.draft_probs, 1.0, cfg.seed, 0, wl.rids, an2, at2, na2, st.workspace)
-            if commit_src is None:
-                commit_src = (an2, na2)
-        spi.specinfer_kv_commit(shape, wl.ai.k_cache, wl.ai.v_cache, wl.tb.prefix_len, commit_src[0], commit_src[1])
+            spi.specinfer_verify_mss(shape_v, wl.vi.logits, wl.vi.tree_tokens, wl.tbv.parent, wl.tbv.n_nodes,
+                                     wl.vi.draft_probs, 1.0, cfg.seed, 0, wl.rids, an2, at2, na2, st_v.workspace)
 
-    launches_per_step = (spi.specinfer_launches_per_call("tree_prepare") + L * spi.specinfer_launches_per_call(
-        "tree_attention") + ("greedy" in wl.verify) * spi.specinfer_launches_per_call("verify_greedy") +
-        ("mss" in wl.verify) * spi.specinfer_launches_per_call("verify_mss") +
-        spi.specinfer_launches_per_call("kv_commit"))
+    def seg_commit():
+        if kv_shard:
+            # every request's accepted path (gathered) -> this rank's kv-head shard of its cache
+            n_all, _, nodes_all = D.unpack_accepted(gather_out)
+            na_all.copy_(n_all)
+            an_all.copy_(nodes_all)
+            src = (an_all, na_all)
+        else:
+            src = (an, na) if "greedy" in wl.verify else (an2, na2)
+        spi.specinfer_kv_commit(shape, wl.ai.k_cache, wl.ai.v_cache, wl.tb.prefix_len, src[0], src[1])
+
+    launches_per_step = (spi.specinfer_launches_per_call("tree_prepare") * (2 if kv_shard else 1) +
+                         L * spi.specinfer_launches_per_call("tree_attention") +
+                         ("greedy" in wl.verify) * spi.specinfer_launches_per_call("verify_greedy") +
+                         ("mss" in wl.verify) * spi.specinfer_launches_per_call("verify_mss") +
+                         spi.specinfer_launches_per_call("kv_commit"))
 
     from paper_conf_asplos_miaoozcwzwzyssc24_b200 import dist as D
 
     def gather():
         # a7: the tokens-only exchange after verification, NCCL over NVLink
-        if ws > 1:
+        if ws > 1 or kv_shard:
             src = (na, at, an) if "greedy" in wl.verify else (na2, at2, an2)
             gather_in.copy_(D.pack_accepted(*src))
-            D.gather_accepted(gather_in, gather_out)
+            if ws > 1:
+                D.gather_accepted(gather_in, gather_out)
+            else:
+                gather_out.copy_(gather_in)
 
-    # ---- capture the three segments as CUDA graphs (one launch each per step) ----
+    def seg_verify_commit():
+        seg_verify()
+        gather()
+        seg_commit()
+
+    # ---- capture the segments as CUDA graphs (one launch each per step; the gather stays eager) ----
     s = torch.cuda.Stream(device)
     s.wait_stream(torch.cuda.current_stream(device))
     with torch.cuda.stream(s):
@@ -233,7 +278,7 @@ def run_ours(args, ws, rank, local):
             seg_prepare(); seg_attention(); seg_verify_commit()
     torch.cuda.synchronize(device)
     graphs = []
-    for fn in (seg_prepare, seg_attention, seg_verify_commit):
+    for fn in (seg_prepare, seg_attention, seg_verify, seg_commit):
         g = torch.cuda.CUDAGraph()
         with torch.cuda.graph(g, stream=s):
             fn()
@@ -245,6 +290,7 @@ def run_ours(args, ws, rank, local):
         graphs[1].replay()
         graphs[2].replay()
         gather()
+        graphs[3].replay()
 
     with torch.cuda.stream(s):
         for _ in range(args.warmup):
@@ -267,6 +313,7 @@ def run_ours(args, ws, rank, local):
             ev[3 + 2 * k].record(s)
             graphs[2].replay()
             gather()
+            graphs[3].replay()
         ev[1].record(s)
     torch.cuda.synchronize(device)
     barrier(ws)
@@ -355,7 +402,6 @@ def run_ours(args, ws, rank, local):
                 st.attention(wl.ai.q[l], wl.ai.k_cache[l], wl.ai.v_cache[l], out[l])
             s.wait_event(ev_lg)
             seg_verify_commit()
-            gather()
             h_res_a.copy_(res_a, non_blocking=True)
             h_res_n.copy_(res_n, non_blocking=True)
 
@@ -410,10 +456,11 @@ def run_ours(args, ws, rank, local):
         "config": {"workload": f"{cfg.name}: {cfg.description}", "layers": L, "batch_per_gpu": B,
                    "global_batch": B * ws, "prefix": wl.P, "tree_nodes": N, "max_depth": Dmax,
                    "num_q_heads": wl.Hq, "num_kv_heads": wl.Hkv, "vocab": wl.V, "verify": list(wl.verify),
-                   "parallelism": f"request-sharded x{ws}" if ws > 1 else "single GPU",
+                   "parallelism": (f"kv-head-sharded attention/commit x{ws}, request-sharded verification" if kv_shard
+                                   else f"request-sharded x{ws}") if ws > 1 else "single GPU",
                    "l2": "no flush: every step streams the full KV cache "
                          f"({2 * L * B * wl.Hkv * wl.smax * 256 / 1e9:.1f} GB/GPU) >> 126 MB L2",
-                   "graph": "3 CUDA graphs per step (prepare | L x attention | verify + commit)"},
+                   "graph": "4 CUDA graphs per step (prepare | L x attention | verify | commit), NCCL gather between"},
         "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
         "gpu_launches": launches_per_step * K, "clocks": clocks,
         "extra": {"tree_tokens_per_step": tokens_step * ws, "mean_n_accepted_greedy": acc_mean if "greedy" in wl.verify else None,

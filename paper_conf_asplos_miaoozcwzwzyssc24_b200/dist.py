@@ -1,10 +1,14 @@
 """Multi-GPU plumbing of the verification step.
 
 The hot path partitions by request: every (request, kv-head) is independent for tree attention and
-KV commit, every request for verification.  Ranks own disjoint request ranges; the only exchange is
-the tokens-only gather after verification (the request manager and GPU workers
-"only communicate tokens").  MSS counters use global request ids, so results are identical at any
-world size.  NCCL (over NVLink/NVSwitch) on GPUs; gloo is accepted for the CPU tests.
+KV commit, every request for verification.  Two layouts:
+  * request sharding (C2, C4, C5): ranks own disjoint request ranges end to end;
+  * kv-head sharding (GQA, C3): ranks own disjoint kv-head ranges (and their q-head groups) of every
+    request for attention and KV commit, while verification stays request-sharded (the logits are
+    per request); the gathered accepted paths let every rank commit its head shard of all requests.
+Either way the only exchange is the tokens-only gather after verification (the
+request manager and GPU workers "only communicate tokens").  MSS counters use global request ids, so
+results are identical at any world size.  NCCL (over NVLink/NVSwitch) on GPUs; gloo for the CPU tests.
 """
 from __future__ import annotations
 
@@ -18,6 +22,17 @@ def shard_requests(batch_global: int, world: int, rank: int) -> Tuple[int, int]:
     base, rem = divmod(batch_global, world)
     start = rank * base + min(rank, rem)
     return start, base + (1 if rank < rem else 0)
+
+
+def shard_kv_heads(num_q_heads: int, num_kv_heads: int, world: int, rank: int) -> Tuple[int, int, int, int]:
+    """kv-head sharding: rank's kv-heads [kv0, kv0 + nkv) and their q-heads [q0, q0 + nq) (each
+    kv-head keeps its whole GQA group, so attention needs no exchange).  Requires Hkv % world == 0."""
+    if num_kv_heads % world != 0 or num_q_heads % num_kv_heads != 0:
+        raise ValueError(f"cannot shard {num_kv_heads} kv-heads over {world} ranks")
+    G = num_q_heads // num_kv_heads
+    nkv = num_kv_heads // world
+    kv0 = rank * nkv
+    return kv0, nkv, kv0 * G, nkv * G
 
 
 def global_request_ids(start: int, count: int, device) -> torch.Tensor:

@@ -79,3 +79,76 @@ def test_two_rank_gather_equals_single_process():
     na, at, an = _verify(tb, vi, 0, tb.parent.shape[0])
     ref = D.pack_accepted(na, at, an).numpy()
     assert np.array_equal(gathered, ref)
+
+
+# ---------------------------------------------------------------------------------------------
+# kv-head sharding (GQA, C3): attention + commit on head shards of every request, verification
+# request-sharded, one gather; the result must equal a single-process run
+# ---------------------------------------------------------------------------------------------
+
+def _kv_inputs():
+    rng = np.random.default_rng(5)
+    B, N, V, Hq, Hkv, P = 4, 12, 30, 8, 4, 9
+    trees = [W.random_tree(int(rng.integers(2, N + 1)), 6, 3, rng) for _ in range(B)]
+    tb = W.make_tree_batch(trees, [P] * B, max_nodes=N, max_depth=6)
+    ai = W.make_attention_inputs(tb, 1, Hq, Hkv, P + N, seed=4)
+    vi = W.make_verify_inputs(tb, V, seed=6, mode="greedy")
+    return tb, ai, vi, Hq, Hkv
+
+
+def _kv_worker(rank, world, port, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    torch.distributed.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        tb, ai, vi, Hq, Hkv = _kv_inputs()
+        B = tb.parent.shape[0]
+        kv0, nkv, q0, nq = D.shard_kv_heads(Hq, Hkv, world, rank)
+        # attention on this rank's head shard of every request
+        out = oracle.tree_attention(ai.q[0][:, :, q0:q0 + nq], ai.k_cache[0][:, kv0:kv0 + nkv],
+                                    ai.v_cache[0][:, kv0:kv0 + nkv], tb.parent, tb.depth, tb.prefix_len, tb.n_nodes)
+        # verification on this rank's requests
+        lo, cnt = D.shard_requests(B, world, rank)
+        sl = slice(lo, lo + cnt)
+        an, at, na = oracle.verify_greedy(vi.logits[sl].numpy(), vi.tree_tokens[sl].numpy(),
+                                          tb.parent[sl].numpy(), tb.n_nodes[sl].numpy(), path_len=7)
+        g = D.gather_accepted(D.pack_accepted(torch.from_numpy(na), torch.from_numpy(at), torch.from_numpy(an)))
+        na_all, _, an_all = D.unpack_accepted(g)
+        # commit this rank's head shard of every request
+        k = ai.k_cache[:, :, kv0:kv0 + nkv].contiguous().view(torch.int16).numpy().astype(np.uint16)
+        v = ai.v_cache[:, :, kv0:kv0 + nkv].contiguous().view(torch.int16).numpy().astype(np.uint16)
+        pl = tb.prefix_len.numpy().copy()
+        oracle.kv_commit(k, v, pl, an_all.contiguous().numpy(), na_all.contiguous().numpy())
+        q.put((rank, out, k, pl))
+    finally:
+        torch.distributed.destroy_process_group()
+
+
+def test_two_rank_kv_head_sharding_equals_single_process():
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_kv_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = dict((r, (o, k, pl)) for r, o, k, pl in [q.get(timeout=120) for _ in range(world)])
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    tb, ai, vi, Hq, Hkv = _kv_inputs()
+    out = oracle.tree_attention(ai.q[0], ai.k_cache[0], ai.v_cache[0], tb.parent, tb.depth, tb.prefix_len,
+                                tb.n_nodes)
+    an, at, na = oracle.verify_greedy(vi.logits.numpy(), vi.tree_tokens.numpy(), tb.parent.numpy(),
+                                      tb.n_nodes.numpy(), path_len=7)
+    k = ai.k_cache.contiguous().view(torch.int16).numpy().astype(np.uint16)
+    v = ai.v_cache.contiguous().view(torch.int16).numpy().astype(np.uint16)
+    pl = tb.prefix_len.numpy().copy()
+    oracle.kv_commit(k, v, pl, an, na)
+    n = tb.n_nodes.numpy()
+    for r in range(world):
+        kv0, nkv, q0, nq = D.shard_kv_heads(Hq, Hkv, world, r)
+        o, kr, plr = res[r]
+        for b in range(len(n)):
+            np.testing.assert_array_equal(o[b, :n[b]], out[b, :n[b], q0:q0 + nq])
+            assert np.array_equal(kr[:, b, :, :plr[b]], k[:, b, kv0:kv0 + nkv, :pl[b]])
+        assert np.array_equal(plr, pl)
