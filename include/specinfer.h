@@ -11,6 +11,8 @@
  *   specinfer_kv_commit       depth-first KV-cache update L635-644; tree-topology KV layout L659-661
  *   specinfer_expansion_topology, specinfer_expand_step, specinfer_tree_merge
  *                             NEXT-2: token-tree construction (§3)
+ *   specinfer_tree_attention_paged, specinfer_kv_commit_paged
+ *                             NEXT-4: paged KV cache (tree layout L659-661 over 128-slot pages)
  *   specinfer_verify_ns       NEXT-3: naive sampling, the baseline of Theorem 4.3 (L747-765)
  *   specinfer_leaf_paths,     NEXT-1 baseline: sequence-based parallel decoding (§4.2,
  *   specinfer_sequence_pack   Fig. 4 left L682, §6.5)
@@ -136,6 +138,26 @@ specinfer_status_t specinfer_verify_mss(const specinfer_shape_t *shape, const fl
                                         const int32_t *request_ids, int32_t *accepted_nodes,
                                         int32_t *accepted_tokens, int32_t *n_accepted,
                                         void *workspace, specinfer_stream_t stream);
+
+/* NEXT-4: paged KV cache (for serving; same computation as tree_attention / kv_commit).
+ * Keys of request b live in pages of 128 slots: slot s is row s % 128 of page
+ * page_table[b][s / 128] (int32 [B][ceil(Smax / 128)], entries in [0, num_pages); pages covering
+ * [0, P_b + n_b) must be valid and the pages of different requests distinct).  A page holds every
+ * kv-head: k_pages / v_pages bf16 [num_pages][Hkv][128][128] for one layer (attention) or
+ * [L][...] `layer_stride` apart (0 => num_pages*Hkv*128*128) for the commit.  Tree node i is at
+ * slot P_b + i as in the contiguous layout.  Results are bit-identical to the contiguous calls on
+ * the same data (same tiles, same schedule). */
+specinfer_status_t specinfer_tree_attention_paged(const specinfer_shape_t *shape, const void *q,
+                                                  const void *k_pages, const void *v_pages,
+                                                  int32_t num_pages, const int32_t *page_table,
+                                                  const int32_t *parent, const int32_t *depth,
+                                                  const int32_t *prefix_len, const int32_t *n_nodes,
+                                                  void *out, void *workspace, specinfer_stream_t stream);
+specinfer_status_t specinfer_kv_commit_paged(const specinfer_shape_t *shape, void *k_pages_all,
+                                             void *v_pages_all, int32_t num_pages,
+                                             const int32_t *page_table, int32_t *prefix_len,
+                                             const int32_t *accepted_nodes, const int32_t *n_accepted,
+                                             specinfer_stream_t stream);
 
 /* NEXT-3: naive sampling (NS), the verifier Theorem 4.3 compares MSS with (L747-765): at each
  * node u on the walk draw x ~ softmax(logits[u]/temperature) by the exponential race of

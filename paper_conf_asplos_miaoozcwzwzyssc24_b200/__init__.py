@@ -32,6 +32,7 @@ EXPORTED_SYMBOLS = (
     "specinfer_launches_per_call",
     "specinfer_status_string", "specinfer_leaf_paths", "specinfer_sequence_pack",
     "specinfer_verify_ns", "specinfer_expansion_topology", "specinfer_expand_step", "specinfer_tree_merge",
+    "specinfer_tree_attention_paged", "specinfer_kv_commit_paged",
 )
 
 
@@ -80,6 +81,8 @@ def load_library(path: str = LIB_PATH):
     lib.specinfer_kv_commit.argtypes = [sp, vp, vp, vp, vp, vp, vp]
     lib.specinfer_read_device_status.argtypes = [vp, vp, ctypes.POINTER(i32)]
     lib.specinfer_philox_debug.argtypes = [vp, vp, i32, vp]
+    lib.specinfer_tree_attention_paged.argtypes = [sp, vp, vp, vp, i32, vp, vp, vp, vp, vp, vp, vp, vp]
+    lib.specinfer_kv_commit_paged.argtypes = [sp, vp, vp, i32, vp, vp, vp, vp, vp]
     lib.specinfer_expansion_topology.argtypes = [sp, vp, i32, vp, vp, vp, vp]
     lib.specinfer_expand_step.argtypes = [sp, i32, i32, vp, f32, vp, vp, vp, vp, vp, vp, vp]
     lib.specinfer_tree_merge.argtypes = [sp, i32, i32, vp, vp, vp, vp, vp, vp, vp, vp, vp, vp]
@@ -95,7 +98,8 @@ def load_library(path: str = LIB_PATH):
     for name in ("specinfer_tree_prepare", "specinfer_tree_attention", "specinfer_verify_greedy",
                  "specinfer_verify_mss", "specinfer_kv_commit", "specinfer_read_device_status",
                  "specinfer_philox_debug", "specinfer_leaf_paths", "specinfer_sequence_pack", "specinfer_verify_ns",
-                 "specinfer_expansion_topology", "specinfer_expand_step", "specinfer_tree_merge"):
+                 "specinfer_expansion_topology", "specinfer_expand_step", "specinfer_tree_merge",
+                 "specinfer_tree_attention_paged", "specinfer_kv_commit_paged"):
         getattr(lib, name).restype = i32
     _lib = lib
     return lib
@@ -170,6 +174,44 @@ def specinfer_tree_attention(shape: Shape, q, k_cache, v_cache, parent, depth, p
     ws = _req("workspace", workspace, torch.uint8, None, dev)
     _check("specinfer_tree_attention",
            load_library().specinfer_tree_attention(ctypes.byref(shape), qp, kp, vp, *args, op, ws, _stream(q)))
+
+
+def specinfer_tree_attention_paged(shape: Shape, q, k_pages, v_pages, page_table, parent, depth, prefix_len, n_nodes,
+                                   out, workspace):
+    """NEXT-4: tree attention over a paged KV cache ([num_pages][Hkv][128][128] pages)."""
+    dev = q.device
+    B, N, Hq, Hkv = shape.batch, shape.max_nodes, shape.num_q_heads, shape.num_kv_heads
+    npg = int(k_pages.shape[0])
+    mp = (shape.max_seq + 127) // 128
+    qp = _req("q", q, torch.bfloat16, (B, N, Hq, 128), dev)
+    kp = _req("k_pages", k_pages, torch.bfloat16, (npg, Hkv, 128, 128), dev)
+    vp_ = _req("v_pages", v_pages, torch.bfloat16, (npg, Hkv, 128, 128), dev)
+    pt = _req("page_table", page_table, torch.int32, (B, mp), dev)
+    op = _req("out", out, torch.bfloat16, (B, N, Hq, 128), dev)
+    args = _tree_args(shape, parent, depth, prefix_len, n_nodes, dev)
+    ws = _req("workspace", workspace, torch.uint8, None, dev)
+    _check("specinfer_tree_attention_paged", load_library().specinfer_tree_attention_paged(
+        ctypes.byref(shape), qp, kp, vp_, npg, pt, *args, op, ws, _stream(q)))
+
+
+def specinfer_kv_commit_paged(shape: Shape, k_pages_all, v_pages_all, page_table, prefix_len, accepted_nodes,
+                              n_accepted):
+    """NEXT-4: KV commit on a paged cache ([L][num_pages][Hkv][128][128])."""
+    dev = k_pages_all.device
+    B, Lp = shape.batch, shape.max_depth + 1
+    npg = int(k_pages_all.shape[-4])
+    mp = (shape.max_seq + 127) // 128
+    for nm, t in (("k_pages_all", k_pages_all), ("v_pages_all", v_pages_all)):
+        _req(nm, t, torch.bfloat16, None, dev)
+        stride = shape.layer_stride or npg * shape.num_kv_heads * 128 * 128
+        if t.numel() < (shape.num_layers - 1) * stride + npg * shape.num_kv_heads * 128 * 128:
+            raise ValueError(f"{nm}: too small for {shape.num_layers} layers")
+    _check("specinfer_kv_commit_paged", load_library().specinfer_kv_commit_paged(
+        ctypes.byref(shape), ctypes.c_void_p(k_pages_all.data_ptr()), ctypes.c_void_p(v_pages_all.data_ptr()), npg,
+        _req("page_table", page_table, torch.int32, (B, mp), dev),
+        _req("prefix_len", prefix_len, torch.int32, (B,), dev),
+        _req("accepted_nodes", accepted_nodes, torch.int32, (B, Lp), dev),
+        _req("n_accepted", n_accepted, torch.int32, (B,), dev), _stream(k_pages_all)))
 
 
 def specinfer_verify_greedy(shape: Shape, logits, tree_tokens, parent, n_nodes, accepted_nodes,

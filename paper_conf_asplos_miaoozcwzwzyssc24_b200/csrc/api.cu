@@ -16,7 +16,8 @@ cudaError_t launch_tree_prepare(const specinfer_shape_t &s, const WsLayout &w, c
                                 char *ws, int num_ctas, cudaStream_t stream);
 cudaError_t launch_tree_attention(const specinfer_shape_t &s, const WsLayout &w, const void *q, const void *k,
                                   const void *v, const int32_t *prefix_len, const int32_t *n_nodes, void *out,
-                                  char *ws, int num_sms, size_t max_smem, cudaStream_t stream);
+                                  char *ws, int num_sms, size_t max_smem, cudaStream_t stream,
+                                  const int32_t *page_table = nullptr, int num_pages = 0);
 cudaError_t launch_verify_greedy(const specinfer_shape_t &s, const WsLayout &w, const float *logits,
                                  const int32_t *tree_tokens, const int32_t *parent, const int32_t *n_nodes,
                                  int32_t *acc_nodes, int32_t *acc_tokens, int32_t *n_acc, char *ws,
@@ -31,7 +32,8 @@ cudaError_t launch_verify_ns(const specinfer_shape_t &s, const WsLayout &w, cons
                              float temperature, uint64_t seed, uint64_t offset, const int32_t *request_ids,
                              int32_t *acc_nodes, int32_t *acc_tokens, int32_t *n_acc, char *ws, cudaStream_t stream);
 cudaError_t launch_kv_commit(const specinfer_shape_t &s, void *k_all, void *v_all, int32_t *prefix_len,
-                             const int32_t *acc_nodes, const int32_t *n_acc, cudaStream_t stream);
+                             const int32_t *acc_nodes, const int32_t *n_acc, cudaStream_t stream,
+                             const int32_t *page_table = nullptr, int num_pages = 0);
 cudaError_t launch_leaf_paths(const specinfer_shape_t &s, const int32_t *parent, const int32_t *n_nodes,
                               int32_t *paths, int32_t *path_len, int32_t *n_leaves, int32_t *status,
                               cudaStream_t stream);
@@ -163,6 +165,44 @@ specinfer_status_t specinfer_tree_attention(const specinfer_shape_t *shape, cons
     return from_cuda(launch_tree_attention(*shape, w, q, k_cache, v_cache, prefix_len, n_nodes, out,
                                            reinterpret_cast<char *>(workspace), w.grid, d.max_smem,
                                            (cudaStream_t)stream));
+}
+
+specinfer_status_t specinfer_tree_attention_paged(const specinfer_shape_t *shape, const void *q, const void *k_pages,
+                                                  const void *v_pages, int32_t num_pages, const int32_t *page_table,
+                                                  const int32_t *parent, const int32_t *depth,
+                                                  const int32_t *prefix_len, const int32_t *n_nodes, void *out,
+                                                  void *workspace, specinfer_stream_t stream) {
+    SPI_TRY(check_shape(shape));
+    if (!q || !k_pages || !v_pages || !page_table || num_pages < 1 || !parent || !depth || !prefix_len ||
+        !n_nodes || !out)
+        return SPECINFER_ERR_INVALID_ARG;
+    if ((long long)num_pages * shape->num_kv_heads * kKeyTile > (1ll << 31) - 1) return SPECINFER_ERR_UNSUPPORTED;
+    if ((reinterpret_cast<uintptr_t>(q) | reinterpret_cast<uintptr_t>(k_pages) |
+         reinterpret_cast<uintptr_t>(v_pages) | reinterpret_cast<uintptr_t>(out)) & 15u)
+        return SPECINFER_ERR_INVALID_ARG;
+    SPI_TRY(check_ws(workspace));
+    DeviceInfo d;
+    SPI_TRY(check_device(&d));
+    const WsLayout w = ws_layout(*shape, d.num_sms);
+    return from_cuda(launch_tree_attention(*shape, w, q, k_pages, v_pages, prefix_len, n_nodes, out,
+                                           reinterpret_cast<char *>(workspace), w.grid, d.max_smem,
+                                           (cudaStream_t)stream, page_table, num_pages));
+}
+
+specinfer_status_t specinfer_kv_commit_paged(const specinfer_shape_t *shape, void *k_pages_all, void *v_pages_all,
+                                             int32_t num_pages, const int32_t *page_table, int32_t *prefix_len,
+                                             const int32_t *accepted_nodes, const int32_t *n_accepted,
+                                             specinfer_stream_t stream) {
+    SPI_TRY(check_shape(shape));
+    if (shape->num_layers < 1 || num_pages < 1) return SPECINFER_ERR_INVALID_ARG;
+    if (!k_pages_all || !v_pages_all || !page_table || !prefix_len || !accepted_nodes || !n_accepted)
+        return SPECINFER_ERR_INVALID_ARG;
+    if ((reinterpret_cast<uintptr_t>(k_pages_all) | reinterpret_cast<uintptr_t>(v_pages_all)) & 15u)
+        return SPECINFER_ERR_INVALID_ARG;
+    DeviceInfo d;
+    SPI_TRY(check_device(&d));
+    return from_cuda(launch_kv_commit(*shape, k_pages_all, v_pages_all, prefix_len, accepted_nodes, n_accepted,
+                                      (cudaStream_t)stream, page_table, num_pages));
 }
 
 specinfer_status_t specinfer_verify_greedy(const specinfer_shape_t *shape, const float *logits,
@@ -360,6 +400,8 @@ int32_t specinfer_launches_per_call(const char *name) {
     if (!strcmp(name, "leaf_paths")) return 1;
     if (!strcmp(name, "verify_ns")) return 1;
     if (!strcmp(name, "expansion_topology")) return 1;
+    if (!strcmp(name, "tree_attention_paged")) return 1;
+    if (!strcmp(name, "kv_commit_paged")) return 2;
     if (!strcmp(name, "expand_step")) return 1;
     if (!strcmp(name, "tree_merge")) return 1;         // race-argmax + walk fused (last CTA walks)
     if (!strcmp(name, "sequence_pack")) return 1;

@@ -21,6 +21,10 @@ struct AttnParams {
     __nv_bfloat16 *out;
     int B, Nmax, Hq, Hkv, G, Smax, chunks, npc, n_items, nk_slots, nv_slots;
     int lanes;  // CTAs per lock-step group (schedule_kernel); 1 = plain stream-K over items
+    // paged KV (NEXT-4): page_table[b][t] = page holding keys [128 t, 128 t + 128) of request b;
+    // a page is [Hkv][128][128] bf16.  nullptr = contiguous [B][Hkv][Smax][128] caches.
+    const int32_t *page_table;
+    int max_pages, n_pages;
     float scale_log2;
     unsigned long long *trace;  // optional per-tile timestamps (debug), nullptr in production
     int debug_flags;            // experiments only: 1 = skip K/V TMA, 2 = skip MMAs (results invalid)
@@ -58,6 +62,14 @@ constexpr int kMaxSlots = 8;
 struct SegDesc {
     int x, begin, end, ib, ie, b, g, c, P, n;
 };
+
+// First cache row (in the 2D [rows][128] view the tensor maps use) of the 128-key tile of request b,
+// kv-head g that starts at key0 (a multiple of 128): contiguous or through the page table.
+__device__ __forceinline__ int kv_tile_row(const AttnParams &p, int b, int g, int key0) {
+    if (p.page_table == nullptr) return (int)((long long)(b * p.Hkv + g) * p.Smax + key0);
+    const int page = __ldg(p.page_table + (size_t)b * p.max_pages + (key0 / kKeyTile));
+    return (page * p.Hkv + g) * kKeyTile;
+}
 
 __device__ __forceinline__ int cta_start(long long c, long long T, long long NC) {
     return (int)((c * T) / NC);

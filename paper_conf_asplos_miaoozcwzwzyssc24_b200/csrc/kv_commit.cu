@@ -13,10 +13,12 @@
 
 namespace specinfer {
 
+// paged KV (NEXT-4): slot s of request b, kv-head g lives at row (page_table[b][s/128] Hkv + g) 128
+// + s % 128 of the layer's [num_pages][Hkv][128][128] pages; page_table == nullptr: contiguous.
 __global__ void __launch_bounds__(256) kv_commit_copy_kernel(
     __nv_bfloat16 *__restrict__ k_all, __nv_bfloat16 *__restrict__ v_all, const int32_t *__restrict__ prefix_len,
     const int32_t *__restrict__ acc_nodes, const int32_t *__restrict__ n_acc, int L, int B, int Hkv, int Smax,
-    long long layer_stride, int path_len) {
+    long long layer_stride, int path_len, const int32_t *__restrict__ page_table, int max_pages) {
     const long long item = (long long)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
     if (item >= (long long)L * B * Hkv) return;
     const int lane = threadIdx.x & 31;
@@ -26,14 +28,19 @@ __global__ void __launch_bounds__(256) kv_commit_copy_kernel(
     const int n = n_acc[b];
     if (n <= 1) return;
     const int P = prefix_len[b];
-    __nv_bfloat16 *base = (lane < 16 ? k_all : v_all) + (size_t)l * layer_stride + ((size_t)b * Hkv + g) * Smax * kHeadDim;
+    __nv_bfloat16 *layer = (lane < 16 ? k_all : v_all) + (size_t)l * layer_stride;
     const int col = (lane & 15) * 8;  // 8 bf16 = 16 bytes
+    auto row = [&](int slot) -> __nv_bfloat16 * {
+        if (page_table == nullptr) return layer + (((size_t)b * Hkv + g) * Smax + slot) * kHeadDim + col;
+        const int page = page_table[(size_t)b * max_pages + slot / kKeyTile];
+        return layer + (((size_t)page * Hkv + g) * kKeyTile + slot % kKeyTile) * kHeadDim + col;
+    };
     const int32_t *path = acc_nodes + (size_t)b * path_len;
     for (int j = 1; j < n; ++j) {
         const int src = path[j];
         if (src == j) continue;
-        const uint4 v = *reinterpret_cast<const uint4 *>(base + (size_t)(P + src) * kHeadDim + col);
-        *reinterpret_cast<uint4 *>(base + (size_t)(P + j) * kHeadDim + col) = v;
+        const uint4 v = *reinterpret_cast<const uint4 *>(row(P + src));
+        *reinterpret_cast<uint4 *>(row(P + j)) = v;
     }
 }
 
@@ -43,17 +50,21 @@ __global__ void kv_commit_prefix_kernel(int32_t *__restrict__ prefix_len, const 
 }
 
 cudaError_t launch_kv_commit(const specinfer_shape_t &s, void *k_all, void *v_all, int32_t *prefix_len,
-                             const int32_t *acc_nodes, const int32_t *n_acc, cudaStream_t stream) {
-    const long long layer_stride = s.layer_stride > 0
-                                       ? s.layer_stride
-                                       : (long long)s.batch * s.num_kv_heads * s.max_seq * kHeadDim;
+                             const int32_t *acc_nodes, const int32_t *n_acc, cudaStream_t stream,
+                             const int32_t *page_table, int num_pages) {
+    const int max_pages = (s.max_seq + kKeyTile - 1) / kKeyTile;
+    const long long layer_stride =
+        s.layer_stride > 0 ? s.layer_stride
+        : page_table     ? (long long)num_pages * s.num_kv_heads * kKeyTile * kHeadDim
+                         : (long long)s.batch * s.num_kv_heads * s.max_seq * kHeadDim;
     const long long items = (long long)s.num_layers * s.batch * s.num_kv_heads;
     if (items > 0) {
         const int warps_per_block = 8;
         const long long blocks = (items + warps_per_block - 1) / warps_per_block;
         kv_commit_copy_kernel<<<(unsigned)blocks, warps_per_block * 32, 0, stream>>>(
             reinterpret_cast<__nv_bfloat16 *>(k_all), reinterpret_cast<__nv_bfloat16 *>(v_all), prefix_len,
-            acc_nodes, n_acc, s.num_layers, s.batch, s.num_kv_heads, s.max_seq, layer_stride, s.max_depth + 1);
+            acc_nodes, n_acc, s.num_layers, s.batch, s.num_kv_heads, s.max_seq, layer_stride, s.max_depth + 1,
+            page_table, max_pages);
         cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return e;
     }

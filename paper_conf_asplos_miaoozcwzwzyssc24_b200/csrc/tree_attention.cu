@@ -175,11 +175,10 @@ __global__ void __launch_bounds__(224, 1)
                 const int node0 = d.b * p.Nmax + d.c * p.npc;
                 tma_load_3d(qdst, &tm_q, &misc->q_full[qb], 0, d.g * p.G, node0);
                 tma_load_3d(qdst + NT * 128, &tm_q, &misc->q_full[qb], 64, d.g * p.G, node0);
-                const long long rowbase = (long long)(d.b * p.Hkv + d.g) * p.Smax;
                 for (int t = d.begin; t < d.end; ++t, ++lt) {
                     const int key0 = (t - d.ib) * kKeyTile;
                     const int nv = min(kKeyTile, Kend - key0);
-                    const int row0 = (int)(rowbase + key0);
+                    const int row0 = kv_tile_row(p, d.b, d.g, key0);
                     const int slot = lt % NK, f = lt / NK;
                     if (f >= 1) mbar_wait(&misc->k_empty[slot], (f - 1) & 1);
                     SPI_TRACE(0);
@@ -206,11 +205,10 @@ __global__ void __launch_bounds__(224, 1)
                 mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
                 const SegDesc d = misc->seg[ls % kSegRing];
                 const int Kend = d.P + d.n;
-                const long long rowbase = (long long)(d.b * p.Hkv + d.g) * p.Smax;
                 for (int t = d.begin; t < d.end; ++t, ++lt) {
                     const int key0 = (t - d.ib) * kKeyTile;
                     const int nv = min(kKeyTile, Kend - key0);
-                    const int row0 = (int)(rowbase + key0);
+                    const int row0 = kv_tile_row(p, d.b, d.g, key0);
                     const int slot = lt % NV, f = lt / NV;
                     if (f >= 1) mbar_wait(&misc->v_empty[slot], (f - 1) & 1);
                     SPI_TRACE(1);
@@ -660,7 +658,8 @@ static cudaError_t launch_nt(const AttnParams &prm0, const void *q, const void *
                              int num_sms, size_t max_smem, cudaStream_t stream) {
     AttnParams prm = prm0;
     CUtensorMap tq, tk, tv, tk16, tv16, tk4, tv4, tk1, tv1;
-    const uint64_t rows = (uint64_t)prm.B * prm.Hkv * prm.Smax;
+    const uint64_t rows = prm.page_table ? (uint64_t)prm.n_pages * prm.Hkv * kKeyTile
+                                         : (uint64_t)prm.B * prm.Hkv * prm.Smax;
     if (!encode_q(&tq, q, prm.Hq, (uint64_t)prm.B * prm.Nmax, prm.G, prm.npc) ||
         !encode_2d(&tk, k, rows, kKeyTile) || !encode_2d(&tv, v, rows, kKeyTile) ||
         !encode_2d(&tk16, k, rows, 16) || !encode_2d(&tv16, v, rows, 16) || !encode_2d(&tk4, k, rows, 4) ||
@@ -704,8 +703,12 @@ int g_attn_debug_flags = 0;                   // debug only (SPECINFER_DEBUG_FLA
 cudaError_t launch_tree_attention(const specinfer_shape_t &s, const WsLayout &w, const void *q,
                                   const void *k, const void *v, const int32_t *prefix_len,
                                   const int32_t *n_nodes, void *out, char *ws, int num_sms,
-                                  size_t max_smem, cudaStream_t stream) {
+                                  size_t max_smem, cudaStream_t stream, const int32_t *page_table,
+                                  int num_pages) {
     AttnParams prm{};
+    prm.page_table = page_table;
+    prm.max_pages = (s.max_seq + kKeyTile - 1) / kKeyTile;
+    prm.n_pages = num_pages;
     prm.prefix_len = prefix_len;
     prm.n_nodes = n_nodes;
     prm.item_start = reinterpret_cast<const int32_t *>(ws + w.item_start);

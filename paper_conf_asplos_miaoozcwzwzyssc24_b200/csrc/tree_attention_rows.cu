@@ -247,10 +247,9 @@ __global__ void __launch_bounds__(352, 1)
             // one tile of K (is_v = 0) or V (1) of segment d, tile t, into the next ring slot
             auto load = [&](const SegDesc &d, int t, bool is_v) {
                 const int Kend = d.P + d.n;
-                const long long rowbase = (long long)(d.b * p.Hkv + d.g) * p.Smax;
                 const int key0 = (t - d.ib) * kKeyTile;
                 const int nv = min(kKeyTile, Kend - key0);
-                const int row0 = (int)(rowbase + key0);
+                const int row0 = kv_tile_row(p, d.b, d.g, key0);
                 const int slot = li % NS, f = li / NS;
                 if (f >= 1) mbar_wait(&misc->empty[slot], (f - 1) & 1);
                 if (li == 0) SPI_TRACE_K(2);
@@ -658,7 +657,8 @@ cudaError_t launch_tree_attention_rows(const AttnParams &prm0, const void *q, co
                                        int num_ctas, size_t max_smem, cudaStream_t stream) {
     AttnParams prm = prm0;
     CUtensorMap tq, tk, tv, tk16, tv16, tk4, tv4, tk1, tv1;
-    const uint64_t rows = (uint64_t)prm.B * prm.Hkv * prm.Smax;
+    const uint64_t rows = prm.page_table ? (uint64_t)prm.n_pages * prm.Hkv * kKeyTile
+                                         : (uint64_t)prm.B * prm.Hkv * prm.Smax;
     if (!encode_q(&tq, q, prm.Hq, (uint64_t)prm.B * prm.Nmax, prm.G, prm.npc) ||
         !encode_2d(&tk, k, rows, kKeyTile) || !encode_2d(&tv, v, rows, kKeyTile) ||
         !encode_2d(&tk16, k, rows, 16) || !encode_2d(&tv16, v, rows, 16) || !encode_2d(&tk4, k, rows, 4) ||
