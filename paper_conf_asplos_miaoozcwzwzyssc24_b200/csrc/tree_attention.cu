@@ -48,7 +48,7 @@ struct SmemMisc {
     uint64_t seg_full[kSegRing];
     SegDesc seg[kSegRing];
     uint32_t tmem_base;
-    int32_t flags[2][4];
+    int32_t flags[2][8];
     int32_t bcast;
     alignas(16) float m_thr[64];   // running row max + threshold (-inf: no key seen yet)
     alignas(16) float m_ref[64];   // running row max used as exp2 reference (0 if none yet)
@@ -62,13 +62,18 @@ struct SmemMisc {
 };
 
 template <int NT>
-__global__ void __launch_bounds__(224, 1)
+__global__ void __launch_bounds__(NT == 64 ? 352 : 224, 1)
     tree_attn_kernel(const __grid_constant__ CUtensorMap tm_q, const __grid_constant__ CUtensorMap tm_k,
                      const __grid_constant__ CUtensorMap tm_v, const __grid_constant__ CUtensorMap tm_k16,
                      const __grid_constant__ CUtensorMap tm_v16, const __grid_constant__ CUtensorMap tm_k4,
                      const __grid_constant__ CUtensorMap tm_v4, const __grid_constant__ CUtensorMap tm_k1,
                      const __grid_constant__ CUtensorMap tm_v1, const AttnParams p) {
     using Plan = SmemPlan<NT>;
+    // NT = 64: 8 softmax warps, two per TMEM lane quarter, each owning half of the query rows
+    // (columns of S^T) of its key: half the registers and two warps per SMSP to hide latency
+    constexpr int kSplit = NT == 64 ? 2 : 1;
+    constexpr int NTH = NT / kSplit;  // query rows per softmax thread
+    constexpr int kSoft = 128 * kSplit;
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     // keep the pointer derived from smem_raw so the compiler emits LDS/STS, not generic LD/ST
     uint8_t *smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
@@ -97,9 +102,9 @@ __global__ void __launch_bounds__(224, 1)
             mbar_init(&misc->q_full[i], 1);
             mbar_init(&misc->q_empty[i], 1);
             mbar_init(&misc->s_full[i], 1);
-            mbar_init(&misc->s_empty[i], 4);
+            mbar_init(&misc->s_empty[i], 4 * kSplit);
         }
-        mbar_init(&misc->p_full, 4);
+        mbar_init(&misc->p_full, 4 * kSplit);
         mbar_init(&misc->p_empty, 1);
         for (int i = 0; i < kSegRing; ++i) mbar_init(&misc->seg_full[i], 1);
         fence_barrier_init();
@@ -117,10 +122,10 @@ __global__ void __launch_bounds__(224, 1)
     }
     if (warp >= 3) {
         // Q rows beyond a chunk's G*npc rows are never written by TMA: keep them zero
-        for (int i = threadIdx.x - 96; i < 2 * Plan::kQBuf / 16; i += 128)
+        for (int i = threadIdx.x - 96; i < 2 * Plan::kQBuf / 16; i += kSoft)
             reinterpret_cast<uint4 *>(s_q)[i] = make_uint4(0, 0, 0, 0);
         // V rows past a request's last key are never loaded: they must hold finite data (0 * NaN)
-        for (int i = threadIdx.x - 96; i < NV * kSlotBytes / 16; i += 128)
+        for (int i = threadIdx.x - 96; i < NV * kSlotBytes / 16; i += kSoft)
             reinterpret_cast<uint4 *>(s_v)[i] = make_uint4(0, 0, 0, 0);
         fence_proxy_async_smem();
     }
@@ -295,7 +300,9 @@ __global__ void __launch_bounds__(224, 1)
         }
     } else {
         // ======================= softmax / epilogue warps =======================
-        const int st = threadIdx.x - 96;       // 0..127
+        const int st = threadIdx.x - 96;       // 0..kSoft-1
+        const int half = st >> 7;              // which half of the query rows (kSplit = 2)
+        const int r0 = half * NTH;             // first query row (S^T / O^T column) of this thread
         const int qd = warp & 3;               // TMEM lane quarter of this warp
         const int kt = qd * 32 + lane;         // key within tile (S^T lane) / head dim (O^T lane)
         const int d = kt;
@@ -320,16 +327,16 @@ __global__ void __launch_bounds__(224, 1)
                     rm[i] = __ldg(p.rowmask + ((size_t)b * p.chunks + c) * p.Nmax + (kk - P));
             }
             // reset row statistics
-            if (qd == 0) {
+            if (st < 32) {
                 for (int r = lane; r < NT; r += 32) {
                     misc->m_thr[r] = -INFINITY;
                     misc->m_ref[r] = 0.f;
                 }
             }
-            float lsum[NT];
+            float lsum[NTH];
 #pragma unroll
-            for (int r = 0; r < NT; ++r) lsum[r] = 0.f;
-            named_bar_sync(1, 128);
+            for (int r = 0; r < NTH; ++r) lsum[r] = 0.f;
+            named_bar_sync(1, kSoft);
             if (st == 0) SPI_TRACE(10);
 
             for (int t = sd.begin; t < sd.end; ++t, ++lt) {
@@ -340,14 +347,15 @@ __global__ void __launch_bounds__(224, 1)
                 mbar_wait(&misc->s_full[sb], (lt >> 1) & 1);
                 tc_fence_after();
                 if (st == 0) SPI_TRACE(4);
-                float xv[NT];
+                float xv[NTH];
                 {
-                    uint32_t r16[NT / 16][16];
+                    uint32_t r16[NTH / 16][16];
 #pragma unroll
-                    for (int c16 = 0; c16 < NT / 16; ++c16) tmem_ld16(tm_S0 + sb * NT + c16 * 16 + lane_off, r16[c16]);
+                    for (int c16 = 0; c16 < NTH / 16; ++c16)
+                        tmem_ld16(tm_S0 + sb * NT + r0 + c16 * 16 + lane_off, r16[c16]);
                     tmem_ld_wait();
 #pragma unroll
-                    for (int c16 = 0; c16 < NT / 16; ++c16)
+                    for (int c16 = 0; c16 < NTH / 16; ++c16)
 #pragma unroll
                         for (int i = 0; i < 16; ++i) xv[c16 * 16 + i] = __uint_as_float(r16[c16][i]) * p.scale_log2;
                 }
@@ -364,36 +372,38 @@ __global__ void __launch_bounds__(224, 1)
                         vis = i == 0 ? rm[0] : (i == 1 ? rm[1] : rm[2]);
                     }
 #pragma unroll
-                    for (int r = 0; r < NT; ++r)
-                        if (!((vis >> r) & 1ull)) xv[r] = -INFINITY;
+                    for (int r = 0; r < NTH; ++r)
+                        if (!((vis >> (r0 + r)) & 1ull)) xv[r] = -INFINITY;
                 }
                 // ---- does this tile raise a row max beyond the stale tolerance? ----
                 bool need = false;
 #pragma unroll
-                for (int r = 0; r < NT; r += 4) {
-                    const float4 m4 = *reinterpret_cast<const float4 *>(&misc->m_thr[r]);
+                for (int r = 0; r < NTH; r += 4) {
+                    const float4 m4 = *reinterpret_cast<const float4 *>(&misc->m_thr[r0 + r]);
                     need |= (xv[r] > m4.x) | (xv[r + 1] > m4.y) | (xv[r + 2] > m4.z) | (xv[r + 3] > m4.w);
                 }
                 const unsigned ballot = __ballot_sync(0xffffffffu, need);
-                if (lane == 0) misc->flags[sb][qd] = ballot != 0u;
+                if (lane == 0) misc->flags[sb][half * 4 + qd] = ballot != 0u;
                 bulk_wait_read_all();  // output staging (P^T buffer) read by the bulk stores
-                named_bar_sync(1, 128);
-                const bool rescale = (misc->flags[sb][0] | misc->flags[sb][1] | misc->flags[sb][2] |
-                                      misc->flags[sb][3]) != 0;
+                named_bar_sync(1, kSoft);
+                int any_flag = 0;
+#pragma unroll
+                for (int f = 0; f < 4 * kSplit; ++f) any_flag |= misc->flags[sb][f];
+                const bool rescale = any_flag != 0;
                 if (rescale) {
                     // exact tile max per row: transpose-reduce within the warp, combine 4 warps
 #pragma unroll
-                    for (int blk = 0; blk < (NT + 31) / 32; ++blk) {
-                        constexpr int W = NT < 32 ? NT : 32;
+                    for (int blk = 0; blk < (NTH + 31) / 32; ++blk) {
+                        constexpr int W = NTH < 32 ? NTH : 32;
                         float mx[W];
 #pragma unroll
                         for (int r = 0; r < W; ++r) mx[r] = xv[blk * 32 + r];
                         transpose_reduce<W, true>(mx);
-                        const int row = blk * 32 + (lane & (W - 1));
+                        const int row = r0 + blk * 32 + (lane & (W - 1));
                         if (lane < W) misc->wred[qd][row] = mx[0];
                     }
-                    named_bar_sync(1, 128);
-                    if (qd == 0) {
+                    named_bar_sync(1, kSoft);
+                    if (st < 32) {
                         for (int r = lane; r < NT; r += 32) {
                             const float tmx = fmaxf(fmaxf(misc->wred[0][r], misc->wred[1][r]),
                                                     fmaxf(misc->wred[2][r], misc->wred[3][r]));
@@ -404,30 +414,30 @@ __global__ void __launch_bounds__(224, 1)
                             misc->m_ref[r] = (mn == -INFINITY) ? 0.f : mn;
                         }
                     }
-                    named_bar_sync(1, 128);
+                    named_bar_sync(1, kSoft);
 #pragma unroll
-                    for (int r = 0; r < NT; ++r) lsum[r] *= misc->alpha[r];
+                    for (int r = 0; r < NTH; ++r) lsum[r] *= misc->alpha[r0 + r];
                     if (t != sd.begin) {
                         // O^T columns (query rows) scaled by alpha: wait for PV of tile lt-1
                         mbar_wait(&misc->p_empty, (lt - 1) & 1);
                         tc_fence_after();
                         uint32_t r16[16];
 #pragma unroll
-                        for (int c16 = 0; c16 < NT / 16; ++c16) {
-                            tmem_ld16(tm_O + c16 * 16 + lane_off, r16);
+                        for (int c16 = 0; c16 < NTH / 16; ++c16) {
+                            tmem_ld16(tm_O + r0 + c16 * 16 + lane_off, r16);
                             tmem_ld_wait();
 #pragma unroll
                             for (int i = 0; i < 16; ++i)
-                                r16[i] = __float_as_uint(__uint_as_float(r16[i]) * misc->alpha[c16 * 16 + i]);
-                            tmem_st16(tm_O + c16 * 16 + lane_off, r16);
+                                r16[i] = __float_as_uint(__uint_as_float(r16[i]) * misc->alpha[r0 + c16 * 16 + i]);
+                            tmem_st16(tm_O + r0 + c16 * 16 + lane_off, r16);
                         }
                         tmem_st_wait();
                     }
                 }
                 // ---- probabilities, row sums ----
 #pragma unroll
-                for (int r = 0; r < NT; r += 4) {
-                    const float4 m4 = *reinterpret_cast<const float4 *>(&misc->m_ref[r]);
+                for (int r = 0; r < NTH; r += 4) {
+                    const float4 m4 = *reinterpret_cast<const float4 *>(&misc->m_ref[r0 + r]);
                     xv[r] = ex2(xv[r] - m4.x);
                     xv[r + 1] = ex2(xv[r + 1] - m4.y);
                     xv[r + 2] = ex2(xv[r + 2] - m4.z);
@@ -435,9 +445,9 @@ __global__ void __launch_bounds__(224, 1)
                 }
                 // P rounded to bf16 once; the row sums use the rounded values so that the
                 // normalisation matches the numerator the PV MMA computes
-                uint32_t pk[NT / 2];
+                uint32_t pk[NTH / 2];
 #pragma unroll
-                for (int i = 0; i < NT / 2; ++i) {
+                for (int i = 0; i < NTH / 2; ++i) {
                     pk[i] = pack_bf16x2(xv[2 * i], xv[2 * i + 1]);
                     lsum[2 * i] += __uint_as_float(pk[i] << 16);
                     lsum[2 * i + 1] += __uint_as_float(pk[i] & 0xFFFF0000u);
@@ -447,8 +457,8 @@ __global__ void __launch_bounds__(224, 1)
                 {
                     uint8_t *pb = s_p;
 #pragma unroll
-                    for (int c8 = 0; c8 < NT / 8; ++c8) {
-                        const uint32_t o = (uint32_t)kt * (NT * 2) + c8 * 16;
+                    for (int c8 = 0; c8 < NTH / 8; ++c8) {
+                        const uint32_t o = (uint32_t)kt * (NT * 2) + (half * (NTH / 8) + c8) * 16;
                         const uint32_t phys = o ^ (((o >> 7) & Plan::kPMask) << 4);
                         *reinterpret_cast<uint4 *>(pb + phys) =
                             make_uint4(pk[c8 * 4], pk[c8 * 4 + 1], pk[c8 * 4 + 2], pk[c8 * 4 + 3]);
@@ -464,34 +474,35 @@ __global__ void __launch_bounds__(224, 1)
                     // ============ epilogue of this segment ============
                     // row sums over the 128 keys of every tile: reduce the per-thread partials
 #pragma unroll
-                    for (int blk = 0; blk < (NT + 31) / 32; ++blk) {
-                        constexpr int W = NT < 32 ? NT : 32;
+                    for (int blk = 0; blk < (NTH + 31) / 32; ++blk) {
+                        constexpr int W = NTH < 32 ? NTH : 32;
                         transpose_reduce<W, false>(lsum + blk * 32);
-                        const int row = blk * 32 + (lane & (W - 1));
+                        const int row = r0 + blk * 32 + (lane & (W - 1));
                         if (lane < W) misc->l_part[qd][row] = lsum[blk * 32];
                     }
                     mbar_wait(&misc->p_empty, lt & 1);  // last PV done
                     tc_fence_after();
                     if (st == 0) SPI_TRACE(6);
-                    float o[NT];
+                    float o[NTH];
                     {
-                        uint32_t r16[NT / 16][16];
+                        uint32_t r16[NTH / 16][16];
 #pragma unroll
-                        for (int c16 = 0; c16 < NT / 16; ++c16) tmem_ld16(tm_O + c16 * 16 + lane_off, r16[c16]);
+                        for (int c16 = 0; c16 < NTH / 16; ++c16)
+                            tmem_ld16(tm_O + r0 + c16 * 16 + lane_off, r16[c16]);
                         tmem_ld_wait();
 #pragma unroll
-                        for (int c16 = 0; c16 < NT / 16; ++c16)
+                        for (int c16 = 0; c16 < NTH / 16; ++c16)
 #pragma unroll
                             for (int i = 0; i < 16; ++i) o[c16 * 16 + i] = __uint_as_float(r16[c16][i]);
                     }
                     tc_fence_before();
-                    named_bar_sync(1, 128);  // all l_part visible
+                    named_bar_sync(1, kSoft);  // all l_part visible
                     if (st < NT) {
                         const float l = misc->l_part[0][st] + misc->l_part[1][st] + misc->l_part[2][st] + misc->l_part[3][st];
                         misc->run_l[st] = l;           // row sum of this segment
                         misc->alpha[st] = 1.0f / l;    // its reciprocal (inf for rows with no key)
                     }
-                    named_bar_sync(1, 128);
+                    named_bar_sync(1, kSoft);
                     if (st == 0) SPI_TRACE(9);
                     const bool full = (sd.begin == sd.ib) && (sd.end == sd.ie);
                     const int rc = G * p.npc;
@@ -500,15 +511,15 @@ __global__ void __launch_bounds__(224, 1)
                         // node contiguous) and write each node's G rows with one bulk async copy
                         __nv_bfloat16 *stg = reinterpret_cast<__nv_bfloat16 *>(s_p);
 #pragma unroll
-                        for (int r = 0; r < NT; r += 4) {
-                            const float4 inv = *reinterpret_cast<const float4 *>(&misc->alpha[r]);
-                            stg[(r + 0) * kHeadDim + d] = __float2bfloat16_rn(o[r + 0] * inv.x);
-                            stg[(r + 1) * kHeadDim + d] = __float2bfloat16_rn(o[r + 1] * inv.y);
-                            stg[(r + 2) * kHeadDim + d] = __float2bfloat16_rn(o[r + 2] * inv.z);
-                            stg[(r + 3) * kHeadDim + d] = __float2bfloat16_rn(o[r + 3] * inv.w);
+                        for (int r = 0; r < NTH; r += 4) {
+                            const float4 inv = *reinterpret_cast<const float4 *>(&misc->alpha[r0 + r]);
+                            stg[(r0 + r + 0) * kHeadDim + d] = __float2bfloat16_rn(o[r + 0] * inv.x);
+                            stg[(r0 + r + 1) * kHeadDim + d] = __float2bfloat16_rn(o[r + 1] * inv.y);
+                            stg[(r0 + r + 2) * kHeadDim + d] = __float2bfloat16_rn(o[r + 2] * inv.z);
+                            stg[(r0 + r + 3) * kHeadDim + d] = __float2bfloat16_rn(o[r + 3] * inv.w);
                         }
                         fence_proxy_async_smem();
-                        named_bar_sync(1, 128);
+                        named_bar_sync(1, kSoft);
                         const int nodes_here = min(p.npc, n - node0);
                         if (st < nodes_here) {
                             bulk_store_s2g(p.out + (((size_t)b * p.Nmax + node0 + st) * p.Hq + g * G) * kHeadDim,
@@ -520,7 +531,7 @@ __global__ void __launch_bounds__(224, 1)
                         const int slot = (sd.begin == t0) ? 0 : 1;
                         float *po = p.part_o + (((size_t)blockIdx.x * 2 + slot) * NT) * kHeadDim;
 #pragma unroll
-                        for (int r = 0; r < NT; ++r) po[(size_t)r * kHeadDim + d] = o[r];
+                        for (int r = 0; r < NTH; ++r) po[(size_t)(r0 + r) * kHeadDim + d] = o[r];
                         float *pml = p.part_ml + ((size_t)blockIdx.x * 2 + slot) * 2 * NT;
                         if (st < NT) {
                             const float mt = misc->m_thr[st];
@@ -528,7 +539,7 @@ __global__ void __launch_bounds__(224, 1)
                             pml[NT + st] = misc->run_l[st];
                         }
                         __threadfence();
-                        named_bar_sync(1, 128);
+                        named_bar_sync(1, kSoft);
                         if (st == 0) {
                             const int c_first = cta_of_tile(sd.ib, T, NC);
                             const int c_last = cta_of_tile(sd.ie - 1, T, NC);
@@ -539,7 +550,7 @@ __global__ void __launch_bounds__(224, 1)
                             misc->bcast = (old == (unsigned)(npieces - 1)) ? 1 : 0;
                             if (misc->bcast) p.item_cnt[sd.x] = 0u;  // ready for the next launch
                         }
-                        named_bar_sync(1, 128);
+                        named_bar_sync(1, kSoft);
                         if (misc->bcast) {
                             // last piece: merge all pieces' (m, l, O) by log-sum-exp, pieces staged
                             // kCombineBatch at a time so every global load of a batch is in flight
@@ -548,9 +559,9 @@ __global__ void __launch_bounds__(224, 1)
                                 misc->run_m[st] = -INFINITY;
                                 misc->run_l[st] = 0.f;
                             }
-                            float acc[NT];
+                            float acc[NTH];
 #pragma unroll
-                            for (int r = 0; r < NT; ++r) acc[r] = 0.f;
+                            for (int r = 0; r < NTH; ++r) acc[r] = 0.f;
                             // the P^T buffer is idle during an epilogue (last PV done, next P not yet written)
                             float *cmb_m = reinterpret_cast<float *>(s_p);
                             float *cmb_l = cmb_m + kCombineBatch * NT;
@@ -561,7 +572,7 @@ __global__ void __launch_bounds__(224, 1)
                                 c_last = cta_of_tile(sd.ie - 1, T, NC);
                             }
                             for (;;) {
-                                named_bar_sync(1, 128);
+                                named_bar_sync(1, kSoft);
                                 if (st == 0) {
                                     int nb = 0;
                                     while (cc <= c_last && nb < kCombineBatch) {
@@ -574,16 +585,16 @@ __global__ void __launch_bounds__(224, 1)
                                     }
                                     misc->bcast = nb;
                                 }
-                                named_bar_sync(1, 128);
+                                named_bar_sync(1, kSoft);
                                 const int nb = misc->bcast;
                                 if (nb == 0) break;
-                                for (int idx = st; idx < nb * NT; idx += 128) {
+                                for (int idx = st; idx < nb * NT; idx += kSoft) {
                                     const int pc = idx / NT, r = idx - pc * NT;
                                     const float *pm = p.part_ml + misc->piece_off[pc] * 2 * NT;
                                     cmb_m[pc * NT + r] = ldcg_f32(pm + r);
                                     cmb_l[pc * NT + r] = ldcg_f32(pm + NT + r);
                                 }
-                                named_bar_sync(1, 128);
+                                named_bar_sync(1, kSoft);
                                 if (st < NT) {
                                     const int r = st;
                                     float bm = -INFINITY;
@@ -602,33 +613,30 @@ __global__ void __launch_bounds__(224, 1)
                                     misc->run_l[r] = L;
                                     misc->alpha[r] = sc;
                                 }
-                                named_bar_sync(1, 128);
+                                named_bar_sync(1, kSoft);
 #pragma unroll
-                                for (int r = 0; r < NT; ++r) acc[r] *= misc->alpha[r];
+                                for (int r = 0; r < NTH; ++r) acc[r] *= misc->alpha[r0 + r];
                                 for (int pc = 0; pc < nb; ++pc) {
                                     const float *po2 = p.part_o + misc->piece_off[pc] * NT * kHeadDim + d;
-                                    float v[NT];
+                                    float v[NTH];
 #pragma unroll
-                                    for (int r = 0; r < NT; ++r) v[r] = ldcg_f32(po2 + (size_t)r * kHeadDim);
+                                    for (int r = 0; r < NTH; ++r) v[r] = ldcg_f32(po2 + (size_t)(r0 + r) * kHeadDim);
 #pragma unroll
-                                    for (int r = 0; r < NT; ++r) acc[r] += cmb_w[pc * NT + r] * v[r];
+                                    for (int r = 0; r < NTH; ++r) acc[r] += cmb_w[pc * NT + r0 + r] * v[r];
                                 }
                             }
-                            int node = node0, hl = 0;
 #pragma unroll
-                            for (int r = 0; r < NT; ++r) {
-                                if (r < rc && node < n) {
+                            for (int r = 0; r < NTH; ++r) {
+                                const int rr = r0 + r;
+                                const int node = node0 + rr / G, hl = rr % G;
+                                if (rr < rc && node < n) {
                                     p.out[(((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim + d] =
-                                        __float2bfloat16_rn(__fdividef(acc[r], misc->run_l[r]));
-                                }
-                                if (++hl == G) {
-                                    hl = 0;
-                                    ++node;
+                                        __float2bfloat16_rn(__fdividef(acc[r], misc->run_l[rr]));
                                 }
                             }
                         }
                     }
-                    named_bar_sync(1, 128);  // stats read by everyone before the next reset
+                    named_bar_sync(1, kSoft);  // stats read by everyone before the next reset
                     if (st == 0) SPI_TRACE(7);
                 }
             }
@@ -683,7 +691,7 @@ static cudaError_t launch_nt(const AttnParams &prm0, const void *q, const void *
     // this grid overlaps the tail of the previous kernel on the stream
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(num_sms);
-    cfg.blockDim = dim3(224);
+    cfg.blockDim = dim3(NT == 64 ? 352 : 224);
     cfg.dynamicSmemBytes = smem;
     cfg.stream = stream;
     cudaLaunchAttribute attr[1];

@@ -26,6 +26,7 @@ def main():
     ap.add_argument("--iters", type=int, default=20)
     ap.add_argument("--trace", action="store_true")
     ap.add_argument("--raw", action="store_true", help="with --trace: print the raw per-tile events")
+    ap.add_argument("--expansion", default=None, help="override the tree: comma list <k1,..,km>")
     ap.add_argument("--lib", default=None, help="load this libspecinfer build instead (A/B experiments)")
     ap.add_argument("--flags", type=int, default=0, help="debug flags: 1 skip TMA, 2 skip MMA (timing only)")
     a = ap.parse_args()
@@ -35,8 +36,8 @@ def main():
     dev = torch.device("cuda:0")
     B = a.batch or cfg.batch
     P = a.prefix or cfg.prefix
-    p, d = cfg.tree
-    tb = W.make_tree_batch([(p, d)] * B, [P] * B, device=dev, max_depth=cfg.max_depth)
+    p, d = cfg.tree if not a.expansion else W.expansion_tree([int(x) for x in a.expansion.split(",")])
+    tb = W.make_tree_batch([(p, d)] * B, [P] * B, device=dev, max_depth=max(cfg.max_depth, int(d.max())))
     smax = P + tb.max_nodes
     ai = W.make_attention_inputs(tb, a.layers, cfg.num_q_heads, cfg.num_kv_heads, smax, seed=1, device=dev)
     shape = spi.make_shape(B, tb.max_nodes, cfg.num_q_heads, cfg.num_kv_heads, smax, max_depth=cfg.max_depth)
