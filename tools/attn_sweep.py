@@ -26,7 +26,10 @@ def main():
     ap.add_argument("--prefix", type=int, default=2048)
     ap.add_argument("--heads", type=int, default=32)
     ap.add_argument("--iters", type=int, default=20)
+    ap.add_argument("--lib", default=None, help="load this libspecinfer build instead (A/B experiments)")
     a = ap.parse_args()
+    if a.lib:
+        spi.load_library(a.lib)
     dev = torch.device("cuda:0")
     H = a.heads
     for n in [int(x) for x in a.ns.split(",")]:
