@@ -285,3 +285,45 @@ def tree_merge(trees):
     new_id = {old: new for new, old in enumerate(order)}
     depth = [len(seqs[o]) - 1 for o in order]
     return new_parent, new_tokens, depth, [[new_id[x] for x in m] for m in maps]
+
+
+# --------------------------------------------------------------------------------------------
+# NEXT-4: rotary position encoding of the tree at position P_b + depth[i] (SURVEY A4 / DESIGN R29)
+# --------------------------------------------------------------------------------------------
+
+def rope_inv_freq(head_dim=128, base=10000.0):
+    """Rotary frequencies theta_i = base^(-2i/D), i < D/2, rounded to fp32 (the contract the CUDA
+    path follows: fp32 table, fp32 angle pos * theta_i)."""
+    i = np.arange(head_dim // 2, dtype=np.float64)
+    return np.power(np.float64(base), -2.0 * i / head_dim).astype(np.float32)
+
+
+def rope_rotate(x, pos, base=10000.0):
+    """x [..., D] rotated at integer positions pos [...] (broadcast over the last axis), in fp64.
+    Rotate-half pairing (dims i and i + D/2), as LLaMA: the angle a_i = fp32(pos) * theta_i is
+    formed in fp32 (the contract), then x'_i = x_i cos a_i - x_{i+D/2} sin a_i and
+    x'_{i+D/2} = x_{i+D/2} cos a_i + x_i sin a_i in fp64."""
+    x = np.asarray(x, np.float64)
+    D = x.shape[-1]
+    th = rope_inv_freq(D, base)
+    ang = (np.asarray(pos).astype(np.float32)[..., None] * th).astype(np.float64)  # fp32 product
+    c, s = np.cos(ang), np.sin(ang)
+    lo, hi = x[..., :D // 2], x[..., D // 2:]
+    return np.concatenate([lo * c - hi * s, hi * c + lo * s], axis=-1)
+
+
+def tree_rope(q, k_cache, prefix_len, depth, n_nodes, base=10000.0):
+    """Reading A4: node i of request b sits at position P_b + depth[i] of its sequence S_u
+    (Def. 4.1 L594-598 places u at index depth(u) after the committed prefix).  Rotates the tree
+    queries q [B][Nmax][Hq][D] (rows i < n_b) and the tree keys k_cache [B][Hkv][Smax][D]
+    (slots P_b + i, i < n_b) at that position; everything else is returned unchanged.
+    Returns fp64 (q_rot, k_rot)."""
+    q = np.array(q, np.float64)
+    k = np.array(k_cache, np.float64)
+    for b in range(q.shape[0]):
+        P, n = int(prefix_len[b]), int(n_nodes[b])
+        for i in range(n):
+            pos = P + int(depth[b][i])
+            q[b, i] = rope_rotate(q[b, i], np.full(q.shape[2], pos), base)
+            k[b, :, P + i] = rope_rotate(k[b, :, P + i], np.full(k.shape[1], pos), base)
+    return q, k
