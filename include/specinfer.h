@@ -11,6 +11,7 @@
  *   specinfer_kv_commit       depth-first KV-cache update L635-644; tree-topology KV layout L659-661
  *   specinfer_expansion_topology, specinfer_expand_step, specinfer_tree_merge
  *                             NEXT-2: token-tree construction (§3)
+ *   specinfer_tree_rope       NEXT-4: position encoding at P_b + depth[i] (Def. 4.1, A4)
  *   specinfer_tree_attention_paged, specinfer_kv_commit_paged
  *                             NEXT-4: paged KV cache (tree layout L659-661 over 128-slot pages)
  *   specinfer_verify_ns       NEXT-3: naive sampling, the baseline of Theorem 4.3 (L747-765)
@@ -138,6 +139,22 @@ specinfer_status_t specinfer_verify_mss(const specinfer_shape_t *shape, const fl
                                         const int32_t *request_ids, int32_t *accepted_nodes,
                                         int32_t *accepted_tokens, int32_t *n_accepted,
                                         void *workspace, specinfer_stream_t stream);
+
+/* NEXT-4: rotary position encoding of the tree (reading A4: node i of request b is token number
+ * depth[i] after the committed prefix of S_u, Def. 4.1, so it is encoded at position
+ * P_b + depth[i]; siblings share a position).  In place, one launch:
+ *   q       bf16 [B][Nmax][Hq][128], rows i < n_b rotated (NULL: keys only);
+ *   k_cache bf16 [B][Hkv][Smax][128], ONE layer, tree slots P_b + i (i < n_b) rotated (NULL:
+ *           queries only); committed slots are assumed already encoded at their own positions.
+ * Rotate-half pairs (d, d + 64), theta_d = fp32(rope_base^(-2d/128)), angle = fp32(pos) * theta_d
+ * in fp32, rotation in fp32, rounded to bf16.  rope_base > 1 (LLaMA: 10000).  depth[] must be the
+ * node depths (tree_prepare validates them); requests with n_b outside [1, Nmax] or
+ * P_b + n_b > Smax are left untouched.  After kv_commit, committed slot P + j holds a key encoded at
+ * P + j (path[j] has depth j).  Errors: INVALID_ARG (both q and k_cache NULL, NULL tree arrays,
+ * rope_base <= 1, misaligned pointers), UNSUPPORTED / ERR_CUDA as elsewhere. */
+specinfer_status_t specinfer_tree_rope(const specinfer_shape_t *shape, void *q, void *k_cache,
+                                      const int32_t *prefix_len, const int32_t *depth,
+                                      const int32_t *n_nodes, float rope_base, specinfer_stream_t stream);
 
 /* NEXT-4: paged KV cache (for serving; same computation as tree_attention / kv_commit).
  * Keys of request b live in pages of 128 slots: slot s is row s % 128 of page

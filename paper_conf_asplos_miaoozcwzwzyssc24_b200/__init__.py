@@ -32,7 +32,7 @@ EXPORTED_SYMBOLS = (
     "specinfer_launches_per_call",
     "specinfer_status_string", "specinfer_leaf_paths", "specinfer_sequence_pack",
     "specinfer_verify_ns", "specinfer_expansion_topology", "specinfer_expand_step", "specinfer_tree_merge",
-    "specinfer_tree_attention_paged", "specinfer_kv_commit_paged",
+    "specinfer_tree_attention_paged", "specinfer_kv_commit_paged", "specinfer_tree_rope",
 )
 
 
@@ -83,6 +83,7 @@ def load_library(path: str = LIB_PATH):
     lib.specinfer_philox_debug.argtypes = [vp, vp, i32, vp]
     lib.specinfer_tree_attention_paged.argtypes = [sp, vp, vp, vp, i32, vp, vp, vp, vp, vp, vp, vp, vp]
     lib.specinfer_kv_commit_paged.argtypes = [sp, vp, vp, i32, vp, vp, vp, vp, vp]
+    lib.specinfer_tree_rope.argtypes = [sp, vp, vp, vp, vp, vp, f32, vp]
     lib.specinfer_expansion_topology.argtypes = [sp, vp, i32, vp, vp, vp, vp]
     lib.specinfer_expand_step.argtypes = [sp, i32, i32, vp, f32, vp, vp, vp, vp, vp, vp, vp]
     lib.specinfer_tree_merge.argtypes = [sp, i32, i32, vp, vp, vp, vp, vp, vp, vp, vp, vp, vp]
@@ -99,7 +100,7 @@ def load_library(path: str = LIB_PATH):
                  "specinfer_verify_mss", "specinfer_kv_commit", "specinfer_read_device_status",
                  "specinfer_philox_debug", "specinfer_leaf_paths", "specinfer_sequence_pack", "specinfer_verify_ns",
                  "specinfer_expansion_topology", "specinfer_expand_step", "specinfer_tree_merge",
-                 "specinfer_tree_attention_paged", "specinfer_kv_commit_paged"):
+                 "specinfer_tree_attention_paged", "specinfer_kv_commit_paged", "specinfer_tree_rope"):
         getattr(lib, name).restype = i32
     _lib = lib
     return lib
@@ -212,6 +213,22 @@ def specinfer_kv_commit_paged(shape: Shape, k_pages_all, v_pages_all, page_table
         _req("prefix_len", prefix_len, torch.int32, (B,), dev),
         _req("accepted_nodes", accepted_nodes, torch.int32, (B, Lp), dev),
         _req("n_accepted", n_accepted, torch.int32, (B,), dev), _stream(k_pages_all)))
+
+
+def specinfer_tree_rope(shape: Shape, q, k_cache, prefix_len, depth, n_nodes, rope_base: float = 10000.0):
+    """NEXT-4: rotary position encoding of the tree in place, node i at position P_b + depth[i]
+    (reading A4).  q [B][Nmax][Hq][128] and/or k_cache [B][Hkv][Smax][128] (one layer; tree slots
+    P_b + i), bf16; either may be None."""
+    ref = q if q is not None else k_cache
+    if ref is None:
+        raise ValueError("specinfer_tree_rope: q and k_cache are both None")
+    dev = ref.device
+    B, N = shape.batch, shape.max_nodes
+    _check("specinfer_tree_rope", load_library().specinfer_tree_rope(
+        ctypes.byref(shape), _opt("q", q, torch.bfloat16, (B, N, shape.num_q_heads, 128), dev),
+        _opt("k_cache", k_cache, torch.bfloat16, (B, shape.num_kv_heads, shape.max_seq, 128), dev),
+        _req("prefix_len", prefix_len, torch.int32, (B,), dev), _req("depth", depth, torch.int32, (B, N), dev),
+        _req("n_nodes", n_nodes, torch.int32, (B,), dev), float(rope_base), _stream(ref)))
 
 
 def specinfer_verify_greedy(shape: Shape, logits, tree_tokens, parent, n_nodes, accepted_nodes,

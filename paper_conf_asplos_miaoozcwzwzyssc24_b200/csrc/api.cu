@@ -51,6 +51,8 @@ cudaError_t launch_tree_merge(const specinfer_shape_t &s, int T, int Nin, const 
                               const int32_t *in_tokens, const int32_t *in_n, int32_t *parent, int32_t *depth,
                               int32_t *tokens, int32_t *n_nodes, int32_t *node_map, int32_t *status,
                               cudaStream_t stream);
+cudaError_t launch_tree_rope(const specinfer_shape_t &s, void *q, void *k, const int32_t *prefix_len,
+                             const int32_t *depth, const int32_t *n_nodes, float base, cudaStream_t stream);
 cudaError_t launch_philox_debug(const uint32_t *ck, uint32_t *out, int n, cudaStream_t stream);
 extern unsigned long long *g_attn_trace;
 extern int g_attn_debug_flags;
@@ -203,6 +205,17 @@ specinfer_status_t specinfer_kv_commit_paged(const specinfer_shape_t *shape, voi
     SPI_TRY(check_device(&d));
     return from_cuda(launch_kv_commit(*shape, k_pages_all, v_pages_all, prefix_len, accepted_nodes, n_accepted,
                                       (cudaStream_t)stream, page_table, num_pages));
+}
+
+specinfer_status_t specinfer_tree_rope(const specinfer_shape_t *shape, void *q, void *k_cache,
+                                      const int32_t *prefix_len, const int32_t *depth, const int32_t *n_nodes,
+                                      float rope_base, specinfer_stream_t stream) {
+    SPI_TRY(check_shape(shape));
+    if ((!q && !k_cache) || !prefix_len || !depth || !n_nodes || !(rope_base > 1.0f)) return SPECINFER_ERR_INVALID_ARG;
+    if ((reinterpret_cast<uintptr_t>(q) | reinterpret_cast<uintptr_t>(k_cache)) & 3u) return SPECINFER_ERR_INVALID_ARG;
+    DeviceInfo d;
+    SPI_TRY(check_device(&d));
+    return from_cuda(launch_tree_rope(*shape, q, k_cache, prefix_len, depth, n_nodes, rope_base, (cudaStream_t)stream));
 }
 
 specinfer_status_t specinfer_verify_greedy(const specinfer_shape_t *shape, const float *logits,
@@ -405,6 +418,7 @@ int32_t specinfer_launches_per_call(const char *name) {
     if (!strcmp(name, "expand_step")) return 1;
     if (!strcmp(name, "tree_merge")) return 1;         // race-argmax + walk fused (last CTA walks)
     if (!strcmp(name, "sequence_pack")) return 1;
+    if (!strcmp(name, "tree_rope")) return 1;
     return -1;
 }
 

@@ -89,6 +89,28 @@ def test_attention_random_trees(Hq, Hkv, Nmax, P):
         assert torch.isnan(out[b, n[b]:].float()).all()
 
 
+@pytest.mark.parametrize("Hq,Hkv,Nmax", [(4, 4, 16), (2, 2, 100), (8, 1, 40)])
+@pytest.mark.parametrize("spike", [8.0, 30.0, 200.0])
+def test_attention_score_spikes(Hq, Hkv, Nmax, spike):
+    """Keys scaled by large factors inside later chunks / tiles (committed and tree keys), so a row's
+    running softmax reference has to move mid-tile and across tiles by far more than any stale-max
+    slack; with spike 200 the scores jump by hundreds of log2 units (one-hot rows)."""
+    B = 2
+    rng = np.random.default_rng(int(spike) + Nmax)
+    trees = [W.random_tree(Nmax, 8, 4, rng), W.random_tree(int(rng.integers(1, Nmax + 1)), 8, 4, rng)]
+    P = 300
+    pls = [P, P - 100]
+    tb = W.make_tree_batch(trees, pls, max_nodes=Nmax, max_depth=8, device=DEV)
+    smax = max(pls) + Nmax + 7
+    ai = W.make_attention_inputs(tb, 1, Hq, Hkv, smax, seed=int(spike), device=DEV, poison=True)
+    for b, pb in enumerate(pls):
+        for j, f in ((70, spike / 4), (150, spike / 2), (pb - 1, spike), (pb + 3, spike * 1.5)):
+            ai.k_cache[0, b, :, j] = (ai.k_cache[0, b, :, j].float() * f).to(torch.bfloat16)
+    out, _ = _gpu_attention(tb, ai, Hq, Hkv)
+    ref = _oracle_attention(ai, tb)
+    _check_rows(out, ref, tb)
+
+
 @pytest.mark.parametrize("peaky", [False, True])
 def test_attention_chain_and_figures(golden, peaky):
     """Fig. 4 tree (L682), a 40-node chain (= causal decoding), root-only trees; peaky q (x4)
