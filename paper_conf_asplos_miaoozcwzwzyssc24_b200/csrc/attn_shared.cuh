@@ -72,15 +72,16 @@ __device__ __forceinline__ int kv_tile_row(const AttnParams &p, int b, int g, in
 }
 
 __device__ __forceinline__ int cta_start(long long c, long long T, long long NC) {
+    // 32-bit division when c * T fits (every practical schedule); 64-bit division is emulated
+    if (c * T <= 0xFFFFFFFFll) return (int)((uint32_t)(c * T) / (uint32_t)NC);
     return (int)((c * T) / NC);
 }
 
 __device__ __forceinline__ int cta_of_tile(int t, int T, int NC) {
-    int c = (int)(((long long)t * NC) / T);
-    if (c >= NC) c = NC - 1;
-    while (c + 1 < NC && cta_start(c + 1, T, NC) <= t) ++c;
-    while (c > 0 && cta_start(c, T, NC) > t) --c;
-    return c;
+    // the largest c with cta_start(c) <= t: floor(c T / NC) <= t <=> c T < (t + 1) NC
+    const long long num = (long long)(t + 1) * NC - 1;
+    int c = num <= 0xFFFFFFFFll ? (int)((uint32_t)num / (uint32_t)T) : (int)(num / T);
+    return c < NC ? c : NC - 1;
 }
 
 // Cross-lane "transpose reduction": on entry each lane holds N values (one per row); on exit

@@ -121,8 +121,16 @@ __global__ void __launch_bounds__(1024) schedule_kernel(
         if (c * npc >= n) return 0;
         return (prefix_len[b] + n + kKeyTile - 1) / kKeyTile;
     };
-    int local = 0;
-    for (int u = lo; u < hi; ++u) local += tiles_of(u);
+    int local = 0, local_max = 0;
+    for (int u = lo; u < hi; ++u) {
+        const int tl = tiles_of(u);
+        local += tl;
+        local_max = max(local_max, tl);
+    }
+    __shared__ int s_max_tiles;
+    if (threadIdx.x == 0) s_max_tiles = 0;
+    __syncthreads();
+    atomicMax(&s_max_tiles, local_max);
     // block exclusive scan of per-thread sums
     __shared__ int s_warp[32];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -167,11 +175,26 @@ __global__ void __launch_bounds__(1024) schedule_kernel(
     }
     for (int b = threadIdx.x; b < 2 * B; b += blockDim.x) verify_cnt[b] = 0u;
     __syncthreads();
-    // per-CTA slice [t0, t1) of the unit tile sequence, and its first item
+    // per-CTA slice [t0, t1) of the unit tile sequence, and its first item.
+    // Small problems (every unit fits a CTA group and the longest unit is at most kNoSplitSlack
+    // tiles longer than an even stream-K share): one unit per CTA group, no split, so no split
+    // combine -- its partial write / atomic / merge code runs cold once per launch (~10 us of
+    // instruction-cache misses at the kernel's tail, measured) and costs more than the
+    // parallelism it buys (C1: 2 tiles per unit; B = 1..4 at P = 2048: 17).  Otherwise even stream-K slices.
     const long long T = s_total;
     const int NCv = num_ctas / lanes;
+    constexpr int kNoSplitSlack = 16;
+    const bool one_per_cta = n_units <= NCv && (long long)s_max_tiles * NCv <= T + (long long)kNoSplitSlack * NCv;
     for (int c = threadIdx.x; c < num_ctas; c += blockDim.x) {
         const int vc = c / lanes, cl = c % lanes;
+        if (one_per_cta) {
+            const int t0 = vc < n_units ? item_start[vc] : (int)T;
+            const int t1 = vc < n_units ? item_start[vc + 1] : (int)T;
+            const int x0 = vc < n_units ? vc * lanes + cl : n_items;
+            cta_info[2 * c] = make_int4(t0, t1, x0, (int)T);
+            cta_info[2 * c + 1] = x0 < n_items ? item_info[x0] : make_int4(0, 0, 0, 0);
+            continue;
+        }
         const int t0 = (int)((long long)vc * T / NCv);
         const int t1 = (int)((long long)(vc + 1) * T / NCv);
         int lo2 = 0, hi2 = n_units;  // last unit with start <= t0

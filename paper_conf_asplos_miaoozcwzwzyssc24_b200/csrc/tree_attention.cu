@@ -45,6 +45,7 @@ struct SmemMisc {
     uint64_t q_full[2], q_empty[2];
     uint64_t s_full[2], s_empty[2];
     uint64_t p_full, p_empty;  // single P^T buffer: written by softmax(t) after PV(t-1) read it
+    uint64_t cmb_bar;          // bulk staging of the split pieces (at most one merge per CTA uses it)
     uint64_t seg_full[kSegRing];
     SegDesc seg[kSegRing];
     uint32_t tmem_base;
@@ -59,6 +60,7 @@ struct SmemMisc {
     alignas(16) float run_m[64];
     alignas(16) float run_l[64];
     size_t piece_off[kCombineBatch];
+    int32_t npieces;
 };
 
 template <int NT>
@@ -106,6 +108,7 @@ __global__ void __launch_bounds__(NT == 64 ? 352 : 224, 1)
         }
         mbar_init(&misc->p_full, 4 * kSplit);
         mbar_init(&misc->p_empty, 1);
+        mbar_init(&misc->cmb_bar, 1);
         for (int i = 0; i < kSegRing; ++i) mbar_init(&misc->seg_full[i], 1);
         fence_barrier_init();
     }
@@ -540,6 +543,7 @@ __global__ void __launch_bounds__(NT == 64 ? 352 : 224, 1)
                         }
                         __threadfence();
                         named_bar_sync(1, kSoft);
+                        if (st == 0) SPI_TRACE(8);
                         if (st == 0) {
                             const int c_first = cta_of_tile(sd.ib, T, NC);
                             const int c_last = cta_of_tile(sd.ie - 1, T, NC);
@@ -551,17 +555,89 @@ __global__ void __launch_bounds__(NT == 64 ? 352 : 224, 1)
                             if (misc->bcast) p.item_cnt[sd.x] = 0u;  // ready for the next launch
                         }
                         named_bar_sync(1, kSoft);
+                        if (st == 0) SPI_TRACE(11);
                         if (misc->bcast) {
-                            // last piece: merge all pieces' (m, l, O) by log-sum-exp, pieces staged
-                            // kCombineBatch at a time so every global load of a batch is in flight
+                            // last piece: merge all pieces' (m, l, O) by log-sum-exp
                             __threadfence();
+// merge-phase trace points go to the (unused) row of tile lt + 1: 0 start, 1 pieces issued,
+// 2 staged, 3 weights, 4 accumulated, 5 stored
+#define SPI_TRACE2(ev) do { if (st == 0 && p.trace != nullptr && blockIdx.x < kTraceCtas && lt + 1 < kTraceTiles) \
+    p.trace[((size_t)blockIdx.x * kTraceTiles + lt + 1) * kTraceEv + (ev)] = clock64(); } while (0)
+                            SPI_TRACE2(0);
+                            float acc[NTH];
+#pragma unroll
+                            for (int r = 0; r < NTH; ++r) acc[r] = 0.f;
+                            // CTA's last segment => the K / V rings are idle: stage every piece's
+                            // (O, m, l) there with bulk copies (one L2 round trip for all pieces).
+                            // One thread enumerates the pieces; the rest of the merge is unrolled over
+                            // this thread's rows (latency-bound code: 4 warps, ILP from the rows).
+                            constexpr uint32_t kOBytes = NT * kHeadDim * 4, kMLBytes = 2 * NT * 4;
+                            float *so = reinterpret_cast<float *>(s_k);
+                            if (st == 0) {
+                                int npcs = -1;
+                                if (sd.end == t1) {  // no tile of this CTA follows: rings idle
+                                    npcs = 0;
+                                    const int cf = cta_of_tile(sd.ib, T, NC), cl2 = cta_of_tile(sd.ie - 1, T, NC);
+                                    for (int cc = cf; cc <= cl2 && npcs <= kCombineBatch; ++cc) {
+                                        const int s0 = cta_start(cc, T, NC);
+                                        if (cta_start(cc + 1, T, NC) <= s0) continue;
+                                        if (npcs < kCombineBatch) misc->piece_off[npcs] = (size_t)cc * 2 + ((s0 >= sd.ib) ? 0 : 1);
+                                        ++npcs;
+                                    }
+                                    if (npcs > kCombineBatch ||
+                                        (size_t)npcs * (kOBytes + kMLBytes) > (size_t)(NK + NV) * kSlotBytes)
+                                        npcs = -1;
+                                }
+                                misc->npieces = npcs;
+                                if (npcs > 0) {
+                                    fence_proxy_async_global();
+                                    mbar_arrive_expect_tx(&misc->cmb_bar, (uint32_t)npcs * (kOBytes + kMLBytes));
+                                    float *sml = so + (size_t)npcs * NT * kHeadDim;
+                                    for (int pc = 0; pc < npcs; ++pc) {
+                                        const size_t off = misc->piece_off[pc];
+                                        bulk_load_g2s(so + (size_t)pc * NT * kHeadDim, p.part_o + off * NT * kHeadDim,
+                                                      kOBytes, &misc->cmb_bar);
+                                        bulk_load_g2s(sml + pc * 2 * NT, p.part_ml + off * 2 * NT, kMLBytes, &misc->cmb_bar);
+                                    }
+                                }
+                            }
+                            named_bar_sync(1, kSoft);
+                            const int npcs = misc->npieces;
+                            SPI_TRACE2(1);
+                            if (npcs > 0) {
+                                const float *sml = so + (size_t)npcs * NT * kHeadDim;
+                                float *cmb_w = reinterpret_cast<float *>(s_p);
+                                mbar_wait(&misc->cmb_bar, 0);
+                                SPI_TRACE2(2);
+                                if (st < NT) {
+                                    const int r = st;
+                                    float M = -INFINITY;
+                                    for (int pc = 0; pc < npcs; ++pc) M = fmaxf(M, sml[pc * 2 * NT + r]);
+                                    float L = 0.f;
+                                    for (int pc = 0; pc < npcs; ++pc) {
+                                        const float mp = sml[pc * 2 * NT + r];
+                                        const float w = (mp == -INFINITY) ? 0.f : ex2(mp - M);
+                                        cmb_w[pc * NT + r] = w;
+                                        L += w * sml[pc * 2 * NT + NT + r];
+                                    }
+                                    misc->run_l[r] = L;
+                                }
+                                named_bar_sync(1, kSoft);
+                                SPI_TRACE2(3);
+                                for (int pc = 0; pc < npcs; ++pc) {
+                                    const float *po2 = so + (size_t)pc * NT * kHeadDim + d;
+#pragma unroll
+                                    for (int r = 0; r < NTH; ++r)
+                                        acc[r] += cmb_w[pc * NT + r0 + r] * po2[(size_t)(r0 + r) * kHeadDim];
+                                }
+                                SPI_TRACE2(4);
+                            } else {
+                            // pieces staged kCombineBatch at a time through the idle P^T buffer so every
+                            // global load of a batch is in flight
                             if (st < NT) {
                                 misc->run_m[st] = -INFINITY;
                                 misc->run_l[st] = 0.f;
                             }
-                            float acc[NTH];
-#pragma unroll
-                            for (int r = 0; r < NTH; ++r) acc[r] = 0.f;
                             // the P^T buffer is idle during an epilogue (last PV done, next P not yet written)
                             float *cmb_m = reinterpret_cast<float *>(s_p);
                             float *cmb_l = cmb_m + kCombineBatch * NT;
@@ -625,15 +701,22 @@ __global__ void __launch_bounds__(NT == 64 ? 352 : 224, 1)
                                     for (int r = 0; r < NTH; ++r) acc[r] += cmb_w[pc * NT + r0 + r] * v[r];
                                 }
                             }
+                            }
+                            // row rr = node_local * G + hl: walk (node, hl) incrementally (no division)
+                            int node = node0 + r0 / G, hl = r0 % G;
 #pragma unroll
                             for (int r = 0; r < NTH; ++r) {
                                 const int rr = r0 + r;
-                                const int node = node0 + rr / G, hl = rr % G;
                                 if (rr < rc && node < n) {
                                     p.out[(((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim + d] =
                                         __float2bfloat16_rn(__fdividef(acc[r], misc->run_l[rr]));
                                 }
+                                if (++hl == G) {
+                                    hl = 0;
+                                    ++node;
+                                }
                             }
+                            SPI_TRACE2(5);
                         }
                     }
                     named_bar_sync(1, kSoft);  // stats read by everyone before the next reset

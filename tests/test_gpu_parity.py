@@ -108,7 +108,15 @@ def test_attention_score_spikes(Hq, Hkv, Nmax, spike):
             ai.k_cache[0, b, :, j] = (ai.k_cache[0, b, :, j].float() * f).to(torch.bfloat16)
     out, _ = _gpu_attention(tb, ai, Hq, Hkv)
     ref = _oracle_attention(ai, tb)
-    _check_rows(out, ref, tb)
+    # near one-hot rows: |out| reaches |v| ~ 4, where one bf16 rounding of the output alone is up
+    # to 2^-7 = 0.0078; the 1e-2 absolute bar assumes |out| <~ 1, so it is
+    # applied relative to max(1, |ref|) here
+    n = tb.n_nodes.cpu().numpy()
+    for b in range(B):
+        g = out[b, :n[b]].float().cpu().numpy()
+        r = ref[b, :n[b]]
+        e = np.abs(g - r)
+        assert np.all(e <= MAX_ABS * np.maximum(1.0, np.abs(r))) and e.mean() <= MEAN_ABS, (b, e.max(), e.mean())
 
 
 @pytest.mark.parametrize("peaky", [False, True])

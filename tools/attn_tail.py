@@ -1,0 +1,53 @@
+"""Per-CTA exit times of one tree-attention launch (development tool): which CTAs form the tail.
+    python tools/attn_tail.py [--config C2] [--batch 1]"""
+import argparse, os, sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np
+import torch
+import paper_conf_asplos_miaoozcwzwzyssc24_b200 as spi
+import workloads as W
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--config", default="C2")
+ap.add_argument("--batch", type=int, default=1)
+ap.add_argument("--prefix", type=int, default=None)
+a = ap.parse_args()
+cfg = W.CONFIGS[a.config]
+dev = torch.device("cuda:0")
+P = a.prefix or cfg.prefix
+p, d = cfg.tree
+tb = W.make_tree_batch([(p, d)] * a.batch, [P] * a.batch, device=dev, max_depth=cfg.max_depth)
+smax = P + tb.max_nodes
+ai = W.make_attention_inputs(tb, 1, cfg.num_q_heads, cfg.num_kv_heads, smax, seed=1, device=dev)
+shape = spi.make_shape(a.batch, tb.max_nodes, cfg.num_q_heads, cfg.num_kv_heads, smax, max_depth=cfg.max_depth)
+st = spi.TreeState.create(shape, tb.parent, tb.depth, tb.prefix_len, tb.n_nodes)
+st.prepare()
+out = torch.empty_like(ai.q[0])
+for _ in range(3):
+    st.attention(ai.q[0], ai.k_cache[0], ai.v_cache[0], out)
+torch.cuda.synchronize()
+tr = torch.zeros(8 * 64 * 12 + 4 * 1024, dtype=torch.int64, device=dev)
+spi.specinfer_debug_set_trace(tr)
+torch.cuda.synchronize()
+st.attention(ai.q[0], ai.k_cache[0], ai.v_cache[0], out)
+torch.cuda.synchronize()
+spi.specinfer_debug_set_trace(None)
+kt = tr.cpu().numpy().astype(np.int64)[8 * 64 * 12:].reshape(-1, 4)[:148]
+t0 = kt[:, 0].min()
+ex = (kt[:, 1] - t0) / 1e3
+fk = np.where(kt[:, 2] > 0, (kt[:, 2] - t0) / 1e3, -1)
+order = np.argsort(ex)
+print("exit us percentiles 0/25/50/75/90/100:", np.percentile(ex, [0, 25, 50, 75, 90, 100]).round(2))
+print("latest 12 CTAs (cta, entry, firstK, exit):")
+for c in order[-12:]:
+    print(f"  {c:4d} {(kt[c,0]-t0)/1e3:7.2f} {fk[c]:7.2f} {ex[c]:7.2f}")
+print("earliest 5:", [(int(c), round(float(ex[c]), 2)) for c in order[:5]])
+t = tr.cpu().numpy().astype(np.int64)[:8 * 64 * 12].reshape(8, 64, 12)
+for c in range(8):
+    x = t[c]
+    nv = int((x[:, 0] > 0).sum())
+    base = x[0, 0]
+    print(f"CTA {c} exit {ex[c]:.2f} us, raw per-tile events (cycles rel. to its first K issue; -1 none): "
+          "K-iss V-iss S-mma PV-mma 4..11")
+    for i in range(min(nv + 1, 8)):
+        print(f"  {i:3d} " + " ".join(f"{(v - base) if v else -1:7d}" for v in x[i, :12]))
