@@ -624,11 +624,30 @@ __global__ void __launch_bounds__(NT == 64 ? 352 : 224, 1)
                                 }
                                 named_bar_sync(1, kSoft);
                                 SPI_TRACE2(3);
-                                for (int pc = 0; pc < npcs; ++pc) {
-                                    const float *po2 = so + (size_t)pc * NT * kHeadDim + d;
+                                // rows in groups of 8 (rolled outer loops): this code is cold in the
+                                // instruction cache once per launch, so it is kept small
+                                int node = node0 + r0 / G, hl = r0 % G;
+#pragma unroll 1
+                                for (int r8 = 0; r8 < NTH; r8 += 8) {
+                                    float a8[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+#pragma unroll 1
+                                    for (int pc = 0; pc < npcs; ++pc) {
+                                        const float *po2 = so + ((size_t)pc * NT + r0 + r8) * kHeadDim + d;
+                                        const float *wv = cmb_w + pc * NT + r0 + r8;
 #pragma unroll
-                                    for (int r = 0; r < NTH; ++r)
-                                        acc[r] += cmb_w[pc * NT + r0 + r] * po2[(size_t)(r0 + r) * kHeadDim];
+                                        for (int i = 0; i < 8; ++i) a8[i] += wv[i] * po2[(size_t)i * kHeadDim];
+                                    }
+#pragma unroll
+                                    for (int i = 0; i < 8; ++i) {
+                                        const int rr = r0 + r8 + i;
+                                        if (rr < rc && node < n)
+                                            p.out[(((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim + d] =
+                                                __float2bfloat16_rn(__fdividef(a8[i], misc->run_l[rr]));
+                                        if (++hl == G) {
+                                            hl = 0;
+                                            ++node;
+                                        }
+                                    }
                                 }
                                 SPI_TRACE2(4);
                             } else {
@@ -702,10 +721,10 @@ __global__ void __launch_bounds__(NT == 64 ? 352 : 224, 1)
                                 }
                             }
                             }
-                            // row rr = node_local * G + hl: walk (node, hl) incrementally (no division)
+                            // fallback: row rr = node_local * G + hl, walked incrementally (no division)
                             int node = node0 + r0 / G, hl = r0 % G;
 #pragma unroll
-                            for (int r = 0; r < NTH; ++r) {
+                            for (int r = 0; r < NTH && npcs <= 0; ++r) {
                                 const int rr = r0 + r;
                                 if (rr < rc && node < n) {
                                     p.out[(((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim + d] =
