@@ -34,6 +34,9 @@ template <int NT>
 struct SmemPlan {
     static constexpr int kQBuf = 2 * NT * 128;         // one Q buffer: 2 halves x NT rows x 128 B
     static constexpr int kPBuf = kKeyTile * NT * 2;    // one P^T buffer: 128 keys x NT bf16
+    // P^T buffers: two (softmax(t) overlaps PV(t-1)) except at NT = 64, where the second 16 KB
+    // would cost a K/V ring slot (measured: width-5 C2 tree 1% slower with two)
+    static constexpr int kNP = NT == 64 ? 1 : 2;
     static constexpr uint32_t kPSwizzle = NT == 64 ? kSw128 : (NT == 32 ? kSw64 : kSw32);
     static constexpr uint32_t kPMask = NT == 64 ? 7u : (NT == 32 ? 3u : 1u);
     static constexpr int kTmemCols = (3 * NT <= 32) ? 32 : (3 * NT <= 64 ? 64 : (3 * NT <= 128 ? 128 : 256));
@@ -44,7 +47,7 @@ struct SmemMisc {
     uint64_t v_full[kMaxSlots], v_empty[kMaxSlots];
     uint64_t q_full[2], q_empty[2];
     uint64_t s_full[2], s_empty[2];
-    uint64_t p_full, p_empty;  // single P^T buffer: written by softmax(t) after PV(t-1) read it
+    uint64_t p_full[2], p_empty[2];  // P^T buffers: tile lt uses buffer lt % kNP, free once PV(lt-kNP) read it
     uint64_t cmb_bar;          // bulk staging of the split pieces (at most one merge per CTA uses it)
     uint64_t seg_full[kSegRing];
     SegDesc seg[kSegRing];
@@ -84,7 +87,7 @@ __global__ void __launch_bounds__(NT == 64 ? 352 : 224, 1)
     uint8_t *s_v = s_k + (size_t)NK * kSlotBytes;
     uint8_t *s_q = s_v + (size_t)NV * kSlotBytes;
     uint8_t *s_p = s_q + 2 * Plan::kQBuf;
-    SmemMisc *misc = reinterpret_cast<SmemMisc *>(s_p + Plan::kPBuf);
+    SmemMisc *misc = reinterpret_cast<SmemMisc *>(s_p + Plan::kNP * Plan::kPBuf);
 
     const int warp = threadIdx.x >> 5;
     const int lane = threadIdx.x & 31;
@@ -106,8 +109,10 @@ __global__ void __launch_bounds__(NT == 64 ? 352 : 224, 1)
             mbar_init(&misc->s_full[i], 1);
             mbar_init(&misc->s_empty[i], 4 * kSplit);
         }
-        mbar_init(&misc->p_full, 4 * kSplit);
-        mbar_init(&misc->p_empty, 1);
+        for (int i = 0; i < Plan::kNP; ++i) {
+            mbar_init(&misc->p_full[i], 4 * kSplit);
+            mbar_init(&misc->p_empty[i], 1);
+        }
         mbar_init(&misc->cmb_bar, 1);
         for (int i = 0; i < kSegRing; ++i) mbar_init(&misc->seg_full[i], 1);
         fence_barrier_init();
@@ -281,7 +286,7 @@ __global__ void __launch_bounds__(NT == 64 ? 352 : 224, 1)
                 mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
                 const SegDesc d = misc->seg[ls % kSegRing];
                 for (int t = d.begin; t < d.end; ++t, ++lt) {
-                    mbar_wait(&misc->p_full, lt & 1);
+                    mbar_wait(&misc->p_full[lt % Plan::kNP], (lt / Plan::kNP) & 1);
                     const int slot = lt % NV;
                     mbar_wait(&misc->v_full[slot], (lt / NV) & 1);
                     tc_fence_after();
@@ -291,11 +296,11 @@ __global__ void __launch_bounds__(NT == 64 ? 352 : 224, 1)
 #pragma unroll
                     for (int kk = 0; kk < kKeyTile / 16; ++kk) {
                         const uint64_t adesc = make_smem_desc(vbase + kk * 16 * 128, kHalfBytes, 1024, kSw128);
-                        const uint64_t bdesc = make_smem_desc(p_addr + kk * 16 * (NT * 2), Plan::kPBuf,
+                        const uint64_t bdesc = make_smem_desc(p_addr + (lt % Plan::kNP) * Plan::kPBuf + kk * 16 * (NT * 2), Plan::kPBuf,
                                                               8 * NT * 2, Plan::kPSwizzle);
                         if (!(p.debug_flags & 2)) umma_bf16_ss(tm_O, adesc, bdesc, idesc_o, (first && kk == 0) ? 0u : 1u);
                     }
-                    umma_commit(&misc->p_empty);
+                    umma_commit(&misc->p_empty[lt % Plan::kNP]);
                     umma_commit(&misc->v_empty[slot]);
                 }
                 ++ls;
@@ -422,7 +427,7 @@ __global__ void __launch_bounds__(NT == 64 ? 352 : 224, 1)
                     for (int r = 0; r < NTH; ++r) lsum[r] *= misc->alpha[r0 + r];
                     if (t != sd.begin) {
                         // O^T columns (query rows) scaled by alpha: wait for PV of tile lt-1
-                        mbar_wait(&misc->p_empty, (lt - 1) & 1);
+                        mbar_wait(&misc->p_empty[(lt - 1) % Plan::kNP], ((lt - 1) / Plan::kNP) & 1);
                         tc_fence_after();
                         uint32_t r16[16];
 #pragma unroll
@@ -456,9 +461,10 @@ __global__ void __launch_bounds__(NT == 64 ? 352 : 224, 1)
                     lsum[2 * i + 1] += __uint_as_float(pk[i] & 0xFFFF0000u);
                 }
                 // ---- P^T row (this key) into smem as bf16, MN-major + swizzle ----
-                if (lt >= 1) mbar_wait(&misc->p_empty, (lt - 1) & 1);  // PV(t-1) has read P^T
+                if (lt >= Plan::kNP)  // PV(t - kNP) has read this buffer
+                    mbar_wait(&misc->p_empty[lt % Plan::kNP], ((lt - Plan::kNP) / Plan::kNP) & 1);
                 {
-                    uint8_t *pb = s_p;
+                    uint8_t *pb = s_p + (lt % Plan::kNP) * Plan::kPBuf;
 #pragma unroll
                     for (int c8 = 0; c8 < NTH / 8; ++c8) {
                         const uint32_t o = (uint32_t)kt * (NT * 2) + (half * (NTH / 8) + c8) * 16;
@@ -470,7 +476,7 @@ __global__ void __launch_bounds__(NT == 64 ? 352 : 224, 1)
                 fence_proxy_async_smem();
                 tc_fence_before();
                 __syncwarp();
-                if (lane == 0) mbar_arrive(&misc->p_full);
+                if (lane == 0) mbar_arrive(&misc->p_full[lt % Plan::kNP]);
                 if (st == 0) SPI_TRACE(5);
 
                 if (t == sd.end - 1) {
@@ -483,7 +489,7 @@ __global__ void __launch_bounds__(NT == 64 ? 352 : 224, 1)
                         const int row = r0 + blk * 32 + (lane & (W - 1));
                         if (lane < W) misc->l_part[qd][row] = lsum[blk * 32];
                     }
-                    mbar_wait(&misc->p_empty, lt & 1);  // last PV done
+                    mbar_wait(&misc->p_empty[lt % Plan::kNP], (lt / Plan::kNP) & 1);  // last PV done (and every earlier one)
                     tc_fence_after();
                     if (st == 0) SPI_TRACE(6);
                     float o[NTH];
@@ -760,7 +766,7 @@ template <int NT>
 static size_t attn_smem_bytes(int num_slots) {
     using Plan = SmemPlan<NT>;
     static_assert(3 * kCombineBatch * NT * 4 <= Plan::kPBuf, "combine staging must fit the P buffer");
-    return 1024 + (size_t)num_slots * kSlotBytes + 2 * Plan::kQBuf + Plan::kPBuf + sizeof(SmemMisc);
+    return 1024 + (size_t)num_slots * kSlotBytes + 2 * Plan::kQBuf + Plan::kNP * Plan::kPBuf + sizeof(SmemMisc);
 }
 
 template <int NT>

@@ -1,0 +1,9 @@
+#!/bin/bash
+timeout 600 python -m pytest tests -x -q -m gpu > gpurun_out/pytest_gpu.log 2>&1; echo pytest=$?; tail -1 gpurun_out/pytest_gpu.log
+for rep in 1 2; do for lib in abtest/lib_*.so; do
+  echo "== $lib"
+  for b in 16; do timeout 120 python tools/attn_probe.py --config C2 --batch $b --layers 4 --iters 40 --lib $lib; done
+  timeout 120 python tools/attn_probe.py --config C2 --expansion 1,1,5,1,1,1,1,1 --layers 4 --iters 20 --lib $lib
+
+  timeout 120 python tools/attn_sweep.py --ns 8,16,64 --batch 16 --prefix 2048 --iters 10 --lib $lib
+done; done
