@@ -67,16 +67,16 @@ struct SmemMisc {
 };
 
 template <int NT>
-__global__ void __launch_bounds__(NT == 64 ? 352 : 224, 1)
+__global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
     tree_attn_kernel(const __grid_constant__ CUtensorMap tm_q, const __grid_constant__ CUtensorMap tm_k,
                      const __grid_constant__ CUtensorMap tm_v, const __grid_constant__ CUtensorMap tm_k16,
                      const __grid_constant__ CUtensorMap tm_v16, const __grid_constant__ CUtensorMap tm_k4,
                      const __grid_constant__ CUtensorMap tm_v4, const __grid_constant__ CUtensorMap tm_k1,
                      const __grid_constant__ CUtensorMap tm_v1, const AttnParams p) {
     using Plan = SmemPlan<NT>;
-    // NT = 64: 8 softmax warps, two per TMEM lane quarter, each owning half of the query rows
+    // NT >= 32: 8 softmax warps, two per TMEM lane quarter, each owning half of the query rows
     // (columns of S^T) of its key: half the registers and two warps per SMSP to hide latency
-    constexpr int kSplit = NT == 64 ? 2 : 1;
+    constexpr int kSplit = NT >= 32 ? 2 : 1;
     constexpr int NTH = NT / kSplit;  // query rows per softmax thread
     constexpr int kSoft = 128 * kSplit;
     extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -799,7 +799,7 @@ static cudaError_t launch_nt(const AttnParams &prm0, const void *q, const void *
     // this grid overlaps the tail of the previous kernel on the stream
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(num_sms);
-    cfg.blockDim = dim3(NT == 64 ? 352 : 224);
+    cfg.blockDim = dim3(NT >= 32 ? 352 : 224);
     cfg.dynamicSmemBytes = smem;
     cfg.stream = stream;
     cudaLaunchAttribute attr[1];
