@@ -581,7 +581,7 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
                             float *so = reinterpret_cast<float *>(s_k);
                             if (st == 0) {
                                 int npcs = -1;
-                                if (sd.end == t1) {  // no tile of this CTA follows: rings idle
+                                if (sd.end == t1 && !(p.debug_flags & 32)) {  // no tile follows: rings idle (32: test the fallback)
                                     npcs = 0;
                                     const int cf = cta_of_tile(sd.ib, T, NC), cl2 = cta_of_tile(sd.ie - 1, T, NC);
                                     for (int cc = cf; cc <= cl2 && npcs <= kCombineBatch; ++cc) {

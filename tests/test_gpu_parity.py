@@ -119,6 +119,30 @@ def test_attention_score_spikes(Hq, Hkv, Nmax, spike):
         assert np.all(e <= MAX_ABS * np.maximum(1.0, np.abs(r))) and e.mean() <= MEAN_ABS, (b, e.max(), e.mean())
 
 
+@pytest.mark.parametrize("force_fallback", [False, True])
+def test_attention_split_merge_paths(force_fallback, monkeypatch):
+    """Stream-K split items (units cut by CTA boundaries): the merge through the bulk-staged path
+    and, forced with debug flag 32, the batched-load fallback path give the oracle's result."""
+    import os
+    if force_fallback:
+        monkeypatch.setenv("SPECINFER_DEBUG_FLAGS", "32")
+    spi.specinfer_debug_set_trace(None)  # (re-reads SPECINFER_DEBUG_FLAGS)
+    try:
+        # 24 units x ~24 tiles over 148 CTAs: stream-K (a unit exceeds an even share by > 16 tiles),
+        # every unit cut into ~6 pieces
+        B, Hq, Hkv, P = 3, 8, 8, 3000
+        parent, depth = W.expansion_tree((1, 1, 3, 1, 1, 1, 1, 1))
+        tb = W.make_tree_batch([(parent, depth)] * B, list(W.ragged_prefix(P, B)), device=DEV, max_depth=8)
+        smax = P + tb.max_nodes + 3
+        ai = W.make_attention_inputs(tb, 1, Hq, Hkv, smax, seed=77, device=DEV, poison=True)
+        out, _ = _gpu_attention(tb, ai, Hq, Hkv)
+        ref = _oracle_attention(ai, tb)
+        _check_rows(out, ref, tb)
+    finally:
+        monkeypatch.delenv("SPECINFER_DEBUG_FLAGS", raising=False)
+        spi.specinfer_debug_set_trace(None)
+
+
 @pytest.mark.parametrize("peaky", [False, True])
 def test_attention_chain_and_figures(golden, peaky):
     """Fig. 4 tree (L682), a 40-node chain (= causal decoding), root-only trees; peaky q (x4)
