@@ -20,6 +20,7 @@ struct AttnParams {
     float *part_ml;
     __nv_bfloat16 *out;
     int B, Nmax, Hq, Hkv, G, Smax, chunks, npc, n_items, nk_slots, nv_slots;
+    int splitk;  // > 1: split-KV mode (cluster of splitk CTAs per item, DSMEM merge)
     int lanes;  // CTAs per lock-step group (schedule_kernel); 1 = plain stream-K over items
     // paged KV (NEXT-4): page_table[b][t] = page holding keys [128 t, 128 t + 128) of request b;
     // a page is [Hkv][128][128] bf16.  nullptr = contiguous [B][Hkv][Smax][128] caches.

@@ -44,7 +44,9 @@ struct WsLayout {
     int chunks;         // chunks per (b, kv-head) item = ceil(Nmax / npc)
     int n_items;        // B * Hkv * chunks
     int lanes;          // CTAs sharing one KV stream in lock-step (rows kernel: chunks; else 1)
-    int grid;           // attention CTAs: the largest multiple of `lanes` <= the SM count
+    int grid;           // attention CTAs: the largest multiple of `lanes` <= the SM count, or
+                        // n_items * splitk in split-KV mode
+    int splitk;         // > 1: split-KV mode, each item's tiles split over a cluster of splitk CTAs
     int max_ctas;
 };
 
@@ -71,7 +73,18 @@ inline WsLayout ws_layout(const specinfer_shape_t &s, int num_sms) {
     w.chunks = (N + w.npc - 1) / w.npc;
     w.n_items = B * s.num_kv_heads * w.chunks;
     w.lanes = (w.nt == kRowsBlock && w.chunks > 1 && 2 * w.chunks <= num_sms) ? w.chunks : 1;
-    w.grid = (num_sms / w.lanes) * w.lanes;
+    // split-KV mode (swapped kernel, few items: batch 1-4 decoding): every item gets a thread-block
+    // cluster of splitk CTAs, each streaming a contiguous part of its tiles, merged through DSMEM;
+    // otherwise the persistent stream-K / one-unit-per-CTA schedule
+    w.splitk = 1;
+    // (only when an item can span enough 128-key tiles for the split to pay for the cluster merge:
+    // the schedule keeps items shorter than 12 tiles whole on rank 0)
+    if (w.nt != kRowsBlock && w.lanes == 1 && (s.max_seq + 127) / 128 >= 12) {
+        int k = 1;
+        while (k < 8 && (long long)w.n_items * k * 2 <= num_sms) k *= 2;
+        w.splitk = k;
+    }
+    w.grid = w.splitk > 1 ? w.n_items * w.splitk : (num_sms / w.lanes) * w.lanes;
     w.max_ctas = num_sms * kMaxCtasPerSm;
     size_t o = 0;
     auto take = [&](size_t bytes) { size_t r = o; o = align256(o + bytes); return r; };

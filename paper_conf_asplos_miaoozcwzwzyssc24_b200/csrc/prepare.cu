@@ -104,7 +104,8 @@ __global__ void __launch_bounds__(1024) schedule_kernel(
     const int32_t *__restrict__ prefix_len, const int32_t *__restrict__ n_nodes,
     const int32_t *__restrict__ req_ok, int B, int Hkv, int chunks, int npc, int lanes,
     int32_t *__restrict__ item_start, uint32_t *__restrict__ item_cnt, int4 *__restrict__ item_info,
-    int4 *__restrict__ cta_info, int num_ctas, uint32_t *__restrict__ verify_cnt, int32_t *__restrict__ status) {
+    int4 *__restrict__ cta_info, int num_ctas, int splitk, uint32_t *__restrict__ verify_cnt,
+    int32_t *__restrict__ status) {
     const int n_items = B * Hkv * chunks;
     const int n_units = n_items / lanes;
     const int per = (n_units + blockDim.x - 1) / blockDim.x;
@@ -187,6 +188,27 @@ __global__ void __launch_bounds__(1024) schedule_kernel(
     const bool one_per_cta = n_units <= NCv && (long long)s_max_tiles * NCv <= T + (long long)kNoSplitSlack * NCv;
     for (int c = threadIdx.x; c < num_ctas; c += blockDim.x) {
         const int vc = c / lanes, cl = c % lanes;
+        if (splitk > 1) {  // split-KV mode (lanes == 1): CTA c = part c % splitk of item c / splitk
+            const int u = c / splitk, r = c % splitk;
+            int t0 = (int)T, t1 = (int)T;
+            if (u < n_units) {
+                // short items stay whole on rank 0 (written directly, no merge): the cluster merge
+                // costs about as much as streaming kMinSplitTiles tiles on one CTA
+                constexpr int kMinSplitTiles = 12;
+                const int s0 = item_start[u], len = item_start[u + 1] - s0;
+                if (len < kMinSplitTiles) {
+                    t0 = r == 0 ? s0 : s0 + len;
+                    t1 = s0 + len;
+                } else {
+                    t0 = s0 + (int)((long long)r * len / splitk);
+                    t1 = s0 + (int)((long long)(r + 1) * len / splitk);
+                }
+            }
+            const int x0 = u < n_units ? u : n_items;
+            cta_info[2 * c] = make_int4(t0, t1, x0, (int)T);
+            cta_info[2 * c + 1] = x0 < n_items ? item_info[x0] : make_int4(0, 0, 0, 0);
+            continue;
+        }
         if (one_per_cta) {
             const int t0 = vc < n_units ? item_start[vc] : (int)T;
             const int t1 = vc < n_units ? item_start[vc + 1] : (int)T;
@@ -226,7 +248,7 @@ cudaError_t launch_tree_prepare(const specinfer_shape_t &s, const WsLayout &w,
         prefix_len, n_nodes, reinterpret_cast<int32_t *>(ws + w.req_ok), s.batch,
         s.num_kv_heads, w.chunks, w.npc, w.lanes, reinterpret_cast<int32_t *>(ws + w.item_start),
         reinterpret_cast<uint32_t *>(ws + w.item_cnt), reinterpret_cast<int4 *>(ws + w.item_info),
-        reinterpret_cast<int4 *>(ws + w.cta_info), num_ctas, reinterpret_cast<uint32_t *>(ws + w.verify_cnt), status);
+        reinterpret_cast<int4 *>(ws + w.cta_info), num_ctas, w.splitk, reinterpret_cast<uint32_t *>(ws + w.verify_cnt), status);
     return cudaGetLastError();
 }
 

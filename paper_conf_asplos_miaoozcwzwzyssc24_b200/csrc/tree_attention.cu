@@ -28,6 +28,8 @@
 //    MMA issuer; warps 2-5: softmax / epilogue / split combine.
 #include "attn_shared.cuh"
 
+#include <cooperative_groups.h>
+
 namespace specinfer {
 
 template <int NT>
@@ -513,6 +515,8 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
                     }
                     named_bar_sync(1, kSoft);
                     if (st == 0) SPI_TRACE(9);
+                    // (split-KV mode: a part of a split item stages a partial, the cluster's rank 0
+                    // merges; an item left whole on rank 0 is written here directly)
                     const bool full = (sd.begin == sd.ib) && (sd.end == sd.ie);
                     const int rc = G * p.npc;
                     if (full) {
@@ -537,6 +541,18 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
                         }
                         if (st == 0) SPI_TRACE(8);
                     } else {
+                      if (p.splitk > 1) {
+                        // split-KV mode: stage this part's (O, m, l) in the idle K ring (its only
+                        // segment is done); the cluster merges them at the end of the kernel
+                        float *so = reinterpret_cast<float *>(s_k);
+#pragma unroll
+                        for (int r = 0; r < NTH; ++r) so[(size_t)(r0 + r) * kHeadDim + d] = o[r];
+                        if (st < NT) {
+                            const float mt = misc->m_thr[st];
+                            so[NT * kHeadDim + st] = mt == -INFINITY ? -INFINITY : mt - kRescaleThreshold;
+                            so[NT * kHeadDim + NT + st] = misc->run_l[st];
+                        }
+                      } else {
                         const int slot = (sd.begin == t0) ? 0 : 1;
                         float *po = p.part_o + (((size_t)blockIdx.x * 2 + slot) * NT) * kHeadDim;
 #pragma unroll
@@ -743,6 +759,7 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
                             }
                             SPI_TRACE2(5);
                         }
+                      }
                     }
                     named_bar_sync(1, kSoft);  // stats read by everyone before the next reset
                     if (st == 0) SPI_TRACE(7);
@@ -755,6 +772,68 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
     if (warp >= 3) bulk_wait_all();  // output bulk stores complete before smem goes away
     tc_fence_before();
     __syncthreads();
+    if (p.splitk > 1) {
+        // ======== split-KV mode: merge the cluster's partials (DSMEM), rank 0 writes the rows ========
+        namespace cg = cooperative_groups;
+        cg::cluster_group cluster = cg::this_cluster();
+        float *so = reinterpret_cast<float *>(s_k);
+        if (ntiles <= 0 && threadIdx.x < NT) {  // no tiles for this part: it saw no key
+            so[NT * kHeadDim + threadIdx.x] = -INFINITY;
+            so[NT * kHeadDim + NT + threadIdx.x] = 0.f;
+        }
+        cluster.sync();  // every part staged (release / acquire at cluster scope)
+        const int K = p.splitk;
+        const int x = blockIdx.x / K;
+        const int4 info = __ldg(p.item_info + x);
+        const bool whole = t0 == info.x && t1 == info.y;  // rank 0 streamed (and wrote) the whole item
+        if (cluster.block_rank() == 0 && warp >= 3 && !whole && info.y > info.x) {
+            const int st = threadIdx.x - 96;
+            const int r0 = (st >> 7) * NTH;
+            const int d = (warp & 3) * 32 + lane;
+            const int n = info.w, G = p.G, rc = G * p.npc;
+            const int c = x % p.chunks, g = (x / p.chunks) % p.Hkv, b = x / (p.chunks * p.Hkv);
+            const int node0 = c * p.npc;
+            float *cmb_w = reinterpret_cast<float *>(s_p);  // [K][NT] weights
+            if (st < NT) {
+                float M = -INFINITY;
+                for (int k = 0; k < K; ++k) M = fmaxf(M, cluster.map_shared_rank(so, k)[NT * kHeadDim + st]);
+                float L = 0.f;
+                for (int k = 0; k < K; ++k) {
+                    const float *rk = cluster.map_shared_rank(so, k);
+                    const float mk = rk[NT * kHeadDim + st];
+                    const float w = (mk == -INFINITY) ? 0.f : ex2(mk - M);
+                    cmb_w[k * NT + st] = w;
+                    L += w * rk[NT * kHeadDim + NT + st];
+                }
+                misc->run_l[st] = L;
+            }
+            named_bar_sync(1, kSoft);
+            float acc[NTH];
+#pragma unroll
+            for (int r = 0; r < NTH; ++r) acc[r] = 0.f;
+            for (int k = 0; k < K; ++k) {
+                const float *rk = cluster.map_shared_rank(so, k) + d;
+#pragma unroll
+                for (int r = 0; r < NTH; ++r) {
+                    const float w = cmb_w[k * NT + r0 + r];
+                    if (w != 0.f) acc[r] += w * rk[(size_t)(r0 + r) * kHeadDim];
+                }
+            }
+            int node = node0 + r0 / G, hl = r0 % G;
+#pragma unroll
+            for (int r = 0; r < NTH; ++r) {
+                const int rr = r0 + r;
+                if (rr < rc && node < n && n > 0)
+                    p.out[(((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim + d] =
+                        __float2bfloat16_rn(__fdividef(acc[r], misc->run_l[rr]));
+                if (++hl == G) {
+                    hl = 0;
+                    ++node;
+                }
+            }
+        }
+        cluster.sync();  // rank 0 has read every part before any CTA's shared memory goes away
+    }
     if (warp == 1) {
         tc_fence_after();
         tmem_dealloc<Plan::kTmemCols>(tmem);
@@ -798,15 +877,22 @@ static cudaError_t launch_nt(const AttnParams &prm0, const void *q, const void *
     // programmatic dependent launch: the prologue (barrier init, TMEM alloc, smem zeroing) of
     // this grid overlaps the tail of the previous kernel on the stream
     cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3(num_sms);
+    cfg.gridDim = dim3(num_sms);  // (the caller's grid: w.grid)
     cfg.blockDim = dim3(NT >= 32 ? 352 : 224);
     cfg.dynamicSmemBytes = smem;
     cfg.stream = stream;
-    cudaLaunchAttribute attr[1];
+    cudaLaunchAttribute attr[2];
     attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
     attr[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
+    if (prm.splitk > 1) {  // split-KV mode: one cluster of splitk CTAs per item
+        attr[1].id = cudaLaunchAttributeClusterDimension;
+        attr[1].val.clusterDim.x = prm.splitk;
+        attr[1].val.clusterDim.y = 1;
+        attr[1].val.clusterDim.z = 1;
+        cfg.numAttrs = 2;
+    }
     return cudaLaunchKernelEx(&cfg, tree_attn_kernel<NT>, tq, tk, tv, tk16, tv16, tk4, tv4, tk1, tv1, prm);
 }
 
@@ -850,7 +936,8 @@ cudaError_t launch_tree_attention(const specinfer_shape_t &s, const WsLayout &w,
     prm.scale_log2 = sm_scale * 1.4426950408889634f;
     prm.trace = g_attn_trace;
     prm.debug_flags = g_attn_debug_flags;
-    const int grid = num_sms;  // persistent: one CTA per SM
+    prm.splitk = w.splitk;
+    const int grid = w.grid;  // persistent one CTA per SM, or n_items x splitk in split-KV mode
     switch (w.nt) {
         case 16: return launch_nt<16>(prm, q, k, v, grid, max_smem, stream);
         case 32: return launch_nt<32>(prm, q, k, v, grid, max_smem, stream);

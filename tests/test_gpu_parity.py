@@ -119,6 +119,26 @@ def test_attention_score_spikes(Hq, Hkv, Nmax, spike):
         assert np.all(e <= MAX_ABS * np.maximum(1.0, np.abs(r))) and e.mean() <= MEAN_ABS, (b, e.max(), e.mean())
 
 
+@pytest.mark.parametrize("Hq,Hkv,pls", [(4, 4, [3000]), (8, 2, [3000, 100]), (16, 8, [1700, 2900, 40])])
+def test_attention_split_kv_clusters(Hq, Hkv, pls):
+    """Split-KV mode (few items: each item's tiles split over a thread-block cluster of up to 8 CTAs,
+    merged through DSMEM by rank 0; items shorter than 12 tiles stay whole on rank 0), ragged prefixes
+    and trees, NaN-poisoned unused cache slots."""
+    rng = np.random.default_rng(sum(pls) + Hq)
+    Nmax = 24
+    B = len(pls)
+    trees = [W.random_tree(int(rng.integers(1, Nmax + 1)), 8, 4, rng) for _ in range(B)]
+    tb = W.make_tree_batch(trees, pls, max_nodes=Nmax, max_depth=8, device=DEV)
+    smax = max(pls) + Nmax + 5
+    ai = W.make_attention_inputs(tb, 1, Hq, Hkv, smax, seed=len(pls) + Hq, device=DEV, poison=True)
+    out, _ = _gpu_attention(tb, ai, Hq, Hkv)
+    ref = _oracle_attention(ai, tb)
+    _check_rows(out, ref, tb)
+    n = tb.n_nodes.cpu().numpy()
+    for b in range(B):
+        assert torch.isnan(out[b, n[b]:].float()).all()
+
+
 @pytest.mark.parametrize("force_fallback", [False, True])
 def test_attention_split_merge_paths(force_fallback, monkeypatch):
     """Stream-K split items (units cut by CTA boundaries): the merge through the bulk-staged path
