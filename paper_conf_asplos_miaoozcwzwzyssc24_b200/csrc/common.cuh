@@ -81,7 +81,9 @@ inline WsLayout ws_layout(const specinfer_shape_t &s, int num_sms) {
     // the schedule keeps items shorter than 12 tiles whole on rank 0)
     if (w.nt != kRowsBlock && w.lanes == 1 && (s.max_seq + 127) / 128 >= 12) {
         int k = 1;
-        while (k < 8 && (long long)w.n_items * k * 2 <= num_sms) k *= 2;
+        // rank 0 gathers the k partials ([nt][128] + 2 [nt] floats each) in its K/V rings (>= 160 KB)
+        const int kmax = w.nt == 64 ? 4 : 8;
+        while (k < kmax && (long long)w.n_items * k * 2 <= num_sms) k *= 2;
         w.splitk = k;
     }
     w.grid = w.splitk > 1 ? w.n_items * w.splitk : (num_sms / w.lanes) * w.lanes;

@@ -781,12 +781,23 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
             so[NT * kHeadDim + threadIdx.x] = -INFINITY;
             so[NT * kHeadDim + NT + threadIdx.x] = 0.f;
         }
-        cluster.sync();  // every part staged (release / acquire at cluster scope)
+        // partial k (O rows [NT][128] then m [NT], l [NT]) lives at kPart floats into rank 0's K/V rings
+        constexpr int kPart = NT * kHeadDim + 2 * NT;
+        cluster.sync();  // every rank's tiles done: rank 0's rings are idle, every part staged locally
+        if (threadIdx.x == 0) SPI_TRACE_K(3);
         const int K = p.splitk;
+        const int rank = (int)cluster.block_rank();
+        if (rank != 0) {
+            // push this part into rank 0's shared memory (fire-and-forget DSMEM stores, 16 B each)
+            uint4 *dst = reinterpret_cast<uint4 *>(cluster.map_shared_rank(so, 0) + (size_t)rank * kPart);
+            const uint4 *src = reinterpret_cast<const uint4 *>(so);
+            for (int i = threadIdx.x; i < kPart / 4; i += blockDim.x) dst[i] = src[i];
+        }
+        cluster.sync();  // every part is in rank 0's shared memory; ranks != 0 may exit
         const int x = blockIdx.x / K;
         const int4 info = __ldg(p.item_info + x);
         const bool whole = t0 == info.x && t1 == info.y;  // rank 0 streamed (and wrote) the whole item
-        if (cluster.block_rank() == 0 && warp >= 3 && !whole && info.y > info.x) {
+        if (rank == 0 && warp >= 3 && !whole && info.y > info.x) {
             const int st = threadIdx.x - 96;
             const int r0 = (st >> 7) * NTH;
             const int d = (warp & 3) * 32 + lane;
@@ -796,10 +807,10 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
             float *cmb_w = reinterpret_cast<float *>(s_p);  // [K][NT] weights
             if (st < NT) {
                 float M = -INFINITY;
-                for (int k = 0; k < K; ++k) M = fmaxf(M, cluster.map_shared_rank(so, k)[NT * kHeadDim + st]);
+                for (int k = 0; k < K; ++k) M = fmaxf(M, so[(size_t)k * kPart + NT * kHeadDim + st]);
                 float L = 0.f;
                 for (int k = 0; k < K; ++k) {
-                    const float *rk = cluster.map_shared_rank(so, k);
+                    const float *rk = so + (size_t)k * kPart;
                     const float mk = rk[NT * kHeadDim + st];
                     const float w = (mk == -INFINITY) ? 0.f : ex2(mk - M);
                     cmb_w[k * NT + st] = w;
@@ -812,7 +823,7 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
 #pragma unroll
             for (int r = 0; r < NTH; ++r) acc[r] = 0.f;
             for (int k = 0; k < K; ++k) {
-                const float *rk = cluster.map_shared_rank(so, k) + d;
+                const float *rk = so + (size_t)k * kPart + d;
 #pragma unroll
                 for (int r = 0; r < NTH; ++r) {
                     const float w = cmb_w[k * NT + r0 + r];
@@ -832,7 +843,6 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
                 }
             }
         }
-        cluster.sync();  // rank 0 has read every part before any CTA's shared memory goes away
     }
     if (warp == 1) {
         tc_fence_after();
@@ -862,6 +872,9 @@ static cudaError_t launch_nt(const AttnParams &prm0, const void *q, const void *
         return cudaErrorInvalidValue;
     int ns = 2 * kMaxSlots;
     while (ns > 2 && attn_smem_bytes<NT>(ns) > max_smem) --ns;
+    // split-KV mode: rank 0 gathers every part's partial in its (contiguous) K/V rings
+    if (prm0.splitk > 1 && (size_t)prm0.splitk * (NT * kHeadDim + 2 * NT) * 4 > (size_t)ns * kSlotBytes)
+        return cudaErrorInvalidConfiguration;
     // K tiles are released right after S = K Q^T; V tiles are held until PV: give V the extra slot
     ns = min(ns, 6);
     prm.nk_slots = ns / 2;

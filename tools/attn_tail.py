@@ -33,6 +33,7 @@ st.attention(ai.q[0], ai.k_cache[0], ai.v_cache[0], out)
 torch.cuda.synchronize()
 spi.specinfer_debug_set_trace(None)
 kt = tr.cpu().numpy().astype(np.int64)[8 * 64 * 12:].reshape(-1, 4)[:148]
+kt = kt[kt[:, 0] > 0]  # CTAs of this launch (the grid may be smaller than 148)
 t0 = kt[:, 0].min()
 ex = (kt[:, 1] - t0) / 1e3
 fk = np.where(kt[:, 2] > 0, (kt[:, 2] - t0) / 1e3, -1)
@@ -42,6 +43,9 @@ print("latest 12 CTAs (cta, entry, firstK, exit):")
 for c in order[-12:]:
     print(f"  {c:4d} {(kt[c,0]-t0)/1e3:7.2f} {fk[c]:7.2f} {ex[c]:7.2f}")
 print("earliest 5:", [(int(c), round(float(ex[c]), 2)) for c in order[:5]])
+if (kt[:, 3] > 0).any():
+    s3 = (kt[:, 3] - t0) / 1e3
+    print("split-KV: first cluster barrier passed (us) min/median/max:", np.percentile(s3[kt[:, 3] > 0], [0, 50, 100]).round(2))
 t = tr.cpu().numpy().astype(np.int64)[:8 * 64 * 12].reshape(8, 64, 12)
 for c in range(8):
     x = t[c]
