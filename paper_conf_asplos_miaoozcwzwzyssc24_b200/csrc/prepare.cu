@@ -184,8 +184,15 @@ __global__ void __launch_bounds__(1024) schedule_kernel(
     // parallelism it buys (C1: 2 tiles per unit; B = 1..4 at P = 2048: 17).  Otherwise even stream-K slices.
     const long long T = s_total;
     const int NCv = num_ctas / lanes;
-    constexpr int kNoSplitSlack = 16;
-    const bool one_per_cta = n_units <= NCv && (long long)s_max_tiles * NCv <= T + (long long)kNoSplitSlack * NCv;
+#ifndef SPECINFER_NOSPLIT_SLACK
+#define SPECINFER_NOSPLIT_SLACK 8
+#endif
+    constexpr int kNoSplitSlack = SPECINFER_NOSPLIT_SLACK;
+    // whole units per CTA group (contiguous ranges of floor / ceil(n_units / NCv) units) when the
+    // busiest group's upper bound exceeds an even share by at most kNoSplitSlack tiles
+    const int upc = (n_units + NCv - 1) / NCv;
+    const bool one_per_cta = n_units > 0 &&
+        (long long)upc * s_max_tiles * NCv <= T + (long long)kNoSplitSlack * NCv;
     for (int c = threadIdx.x; c < num_ctas; c += blockDim.x) {
         const int vc = c / lanes, cl = c % lanes;
         if (splitk > 1) {  // split-KV mode (lanes == 1): CTA c = part c % splitk of item c / splitk
@@ -210,9 +217,10 @@ __global__ void __launch_bounds__(1024) schedule_kernel(
             continue;
         }
         if (one_per_cta) {
-            const int t0 = vc < n_units ? item_start[vc] : (int)T;
-            const int t1 = vc < n_units ? item_start[vc + 1] : (int)T;
-            const int x0 = vc < n_units ? vc * lanes + cl : n_items;
+            const int u_lo = (int)((long long)vc * n_units / NCv), u_hi = (int)((long long)(vc + 1) * n_units / NCv);
+            const int t0 = item_start[u_lo];
+            const int t1 = item_start[u_hi];
+            const int x0 = u_lo < u_hi ? u_lo * lanes + cl : n_items;
             cta_info[2 * c] = make_int4(t0, t1, x0, (int)T);
             cta_info[2 * c + 1] = x0 < n_items ? item_info[x0] : make_int4(0, 0, 0, 0);
             continue;
