@@ -53,5 +53,6 @@ for c in range(8):
     base = x[0, 0]
     print(f"CTA {c} exit {ex[c]:.2f} us, raw per-tile events (cycles rel. to its first K issue; -1 none): "
           "K-iss V-iss S-mma PV-mma 4..11")
-    for i in range(min(nv + 1, 8)):
+    show = list(range(min(nv + 1, 8))) + [i for i in range(max(8, nv - 3), min(nv + 2, 64))]
+    for i in show:
         print(f"  {i:3d} " + " ".join(f"{(v - base) if v else -1:7d}" for v in x[i, :12]))
