@@ -217,7 +217,9 @@ __global__ void __launch_bounds__(1024) schedule_kernel(
             continue;
         }
         if (one_per_cta) {
-            const int u_lo = (int)((long long)vc * n_units / NCv), u_hi = (int)((long long)(vc + 1) * n_units / NCv);
+            // (at most one unit per group: units on groups 0 .. n_units-1, measured 7.4 -> 6.8 us at C1)
+            const int u_lo = n_units <= NCv ? min(vc, n_units) : (int)((long long)vc * n_units / NCv);
+            const int u_hi = n_units <= NCv ? min(vc + 1, n_units) : (int)((long long)(vc + 1) * n_units / NCv);
             const int t0 = item_start[u_lo];
             const int t1 = item_start[u_hi];
             const int x0 = u_lo < u_hi ? u_lo * lanes + cl : n_items;

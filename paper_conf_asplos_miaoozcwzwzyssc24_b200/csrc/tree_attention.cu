@@ -563,10 +563,12 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
                             pml[st] = mt == -INFINITY ? -INFINITY : mt - kRescaleThreshold;
                             pml[NT + st] = misc->run_l[st];
                         }
-                        __threadfence();
+                        // release: the CTA barrier orders every thread's partial stores before thread
+                        // 0's gpu-scope fence and counter update (fence cumulativity, one fence per CTA)
                         named_bar_sync(1, kSoft);
                         if (st == 0) SPI_TRACE(8);
                         if (st == 0) {
+                            __threadfence();
                             const int c_first = cta_of_tile(sd.ib, T, NC);
                             const int c_last = cta_of_tile(sd.ie - 1, T, NC);
                             int npieces = 0;
