@@ -84,11 +84,29 @@ __device__ __forceinline__ void tile_max(uint32_t s_col, const uint32_t (&vis)[4
     }
 }
 
+// Blackwell paired fp32 arithmetic (FFMA2 / FADD2: two lanes of work per instruction); the softmax
+// is issue-bound, so halving its FMA and FADD instruction count shortens the per-tile chain
+__device__ __forceinline__ uint64_t f2_bits(float a, float b) {
+    return (uint64_t)__float_as_uint(a) | ((uint64_t)__float_as_uint(b) << 32);
+}
+__device__ __forceinline__ uint64_t ffma2(uint64_t a, uint64_t b, uint64_t c) {
+    uint64_t d;
+    asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(d) : "l"(a), "l"(b), "l"(c));
+    return d;
+}
+__device__ __forceinline__ uint64_t fadd2(uint64_t a, uint64_t b) {
+    uint64_t d;
+    asm("add.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+    return d;
+}
+
 // P = 2^(s * scale_log2 - mref) of one S tile, packed to bf16 pairs over the first 64 columns of the
 // same TMEM buffer; accumulates the fp32 row sum.
 template <bool kMask>
 __device__ __forceinline__ void tile_exp(uint32_t s_col, const uint32_t (&vis)[4], float scale_log2, float mref,
                                          float (&l4)[4]) {
+    const uint64_t sc2 = f2_bits(scale_log2, scale_log2), nm2 = f2_bits(-mref, -mref);
+    uint64_t la = f2_bits(0.f, 0.f), lb = f2_bits(0.f, 0.f);  // paired row-sum accumulators
 #pragma unroll
     for (int h = 0; h < 2; ++h) {
         uint32_t v[2][32];
@@ -105,15 +123,20 @@ __device__ __forceinline__ void tile_exp(uint32_t s_col, const uint32_t (&vis)[4
                     x0 = ((vis[2 * h + q] >> (2 * i)) & 1u) ? x0 : -INFINITY;
                     x1 = ((vis[2 * h + q] >> (2 * i + 1)) & 1u) ? x1 : -INFINITY;
                 }
-                const float e0 = ex2(fmaf(x0, scale_log2, -mref));
-                const float e1 = ex2(fmaf(x1, scale_log2, -mref));
+                const uint64_t y = ffma2(f2_bits(x0, x1), sc2, nm2);
+                const float e0 = ex2(__uint_as_float((uint32_t)y));
+                const float e1 = ex2(__uint_as_float((uint32_t)(y >> 32)));
                 w16[i] = pack_bf16x2(e0, e1);
-                l4[(2 * i) & 3] += e0;
-                l4[(2 * i + 1) & 3] += e1;
+                if (i & 1) lb = fadd2(lb, f2_bits(e0, e1));
+                else la = fadd2(la, f2_bits(e0, e1));
             }
             tmem_st16(s_col + (2 * h + q) * 16, w16);
         }
     }
+    l4[0] += __uint_as_float((uint32_t)la);
+    l4[1] += __uint_as_float((uint32_t)(la >> 32));
+    l4[2] += __uint_as_float((uint32_t)lb);
+    l4[3] += __uint_as_float((uint32_t)(lb >> 32));
 }
 
 }  // namespace rows
