@@ -84,22 +84,6 @@ __device__ __forceinline__ void tile_max(uint32_t s_col, const uint32_t (&vis)[4
     }
 }
 
-// Blackwell paired fp32 arithmetic (FFMA2 / FADD2: two lanes of work per instruction); the softmax
-// is issue-bound, so halving its FMA and FADD instruction count shortens the per-tile chain
-__device__ __forceinline__ uint64_t f2_bits(float a, float b) {
-    return (uint64_t)__float_as_uint(a) | ((uint64_t)__float_as_uint(b) << 32);
-}
-__device__ __forceinline__ uint64_t ffma2(uint64_t a, uint64_t b, uint64_t c) {
-    uint64_t d;
-    asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(d) : "l"(a), "l"(b), "l"(c));
-    return d;
-}
-__device__ __forceinline__ uint64_t fadd2(uint64_t a, uint64_t b) {
-    uint64_t d;
-    asm("add.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
-    return d;
-}
-
 // P = 2^(s * scale_log2 - mref) of one S tile, packed to bf16 pairs over the first 64 columns of the
 // same TMEM buffer; accumulates the fp32 row sum.
 template <bool kMask>
