@@ -98,3 +98,46 @@ def test_tree_rope_then_attention(Hq, Hkv, Nmax):
         errs.append(np.abs(out[b, :n].float().cpu().numpy() - ref[b, :n]).reshape(-1))
     e = np.concatenate(errs)
     assert e.max() <= 1e-2 and e.mean() <= 1e-3, (e.max(), e.mean())
+
+
+def test_rope_then_commit_keeps_slot_positions():
+    """R29: after the tree is encoded at P_b + depth[i] and the accepted path is committed, every
+    committed slot P + j holds a key encoded at position P + j (path[j] has depth j), so the cache
+    stays a plain position-encoded sequence.  Checked against oracle.rope_rotate of the raw keys."""
+    rng = np.random.default_rng(21)
+    B, Hq, Hkv, Nmax, P = 3, 8, 4, 24, 257
+    trees = [W.random_tree(Nmax, 8, 3, rng) for _ in range(B)]
+    tb = W.make_tree_batch(trees, [P, P - 40, P + 9], max_nodes=Nmax, max_depth=8, device=DEV)
+    smax = P + 9 + Nmax + 3
+    ai = W.make_attention_inputs(tb, 1, Hq, Hkv, smax, seed=21, device=DEV)
+    shape = spi.make_shape(B, Nmax, Hq, Hkv, smax, max_depth=8)
+    k_raw = ai.k_cache[0].float().cpu().numpy()
+    spi.specinfer_tree_rope(shape, None, ai.k_cache[0], tb.prefix_len, tb.depth, tb.n_nodes)
+    # accepted path: root -> deepest-first-child chain (a valid root path of each tree)
+    par = tb.parent.cpu().numpy()
+    nn_ = tb.n_nodes.cpu().numpy()
+    paths = np.zeros((B, 9), np.int32)
+    n_acc = np.zeros(B, np.int32)
+    for b in range(B):
+        path = [0]
+        while True:
+            kids = [c for c in range(1, nn_[b]) if par[b, c] == path[-1]]
+            if not kids:
+                break
+            path.append(kids[-1])
+        paths[b, :len(path)] = path
+        n_acc[b] = len(path)
+    pl = tb.prefix_len.clone()
+    spi.specinfer_kv_commit(shape, ai.k_cache, ai.v_cache, pl, torch.from_numpy(paths).to(DEV),
+                            torch.from_numpy(n_acc).to(DEV))
+    torch.cuda.synchronize()
+    kg = ai.k_cache[0].float().cpu().numpy()
+    p0 = tb.prefix_len.cpu().numpy()
+    for b in range(B):
+        for j in range(n_acc[b]):
+            slot = int(p0[b]) + j
+            want = oracle.rope_rotate(k_raw[b, :, int(p0[b]) + paths[b, j]], np.full(Hkv, slot))
+            got = kg[b, :, slot]
+            raw = k_raw[b, :, int(p0[b]) + paths[b, j]]
+            assert np.all(np.abs(got - want) <= _bound(want, raw)), (b, j)
+    assert np.array_equal(pl.cpu().numpy(), p0 + n_acc)
