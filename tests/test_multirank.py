@@ -152,3 +152,26 @@ def test_two_rank_kv_head_sharding_equals_single_process():
             np.testing.assert_array_equal(o[b, :n[b]], out[b, :n[b], q0:q0 + nq])
             assert np.array_equal(kr[:, b, :, :plr[b]], k[:, b, kv0:kv0 + nkv, :pl[b]])
         assert np.array_equal(plr, pl)
+
+
+def test_bench_reference_arm_two_ranks_prints_one_line():
+    """`bench.py --impl reference` under torchrun at N = 2 (the driver's launch): rank 0 alone
+    times the oracle and prints ONE JSON line with the reference-arm keys; rank 1 exits 0."""
+    import json
+    import subprocess
+    import sys
+
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+           "--master-addr", "127.0.0.1", "--master-port", str(_free_port()), "bench.py",
+           "--impl", "reference", "--gpus", "2", "--steps", "1", "--warmup", "0", "--config", "C1"]
+    r = subprocess.run(cmd, cwd=root, capture_output=True, text=True, timeout=300)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1, r.stdout
+    d = json.loads(lines[0])
+    assert d["impl"] == "reference" and d["n_gpus"] == 2 and d["steps"] == 1
+    assert d["value"] > 0 and d["higher_is_better"] is True
+    assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["value"] == d["value"]
+    assert d["e2e"] == {"value": d["value"], "unit": d["unit"], "h2d_bytes_per_step": 0,
+                        "d2h_bytes_per_step": 0}
