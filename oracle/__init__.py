@@ -46,9 +46,11 @@ def lib():
         _lib.oracle_verify_greedy.argtypes = [i32, i32, i32, i32, i32, i32, vp, vp, vp, vp, vp,
                                               vp, vp, vp, vp]
         _lib.oracle_verify_mss.argtypes = [i32, i32, i32, i32, i32, i32, vp, vp, vp, vp, vp, vp,
-                                           vp, dbl, u64, u64, vp, vp, vp, vp, vp]
+                                           vp, dbl, u64, u64, vp, vp, vp, vp, vp,
+                                           i32, vp, vp, vp, vp, vp]
         _lib.oracle_verify_ns.argtypes = [i32, i32, i32, i32, i32, i32, vp, vp, vp, vp, vp, vp,
-                                          dbl, u64, u64, vp, vp, vp, vp, vp]
+                                          dbl, u64, u64, vp, vp, vp, vp, vp,
+                                          i32, vp, vp, vp, vp, vp]
         _lib.oracle_philox4x32_10.argtypes = [vp, vp, vp]
     return _lib
 
@@ -127,10 +129,31 @@ def verify_greedy(logits, tree_tokens, parent, n_nodes, *, depth=None, prefix_le
     return an, at, na
 
 
+class VerifyResult(tuple):
+    """(accepted_nodes, accepted_tokens, n_accepted, margin) plus ``.decisions``: per request the
+    list of decision records (node u, child s or -1 for a race, value, relative margin) in the
+    order the sampler took them (c4's decision log)."""
+    decisions: list
+
+
+def _decision_log(B, stride):
+    return (stride, np.full((B, stride), -1, np.int32), np.full((B, stride), -1, np.int32),
+            np.full((B, stride), -1, np.int32), np.full((B, stride), np.inf), np.zeros((B,), np.int32))
+
+
+def _result(an, at, na, mg, log):
+    _, dn, dc, dv, dm, nd = log
+    r = VerifyResult((an, at, na, mg))
+    r.decisions = [[(int(dn[b, k]), int(dc[b, k]), int(dv[b, k]), float(dm[b, k])) for k in range(nd[b])]
+                   for b in range(len(nd))]
+    return r
+
+
 def verify_mss(logits, tree_tokens, parent, n_nodes, draft_probs, *, temperature=1.0, seed=0,
                offset=0, request_ids=None, depth=None, prefix_len=None, smax=1 << 30,
                max_depth=255, path_len=None):
-    """c4 (Alg. 2).  Returns (accepted_nodes, accepted_tokens, n_accepted, margin)."""
+    """c4 (Alg. 2).  Returns (accepted_nodes, accepted_tokens, n_accepted, margin) with the
+    per-decision log in ``.decisions`` (VerifyResult)."""
     logits = _c(logits, np.float32)
     draft_probs = _c(draft_probs, np.float32)
     B, Nmax, V = logits.shape
@@ -141,14 +164,15 @@ def verify_mss(logits, tree_tokens, parent, n_nodes, draft_probs, *, temperature
     na = np.empty((B,), np.int32)
     mg = np.empty((B,), np.float64)
     rids = None if request_ids is None else _c(request_ids, np.int32)
+    log = _decision_log(B, Nmax + 1)
     lib().oracle_verify_mss(B, Nmax, V, smax, max_depth, path_len, _p(logits),
                             _p(_c(tree_tokens, np.int32)), _p(_c(parent, np.int32)),
                             _p(None if depth is None else _c(depth, np.int32)),
                             _p(None if prefix_len is None else _c(prefix_len, np.int32)),
                             _p(_c(n_nodes, np.int32)), _p(draft_probs), float(temperature),
                             int(seed) & (2**64 - 1), int(offset) & (2**64 - 1), _p(rids),
-                            _p(an), _p(at), _p(na), _p(mg))
-    return an, at, na, mg
+                            _p(an), _p(at), _p(na), _p(mg), log[0], *[_p(a) for a in log[1:]])
+    return _result(an, at, na, mg, log)
 
 
 def verify_ns(logits, tree_tokens, parent, n_nodes, *, temperature=1.0, seed=0, offset=0, request_ids=None,
@@ -164,12 +188,14 @@ def verify_ns(logits, tree_tokens, parent, n_nodes, *, temperature=1.0, seed=0, 
     na = np.empty((B,), np.int32)
     mg = np.empty((B,), np.float64)
     rids = None if request_ids is None else _c(request_ids, np.int32)
+    log = _decision_log(B, Nmax + 1)
     lib().oracle_verify_ns(B, Nmax, V, smax, max_depth, path_len, _p(logits), _p(_c(tree_tokens, np.int32)),
                            _p(_c(parent, np.int32)), _p(None if depth is None else _c(depth, np.int32)),
                            _p(None if prefix_len is None else _c(prefix_len, np.int32)),
                            _p(_c(n_nodes, np.int32)), float(temperature), int(seed) & (2**64 - 1),
-                           int(offset) & (2**64 - 1), _p(rids), _p(an), _p(at), _p(na), _p(mg))
-    return an, at, na, mg
+                           int(offset) & (2**64 - 1), _p(rids), _p(an), _p(at), _p(na), _p(mg),
+                           log[0], *[_p(a) for a in log[1:]])
+    return _result(an, at, na, mg, log)
 
 
 def philox4x32_10(ctr, key) -> np.ndarray:
@@ -255,6 +281,14 @@ def expand_topk(ssm_logits_row, k):
     row = np.asarray(ssm_logits_row, np.float64)
     order = sorted(range(len(row)), key=lambda x: (-row[x], x))
     return order[:k]
+
+
+def ssm_distribution(ssm_logits_row, temperature=1.0):
+    """The SSM distribution a node's children are drawn from (L455-468; reading R12: the draft row
+    of child c is the q that drew t_c), softmax(logits / T) in fp64, written out."""
+    x = np.asarray(ssm_logits_row, np.float64) / float(temperature)
+    e = np.exp(x - x.max())
+    return e / e.sum()
 
 
 def tree_merge(trees):

@@ -71,9 +71,7 @@ def test_expand_steps_parity(expansion, V):
             for c, t in _oracle_expand(rows, pd, dd, level).items():
                 expect[(b, c)] = t
                 f = frontier.index(pd[c])
-                x = rows[f].astype(np.float64) / 0.8
-                q = np.exp(x - x.max())
-                qrows[(b, c)] = q / q.sum()
+                qrows[(b, c)] = oracle.ssm_distribution(rows[f], 0.8)
     torch.cuda.synchronize()
     got = toks.cpu().numpy()
     dr = draft.cpu().numpy()

@@ -29,7 +29,7 @@ def test_verify_ns_parity(V, T):
     ref = oracle.verify_ns(vi.logits.cpu().numpy(), vi.tree_tokens.cpu().numpy(), tb.parent.cpu().numpy(),
                            tb.n_nodes.cpu().numpy(), temperature=T, seed=99, offset=5,
                            request_ids=rids.cpu().numpy(), path_len=9)
-    _mss_compare(outs, ref, ref[3])
+    _mss_compare(outs, ref, f"ns V={V} T={T}")
 
 
 def test_verify_ns_config_c2_full_and_leaf_contract():
@@ -42,7 +42,7 @@ def test_verify_ns_config_c2_full_and_leaf_contract():
     torch.cuda.synchronize()
     ref = oracle.verify_ns(vi.logits.cpu().numpy(), vi.tree_tokens.cpu().numpy(), tb.parent.cpu().numpy(),
                            tb.n_nodes.cpu().numpy(), seed=2, offset=0, path_len=cfg.max_depth + 1)
-    _mss_compare((an, at, na), ref, ref[3])
+    _mss_compare((an, at, na), ref, "ns C2 full")
     B = 32
     tb1 = W.make_tree_batch([W.chain_tree(1)] * B, [0] * B, max_depth=8, device=DEV)
     shape1, st1, vi1, o1 = _verify_setup(tb1, 4096, "mss", seed=5)

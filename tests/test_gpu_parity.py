@@ -10,6 +10,7 @@ import torch
 
 import oracle
 import workloads as W
+from tests.mss_compare import compare_sampled
 
 pytestmark = pytest.mark.gpu
 
@@ -394,15 +395,10 @@ def test_verify_greedy_fig2_and_ties(golden):
     assert at[0, 0].item() == 0 and na.item() == 1
 
 
-def _mss_compare(got, ref, margins, excuse=1e-5):
-    an, at, na = [x.cpu().numpy() for x in got]
-    r_an, r_at, r_na, _ = ref
-    bad = [b for b in range(len(na)) if not (na[b] == r_na[b] and np.array_equal(an[b], r_an[b])
-                                              and np.array_equal(at[b], r_at[b]))]
-    unexcused = [b for b in bad if margins[b] >= excuse]
-    assert not unexcused, f"MSS mismatches with margin >= {excuse}: {unexcused[:10]} (margins {margins[unexcused[:10]]})"
-    assert len(bad) <= max(1, int(1e-3 * len(na))), f"too many boundary cases: {len(bad)}"
-    return len(bad)
+def _mss_compare(got, ref, label=""):
+    """Bit-exact up to requests whose FIRST divergent decision has an oracle margin < 1e-5, at most
+    1e-4 of the requests, each printed (tests/mss_compare.py)."""
+    return compare_sampled(got, ref, label=label)
 
 
 @pytest.mark.parametrize("V,T", [(5, 1.0), (1000, 0.7), (32000, 1.0), (50272, 1.3)])
@@ -419,7 +415,7 @@ def test_verify_mss_parity(V, T):
     ref = oracle.verify_mss(vi.logits.cpu().numpy(), vi.tree_tokens.cpu().numpy(), tb.parent.cpu().numpy(),
                             tb.n_nodes.cpu().numpy(), vi.draft_probs.cpu().numpy(), temperature=T, seed=1234,
                             offset=17, request_ids=rids.cpu().numpy(), path_len=9)
-    _mss_compare(outs, ref, ref[3])
+    _mss_compare(outs, ref, f"mss V={V} T={T}")
 
 
 def test_verify_mss_config_c4_full():
@@ -433,7 +429,7 @@ def test_verify_mss_config_c4_full():
     ref = oracle.verify_mss(vi.logits.cpu().numpy(), vi.tree_tokens.cpu().numpy(), tb.parent.cpu().numpy(),
                             tb.n_nodes.cpu().numpy(), vi.draft_probs.cpu().numpy(), seed=4, offset=0,
                             path_len=cfg.max_depth + 1)
-    _mss_compare(outs, ref, ref[3])
+    _mss_compare(outs, ref, "mss C4 full")
 
 
 def test_verify_config_c2_full_greedy_and_mss():
@@ -456,7 +452,7 @@ def test_verify_config_c2_full_greedy_and_mss():
             r = oracle.verify_mss(vi.logits.cpu().numpy(), vi.tree_tokens.cpu().numpy(), tb.parent.cpu().numpy(),
                                   tb.n_nodes.cpu().numpy(), vi.draft_probs.cpu().numpy(), seed=2, offset=0,
                                   path_len=9)
-            _mss_compare((an, at, na), r, r[3])
+            _mss_compare((an, at, na), r, "mss C2 full")
 
 
 def test_philox_kat_on_device(golden):

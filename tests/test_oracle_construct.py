@@ -8,6 +8,7 @@ enumeration of the sequence sets S_u (Def. 3.1), and numpy's stable argsort for 
 import itertools
 
 import numpy as np
+import pytest
 
 import oracle
 import workloads as W
@@ -115,3 +116,43 @@ def test_merge_definition_3_2_brute_force():
         assert all(par[i] < i for i in range(1, len(par))) and par[0] == -1
     # roots must agree
     assert oracle.tree_merge([([-1], [1]), ([-1], [2])]) is None
+
+
+def test_ssm_distribution_pins():
+    """The draft row (R12) against a library routine (scipy softmax of logits / T), a closed form
+    (two tokens: p0 = 1 / (1 + e^{(l1 - l0) / T})) and the T -> 0 / uniform special cases."""
+    from scipy.special import softmax
+    rng = np.random.default_rng(3)
+    for T in (0.5, 1.0, 1.7):
+        row = rng.normal(size=97).astype(np.float32) * 3
+        np.testing.assert_allclose(oracle.ssm_distribution(row, T), softmax(row.astype(np.float64) / T),
+                                   rtol=1e-12, atol=0)
+    q = oracle.ssm_distribution(np.array([1.0, -0.5], np.float32), 0.8)
+    assert q[0] == pytest.approx(1.0 / (1.0 + np.exp((-0.5 - 1.0) / 0.8)), rel=1e-14)
+    assert np.array_equal(oracle.ssm_distribution(np.zeros(8, np.float32)), np.full(8, 1 / 8))
+    assert oracle.ssm_distribution(np.array([2.0, 1.0], np.float32), 1e-3)[0] == 1.0
+
+
+def test_validate_tree_every_branch():
+    """Def. 3.1 (L450-454) validity, one defect at a time on the Fig. 4 tree (golden): n_nodes out
+    of [1, Nmax], P + n > Smax, a root with a parent, a parent not before its child, depth not
+    parent's + 1, depth beyond Dmax; the valid tree passes at exactly the limits."""
+    g = load_golden("fig4_mask.json")
+    par = np.asarray(g["parent"], np.int32)
+    n = len(par)
+    dep = np.zeros(n, np.int32)
+    for i in range(1, n):
+        dep[i] = dep[par[i]] + 1
+    D = int(dep.max())
+    ok = lambda p, d, P=5, nn=n, nmax=n, dmax=D, smax=5 + n: oracle.validate_tree(p, d, P, nn, nmax, dmax, smax)
+    assert ok(par, dep) == 0
+    assert ok(par, dep, nn=0) != 0 and ok(par, dep, nn=n + 1) != 0            # n_nodes range
+    assert ok(par, dep, smax=5 + n - 1) != 0 and ok(par, dep, P=-1) != 0      # P + n > Smax, P < 0
+    p2 = par.copy(); p2[0] = 0
+    assert ok(p2, dep) != 0                                                   # root has a parent
+    p3 = par.copy(); p3[3] = 5
+    assert ok(p3, dep) != 0                                                   # parent after child
+    d2 = dep.copy(); d2[4] += 1
+    assert ok(par, d2) != 0                                                   # depth != depth[parent] + 1
+    assert ok(par, dep, dmax=D - 1) != 0                                      # depth > Dmax
+    assert ok(par, None, dmax=0) == 0                                         # no depth array: topology only
