@@ -1,18 +1,26 @@
 """bench.py — SpecInfer token-tree verification hot path on B200.
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--impl ours|reference]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--scaling strong|weak]
+                    [--impl ours|reference]
 
-One step = one verification iteration of the whole hot path over one
-batch of synthetic input: tree_prepare -> L x tree_attention -> verify_greedy and/or
-verify_mss -> (N>1: NCCL all-gather of accepted tokens) -> kv_commit.  The default workload is
-BASELINE.json configs[1] (C2, LLaMA-7B shape), the configuration the metric is quoted on.
+One step = one verification iteration of the whole hot path over one batch
+of synthetic input: tree_prepare -> L x tree_attention -> verify_greedy and/or verify_mss ->
+tokens-only gather of the accepted paths (NCCL at N > 1) -> kv_commit
+(paper_conf_asplos_miaoozcwzwzyssc24_b200/step.py).  The default workload is BASELINE.json
+configs[1] (C2, LLaMA-7B shape), the configuration the metric is quoted on.
 
-Prints ONE JSON line (rank 0).  `value` = verified tree tokens / s for the whole job with
-inputs resident in HBM; `e2e` = the same metric through the public API with host buffers
-(H2D of the step's q / logits / draft probabilities / tree, D2H of the accepted tokens inside
-the timed region).  `roofline` reports the dominant kernel (tree attention) against the
-measured HBM copy bandwidth; `cpu_baseline` times the fp64 oracle on a bounded sample.
-`--impl reference` times the oracle itself as the reference arm (there is no reference code).
+Scaling: `strong` (default) keeps the config's GLOBAL batch and splits it over the
+N ranks (request sharding; kv-head sharding for GQA configs); `weak` gives every rank the config's
+batch.  Every request's inputs come from its own seeded generator, so a rank materialises exactly
+its share of the global problem and the integer results equal the N = 1 run's.
+
+Prints ONE JSON line (rank 0).  `value` = verified tree tokens / s for the whole job with inputs
+resident in HBM; `e2e` = the same metric through the public API with host buffers (H2D of the
+step's q / logits / draft probabilities / tree, D2H of the accepted tokens inside the timed
+region).  `roofline` reports the dominant kernel (tree attention) against the measured HBM copy
+bandwidth (and the library's TMA read probe on the same bytes); `cpu_baseline` times the fp64
+oracle on a bounded sample, at all host cores and at one thread.  `--impl reference` times the
+oracle itself as the reference arm (there is no reference code).
 """
 from __future__ import annotations
 
@@ -44,14 +52,18 @@ def parse():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--config", default="C2", choices=sorted(W.CONFIGS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--scaling", default="strong", choices=["strong", "weak"],
+                    help="strong: the config's global batch split over the ranks; weak: that batch per rank")
     ap.add_argument("--layers", type=int, default=None, help="override layer count (sweeps only)")
-    ap.add_argument("--batch", type=int, default=None, help="override per-GPU batch (sweeps only)")
+    ap.add_argument("--batch", type=int, default=None,
+                    help="override the batch (global for --scaling strong, per GPU for weak; sweeps only)")
     ap.add_argument("--prefix", type=int, default=None, help="override prefix (sweeps only)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-early", action="store_true", help="plain attention launches (no EARLY_PREFIX)")
     ap.add_argument("--verify", default=None, help="comma list overriding the config's verify modes")
     ap.add_argument("--shard", default="auto", choices=["auto", "request", "kv"],
-                    help="N > 1 layout: request sharding, or kv-head sharding (GQA; auto for G > 1)")
+                    help="layout: request sharding, or kv-head sharding (GQA; auto for G > 1 at N > 1)")
     return ap.parse_args()
 
 
@@ -127,46 +139,55 @@ class ClockSampler:
 
 
 # ------------------------------------------------------------------------------------------
-# workload
+# workload: this rank's share of the global problem
 # ------------------------------------------------------------------------------------------
-class Workload:
-    """One GPU's share of the step.  Request sharding: this rank's B requests end to end.  kv-head
-    sharding (GQA, N > 1): attention and KV commit over ALL B*N requests for this rank's Hkv/N
-    kv-heads (and their q-heads), verification over this rank's B requests (dist.py)."""
+def global_batch(cfg: W.Config, args, ws: int) -> int:
+    b = args.batch or cfg.batch
+    return b * ws if args.scaling == "weak" else b
 
-    def __init__(self, cfg: W.Config, args, rank: int, device, ws: int = 1, kv_shard: bool = False):
-        self.cfg = cfg
+
+def use_kv_shard(cfg: W.Config, args, ws: int) -> bool:
+    G = cfg.num_q_heads // cfg.num_kv_heads
+    if args.shard == "kv":
+        return True
+    return ws > 1 and args.shard == "auto" and G > 1 and cfg.num_kv_heads % ws == 0
+
+
+class Workload:
+    """One rank's inputs (step.Layout): the attention batch (its requests, or all requests for its
+    kv-head shard) and the verification batch (its requests), generated per global request id."""
+
+    def __init__(self, cfg: W.Config, args, layout, device):
+        self.cfg, self.layout = cfg, layout
         self.L = args.layers or cfg.layers
-        self.B = args.batch or cfg.batch
         self.P = args.prefix or cfg.prefix
-        self.kv_shard = kv_shard
-        self.Batt = self.B * ws if kv_shard else self.B
-        self.Hq, self.Hkv, self.V = cfg.num_q_heads, cfg.num_kv_heads, cfg.vocab
-        self.req_lo = rank * self.B if kv_shard else 0
-        if kv_shard:
-            from paper_conf_asplos_miaoozcwzwzyssc24_b200 import dist as D
-            _, self.Hkv, _, self.Hq = D.shard_kv_heads(cfg.num_q_heads, cfg.num_kv_heads, ws, rank)
+        self.V = cfg.vocab
         self.verify = tuple(args.verify.split(",")) if args.verify else cfg.verify
         parent, depth = cfg.tree
         self.N = int(parent.shape[0])
         self.Dmax = cfg.max_depth
         self.smax = self.P + self.N
-        self.device = device
-        self.tb = W.make_tree_batch([(parent, depth)] * self.Batt, [self.P] * self.Batt, device=device,
-                                    max_depth=self.Dmax)
-        seed = cfg.seed + 1000 * rank
-        self.ai = W.make_attention_inputs(self.tb, self.L, self.Hq, self.Hkv, self.smax, seed=seed, device=device)
-        mode = "mss" if self.verify == ("mss",) else "greedy"
-        lo, hi = self.req_lo, self.req_lo + self.B
-        self.tbv = W.TreeBatch(self.tb.parent[lo:hi], self.tb.depth[lo:hi], self.tb.prefix_len[lo:hi],
-                               self.tb.n_nodes[lo:hi], self.tb.max_nodes, self.tb.max_depth)
-        self.vi = W.make_verify_inputs(self.tbv, self.V, seed=seed, mode=mode, device=device)
-        self.rids = torch.arange(rank * self.B, (rank + 1) * self.B, dtype=torch.int32, device=device)
-        self.bytes_launch = self.attn_bytes_per_launch()   # before any commit moves prefix_len
+        self.Hq, self.Hkv = layout.nq, layout.nkv
+        self.tb = W.make_tree_batch([(parent, depth)] * layout.attn_cnt, [self.P] * layout.attn_cnt,
+                                    device=device, max_depth=self.Dmax)
+        if layout.kv_shard:
+            self.tbv = W.make_tree_batch([(parent, depth)] * layout.req_cnt, [self.P] * layout.req_cnt,
+                                         device=device, max_depth=self.Dmax)
+        else:
+            self.tbv = self.tb
+        self.ai = W.make_request_attention_inputs(self.tb, list(layout.attn_ids), self.L, cfg.num_q_heads,
+                                                  cfg.num_kv_heads, self.smax, cfg.seed,
+                                                  q_heads=(layout.q0, layout.nq), kv_heads=(layout.kv0, layout.nkv),
+                                                  device=device)
+        # greedy trees take the top-k draft tokens, MSS trees i.i.d. draws (R13: only the latter carry
+        # MSS's distributional guarantee), so each verifier gets the tree tokens of its own mode
+        self.vi = {m: W.make_request_verify_inputs(self.tbv, list(layout.verify_ids), self.V, cfg.seed, m,
+                                                   device=device) for m in self.verify}
+        self.bytes_launch = self.attn_bytes_per_launch()
         self.flops_launch = self.attn_flops_per_launch()
 
     def tree_tokens_per_step(self) -> int:
-        """Tree tokens this rank verifies per step (its B requests)."""
+        """Tree tokens this rank verifies per step (its requests)."""
         return int(self.tbv.n_nodes.sum().item())
 
     def attn_bytes_per_launch(self) -> int:
@@ -182,70 +203,51 @@ class Workload:
         pl = self.tb.prefix_len.cpu().numpy().astype(np.int64)
         n = self.tb.n_nodes.cpu().numpy().astype(np.int64)
         dep = self.tb.depth.cpu().numpy()
-        tree_pairs = np.array([int((dep[b, :n[b]] + 1).sum()) for b in range(self.Batt)])
+        tree_pairs = np.array([int((dep[b, :n[b]] + 1).sum()) for b in range(len(n))])
         return int((4 * 128 * (n * pl + tree_pairs) * self.Hq).sum())
+
+
+def percentiles(xs, qs=(10, 50, 90)):
+    return {f"p{q}": round(float(np.percentile(xs, q)), 4) for q in qs}
 
 
 def run_ours(args, ws, rank, local):
     import paper_conf_asplos_miaoozcwzwzyssc24_b200 as spi
+    from paper_conf_asplos_miaoozcwzwzyssc24_b200 import step as S
 
     device = torch.device("cuda", local)
     torch.cuda.set_device(device)
     cfg = W.CONFIGS[args.config]
-    G = cfg.num_q_heads // cfg.num_kv_heads
-    # (--shard kv also runs at N = 1, where the gather degenerates to a copy: exercises the layout)
-    kv_shard = args.shard == "kv" or (ws > 1 and args.shard == "auto" and G > 1 and cfg.num_kv_heads % ws == 0)
-    wl = Workload(cfg, args, rank, device, ws=ws, kv_shard=kv_shard)
-    L, B, N, Dmax = wl.L, wl.B, wl.N, wl.Dmax
-    Ba = wl.Batt
-    Lp = Dmax + 1
-    # attention / commit shape (all B*N requests x local heads when kv-sharded) and verify shape
-    shape = spi.make_shape(Ba, N, wl.Hq, wl.Hkv, wl.smax, num_layers=L, vocab=wl.V, max_depth=Dmax)
-    st = spi.TreeState.create(shape, wl.tb.parent, wl.tb.depth, wl.tb.prefix_len, wl.tb.n_nodes)
-    if kv_shard:
-        shape_v = spi.make_shape(B, N, 1, 1, wl.smax, num_layers=L, vocab=wl.V, max_depth=Dmax)
-        st_v = spi.TreeState.create(shape_v, wl.tbv.parent, wl.tbv.depth, wl.tbv.prefix_len, wl.tbv.n_nodes)
-    else:
-        shape_v, st_v = shape, st
+    Bg = global_batch(cfg, args, ws)
+    kv_shard = use_kv_shard(cfg, args, ws)
+    layout = S.make_layout(Bg, ws, rank, cfg.num_q_heads, cfg.num_kv_heads, kv_shard)
+    wl = Workload(cfg, args, layout, device)
+    L, N, Dmax, Lp = wl.L, wl.N, wl.Dmax, wl.Dmax + 1
+    shape = spi.make_shape(layout.attn_cnt, N, wl.Hq, wl.Hkv, wl.smax, num_layers=L, vocab=wl.V, max_depth=Dmax)
+    shape_v = (spi.make_shape(layout.req_cnt, N, 1, 1, wl.smax, num_layers=L, vocab=wl.V, max_depth=Dmax)
+               if kv_shard else shape)
+    tree = (wl.tb.parent, wl.tb.depth, wl.tb.prefix_len, wl.tb.n_nodes)
+    tree_v = (wl.tbv.parent, wl.tbv.depth, wl.tbv.prefix_len, wl.tbv.n_nodes) if kv_shard else tree
+    step = S.VerifyStep(S.DeviceOps(), layout, shape, shape_v, tree, tree_v, wl.verify, Lp, device)
+    inputs = {m: (wl.vi[m].logits, wl.vi[m].tree_tokens, wl.vi[m].draft_probs if m == "mss" else None)
+              for m in wl.verify}
     out = torch.empty_like(wl.ai.q)
     prefix0 = wl.tb.prefix_len.clone()
-    an = torch.empty((B, Lp), dtype=torch.int32, device=device)
-    at, na = torch.empty_like(an), torch.empty((B,), dtype=torch.int32, device=device)
-    an2, at2, na2 = torch.empty_like(an), torch.empty_like(an), torch.empty_like(na)
-    gather_in = torch.empty((B, 2 * Lp + 1), dtype=torch.int32, device=device)
-    gather_out = torch.empty((ws * B, 2 * Lp + 1), dtype=torch.int32, device=device)
-    an_all = torch.empty((Ba, Lp), dtype=torch.int32, device=device)   # kv-sharded commit input
-    na_all = torch.empty((Ba,), dtype=torch.int32, device=device)
-    iteration = [0]
+    early = not args.no_early
 
     def seg_prepare():
-        wl.tb.prefix_len.copy_(prefix0)
-        st.prepare()
-        if kv_shard:
-            st_v.prepare()
+        wl.tb.prefix_len.copy_(prefix0)   # every step verifies a fresh tree over the same prefix
+        step.prepare()
 
     def seg_attention():
         for l in range(L):
-            st.attention(wl.ai.q[l], wl.ai.k_cache[l], wl.ai.v_cache[l], out[l])
+            step.attention(wl.ai.q[l], wl.ai.k_cache[l], wl.ai.v_cache[l], out[l], layer=l if early else 0)
 
     def seg_verify():
-        if "greedy" in wl.verify:
-            spi.specinfer_verify_greedy(shape_v, wl.vi.logits, wl.vi.tree_tokens, wl.tbv.parent, wl.tbv.n_nodes,
-                                        an, at, na, st_v.workspace)
-        if "mss" in wl.verify:
-            spi.specinfer_verify_mss(shape_v, wl.vi.logits, wl.vi.tree_tokens, wl.tbv.parent, wl.tbv.n_nodes,
-                                     wl.vi.draft_probs, 1.0, cfg.seed, 0, wl.rids, an2, at2, na2, st_v.workspace)
+        step.verify(inputs, seed=cfg.seed, offset=0)
 
     def seg_commit():
-        if kv_shard:
-            # every request's accepted path (gathered) -> this rank's kv-head shard of its cache
-            n_all, _, nodes_all = D.unpack_accepted(gather_out)
-            na_all.copy_(n_all)
-            an_all.copy_(nodes_all)
-            src = (an_all, na_all)
-        else:
-            src = (an, na) if "greedy" in wl.verify else (an2, na2)
-        spi.specinfer_kv_commit(shape, wl.ai.k_cache, wl.ai.v_cache, wl.tb.prefix_len, src[0], src[1])
+        step.commit(wl.ai.k_cache, wl.ai.v_cache)
 
     launches_per_step = (spi.specinfer_launches_per_call("tree_prepare") * (2 if kv_shard else 1) +
                          L * spi.specinfer_launches_per_call("tree_attention") +
@@ -253,29 +255,12 @@ def run_ours(args, ws, rank, local):
                          ("mss" in wl.verify) * spi.specinfer_launches_per_call("verify_mss") +
                          spi.specinfer_launches_per_call("kv_commit"))
 
-    from paper_conf_asplos_miaoozcwzwzyssc24_b200 import dist as D
-
-    def gather():
-        # a7: the tokens-only exchange after verification, NCCL over NVLink
-        if ws > 1 or kv_shard:
-            src = (na, at, an) if "greedy" in wl.verify else (na2, at2, an2)
-            gather_in.copy_(D.pack_accepted(*src))
-            if ws > 1:
-                D.gather_accepted(gather_in, gather_out)
-            else:
-                gather_out.copy_(gather_in)
-
-    def seg_verify_commit():
-        seg_verify()
-        gather()
-        seg_commit()
-
     # ---- capture the segments as CUDA graphs (one launch each per step; the gather stays eager) ----
     s = torch.cuda.Stream(device)
     s.wait_stream(torch.cuda.current_stream(device))
     with torch.cuda.stream(s):
         for _ in range(2):  # eager warm-up (lazy init, tensor-map encode, func attributes)
-            seg_prepare(); seg_attention(); seg_verify_commit()
+            seg_prepare(); seg_attention(); seg_verify(); step.gather(); seg_commit()
     torch.cuda.synchronize(device)
     graphs = []
     for fn in (seg_prepare, seg_attention, seg_verify, seg_commit):
@@ -285,19 +270,13 @@ def run_ours(args, ws, rank, local):
         graphs.append(g)
     torch.cuda.synchronize(device)
 
-    def step():
-        graphs[0].replay()
-        graphs[1].replay()
-        graphs[2].replay()
-        gather()
-        graphs[3].replay()
-
     with torch.cuda.stream(s):
         for _ in range(args.warmup):
-            step()
+            graphs[0].replay(); graphs[1].replay(); graphs[2].replay(); step.gather(); graphs[3].replay()
     torch.cuda.synchronize(device)
     K = args.steps
-    ev = [torch.cuda.Event(enable_timing=True) for _ in range(2 * K + 2)]
+    ev = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(K)]
+    e_all = [torch.cuda.Event(enable_timing=True) for _ in range(2)]
     sampler = ClockSampler(local) if rank == 0 else None
     barrier(ws)
     torch.cuda.synchronize(device)
@@ -305,28 +284,34 @@ def run_ours(args, ws, rank, local):
         sampler.start()
         time.sleep(0.3)
     with torch.cuda.stream(s):
-        ev[0].record(s)
+        e_all[0].record(s)
         for k in range(K):
+            ev[k][0].record(s)
             graphs[0].replay()
-            ev[2 + 2 * k].record(s)
+            ev[k][1].record(s)
             graphs[1].replay()
-            ev[3 + 2 * k].record(s)
+            ev[k][2].record(s)
             graphs[2].replay()
-            gather()
+            step.gather()
             graphs[3].replay()
-        ev[1].record(s)
+        e_all[1].record(s)
     torch.cuda.synchronize(device)
     barrier(ws)
     clocks = sampler.stop() if sampler else None
-    total_ms = ev[0].elapsed_time(ev[1])
-    attn_ms = sum(ev[2 + 2 * k].elapsed_time(ev[3 + 2 * k]) for k in range(K))
-    total_ms = max_over_ranks(total_ms, ws, device)
+    total_ms = max_over_ranks(e_all[0].elapsed_time(e_all[1]), ws, device)
+    step_ms = [ev[k][0].elapsed_time(ev[k + 1][0]) for k in range(K - 1)] + \
+              [ev[K - 1][0].elapsed_time(e_all[1])]
+    attn_ms = sum(ev[k][1].elapsed_time(ev[k][2]) for k in range(K))
     attn_ms_max = max_over_ranks(attn_ms, ws, device)
     ms_per_step = total_ms / K
-    tokens_step = wl.tree_tokens_per_step()
-    value = tokens_step * ws * K / (total_ms / 1e3)
-    acc_mean = float((na if "greedy" in wl.verify else na2).float().mean().item())
-    acc_mss = float(na2.float().mean().item()) if "mss" in wl.verify else None
+    tokens_step_global = int(wl.tree_tokens_per_step())
+    if ws > 1:
+        t = torch.tensor([tokens_step_global], dtype=torch.int64, device=device)
+        torch.distributed.all_reduce(t)
+        tokens_step_global = int(t.item())
+    value = tokens_step_global * K / (total_ms / 1e3)
+    na_c = step.accepted()[0]
+    acc = {m: float(step.res[m][2].float().mean().item()) for m in wl.verify}
 
     # ---- roofline of the dominant kernel (tree attention), measured in the timed region ----
     attn_launch_s = attn_ms_max / (K * L) / 1e3
@@ -342,13 +327,14 @@ def run_ours(args, ws, rank, local):
     traffic = None
     try:
         tr = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
-        ent = tr.get(f"{args.config}:L{L}:B{B}:P{wl.P}") or tr.get(args.config)
+        ent = tr.get(f"{args.config}:L{L}:B{layout.attn_cnt}:P{wl.P}") or (tr.get(args.config) if ws == 1 else None)
         if ent:
             traffic = ent["dram_bytes_per_launch"]
     except Exception:
         pass
-    # a kernel timed inside a long step takes the sustained tensor figure when the driver measured it
+    # a kernel timed inside a long step takes the sustained tensor figure; the burst one is reported beside
     tf_peak, tf_src = 1590.0, "fallback (B200_PROFILING.md)"
+    tf_burst = float(peaks.get("bf16_tflops", 1590.0)) if peaks else 1590.0
     if peaks:
         if "bf16_tflops_sustained" in peaks:
             tf_peak, tf_src = float(peaks["bf16_tflops_sustained"]), "measured sustained (MEASURED_PEAKS.json)"
@@ -363,32 +349,51 @@ def run_ours(args, ws, rank, local):
         roofline = {"bound": "tensor", "kernel": kname, "achieved": round(tflops, 2), "peak": tf_peak,
                     "unit": "TFLOP/s", "frac": round(tflops / tf_peak, 4), "traffic": traffic,
                     "peak_source": tf_src, "algorithmic_flops_per_launch": flops_launch,
+                    "frac_of_burst_tensor": round(tflops / tf_burst, 4), "burst_tensor_peak": tf_burst,
                     "hbm_gbs": round(achieved, 1), "hbm_frac": round(achieved / peak, 4), "hbm_peak": peak,
                     "hbm_peak_source": peak_src}
     else:
         roofline = {"bound": "hbm", "kernel": kname, "achieved": round(achieved, 1), "peak": peak,
                     "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": traffic,
                     "peak_source": peak_src, "tensor_tflops": round(tflops, 2),
-                    "tensor_frac": round(tflops / tf_peak, 4), "tensor_peak": tf_peak}
+                    "tensor_frac": round(tflops / tf_peak, 4), "tensor_peak": tf_peak,
+                    "tensor_frac_of_burst": round(tflops / tf_burst, 4)}
     # BASELINE.json's north star quotes the KV stream against "about 8 TB/s": context only
     roofline["hbm_frac_of_8TBps"] = round(achieved / 8000.0, 4)
     roofline.update({"algorithmic_bytes_per_launch": bytes_launch, "arithmetic_intensity": round(ai_launch, 1),
                      "avg_launch_us": round(attn_launch_s * 1e6, 2),
                      "share_of_step": round(attn_ms_max / total_ms, 4)})
+    # the practical ceiling: the library's TMA read probe over the same K and V bytes (one layer)
+    probe_ms = []
+    with torch.cuda.stream(s):
+        for it in range(6):
+            p0, p1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            p0.record(s)
+            spi.specinfer_hbm_read_probe(wl.ai.k_cache[it % L])
+            spi.specinfer_hbm_read_probe(wl.ai.v_cache[it % L])
+            p1.record(s)
+            probe_ms.append((p0, p1))
+    torch.cuda.synchronize(device)
+    probe_s = statistics.median(a.elapsed_time(b) for a, b in probe_ms[1:]) / 1e3
+    probe_gbs = 2 * wl.ai.k_cache[0].numel() * 2 / probe_s / 1e9
+    roofline["tma_read_probe_gbs"] = round(probe_gbs, 1)
+    roofline["hbm_frac_of_tma_probe"] = round(achieved / probe_gbs, 4)
 
     # ---- end to end through the public API with host buffers ----
     e2e = None
     if not args.no_e2e:
         h_q = torch.empty_like(wl.ai.q, device="cpu").pin_memory()
         h_q.copy_(wl.ai.q)
-        h_logits = wl.vi.logits.cpu().pin_memory()
-        h_draft = wl.vi.draft_probs.cpu().pin_memory() if "mss" in wl.verify else None
-        h_tree = [t.cpu().pin_memory() for t in (wl.tb.parent, wl.tb.depth, wl.vi.tree_tokens, wl.tb.n_nodes, prefix0)]
-        h_res_a = torch.empty((B, Lp), dtype=torch.int32).pin_memory()
-        h_res_n = torch.empty((B,), dtype=torch.int32).pin_memory()
-        res_a, res_n = (at, na) if "greedy" in wl.verify else (at2, na2)
-        dsts = [wl.tb.parent, wl.tb.depth, wl.vi.tree_tokens, wl.tb.n_nodes, prefix0]
-        h2d = h_q.numel() * 2 + h_logits.numel() * 4 + (h_draft.numel() * 4 if h_draft is not None else 0) + \
+        h_in = {m: [t.cpu().pin_memory() for t in (wl.vi[m].logits, wl.vi[m].tree_tokens)] +
+                ([wl.vi[m].draft_probs.cpu().pin_memory()] if m == "mss" else []) for m in wl.verify}
+        d_in = {m: [wl.vi[m].logits, wl.vi[m].tree_tokens] + ([wl.vi[m].draft_probs] if m == "mss" else [])
+                for m in wl.verify}
+        tree_dev = [wl.tb.parent, wl.tb.depth, wl.tb.n_nodes, prefix0]
+        h_tree = [t.cpu().pin_memory() for t in tree_dev]
+        res_a, res_n = step.res[step.commit_mode][1], step.res[step.commit_mode][2]
+        h_res_a = torch.empty(tuple(res_a.shape), dtype=torch.int32).pin_memory()
+        h_res_n = torch.empty(tuple(res_n.shape), dtype=torch.int32).pin_memory()
+        h2d = h_q.numel() * 2 + sum(t.numel() * t.element_size() for v in h_in.values() for t in v) + \
             sum(t.numel() * 4 for t in h_tree)
         d2h = h_res_a.numel() * 4 + h_res_n.numel() * 4
 
@@ -396,32 +401,32 @@ def run_ours(args, ws, rank, local):
         # engines) and each layer's attention waits only for its own q, so the PCIe transfer of
         # layer l+1's q and of the logits / draft probabilities overlaps the attention of layer l.
         copy_s = torch.cuda.Stream(device)
-        ev_fork = torch.cuda.Event()
-        ev_tree = torch.cuda.Event()
+        ev_fork, ev_tree, ev_lg = torch.cuda.Event(), torch.cuda.Event(), torch.cuda.Event()
         ev_q = [torch.cuda.Event() for _ in range(L)]
-        ev_lg = torch.cuda.Event()
 
         def e2e_step():
             ev_fork.record(s)
             copy_s.wait_event(ev_fork)
             with torch.cuda.stream(copy_s):
-                for d, h in zip(dsts, h_tree):
+                for d, h in zip(tree_dev, h_tree):
                     d.copy_(h, non_blocking=True)
                 ev_tree.record(copy_s)
                 for l in range(L):
                     wl.ai.q[l].copy_(h_q[l], non_blocking=True)
                     ev_q[l].record(copy_s)
-                wl.vi.logits.copy_(h_logits, non_blocking=True)
-                if h_draft is not None:
-                    wl.vi.draft_probs.copy_(h_draft, non_blocking=True)
+                for m in wl.verify:
+                    for d, h in zip(d_in[m], h_in[m]):
+                        d.copy_(h, non_blocking=True)
                 ev_lg.record(copy_s)
             s.wait_event(ev_tree)
             seg_prepare()
             for l in range(L):
                 s.wait_event(ev_q[l])
-                st.attention(wl.ai.q[l], wl.ai.k_cache[l], wl.ai.v_cache[l], out[l])
+                step.attention(wl.ai.q[l], wl.ai.k_cache[l], wl.ai.v_cache[l], out[l], layer=l if early else 0)
             s.wait_event(ev_lg)
-            seg_verify_commit()
+            seg_verify()
+            step.gather()
+            seg_commit()
             h_res_a.copy_(res_a, non_blocking=True)
             h_res_n.copy_(res_n, non_blocking=True)
 
@@ -455,12 +460,12 @@ def run_ours(args, ws, rank, local):
         torch.cuda.synchronize(device)
         barrier(ws)
         e2e_ms = max_over_ranks(e0.elapsed_time(e1), ws, device)
-        e2e = {"value": round(tokens_step * ws * K / (e2e_ms / 1e3), 1), "unit": UNIT,
+        e2e = {"value": round(tokens_step_global * K / (e2e_ms / 1e3), 1), "unit": UNIT,
                "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
                "ms_per_step": round(e2e_ms / K, 4),
-               "inputs": "per step from pinned host memory: tree arrays, q of every layer, logits"
-                         + (", draft probabilities" if h_draft is not None else "")
-                         + "; result read back: accepted tokens + counts; H2D on a copy stream "
+               "inputs": "per step from pinned host memory: tree arrays, q of every layer, logits + tree tokens"
+                         + (" + draft probabilities" if "mss" in wl.verify else "")
+                         + " of each verifier; result read back: accepted tokens + counts; H2D on a copy stream "
                            "overlapping the attention of earlier layers"}
 
     cpu = None
@@ -472,21 +477,25 @@ def run_ours(args, ws, rank, local):
     line = {
         "metric": METRIC, "value": round(value, 1), "unit": UNIT, "n_gpus": ws, "steps": K,
         "warmup": args.warmup, "ms_per_step": round(ms_per_step, 4), "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
-        "config": {"workload": f"{cfg.name}: {cfg.description}", "layers": L, "batch_per_gpu": B,
-                   "global_batch": B * ws, "prefix": wl.P, "tree_nodes": N, "max_depth": Dmax,
-                   "num_q_heads": wl.Hq, "num_kv_heads": wl.Hkv, "vocab": wl.V, "verify": list(wl.verify),
-                   "parallelism": (f"kv-head-sharded attention/commit x{ws}, request-sharded verification" if kv_shard
+        "scaling": args.scaling, "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
+        "config": {"workload": f"{cfg.name}: {cfg.description}", "layers": L, "global_batch": Bg,
+                   "batch_per_gpu": layout.req_cnt, "prefix": wl.P, "tree_nodes": N, "max_depth": Dmax,
+                   "num_q_heads": cfg.num_q_heads, "num_kv_heads": cfg.num_kv_heads, "vocab": wl.V,
+                   "verify": list(wl.verify),
+                   "parallelism": (f"kv-head-sharded attention/commit x{ws} ({layout.nkv} kv-heads per GPU), "
+                                   f"request-sharded verification" if kv_shard
                                    else f"request-sharded x{ws}") if ws > 1 else "single GPU",
-                   "l2": "no flush: every step streams the full KV cache "
-                         f"({2 * L * B * wl.Hkv * wl.smax * 256 / 1e9:.1f} GB/GPU) >> 126 MB L2",
-                   "graph": "4 CUDA graphs per step (prepare | L x attention | verify | commit), NCCL gather between"},
+                   "l2": "no flush: every step streams this GPU's KV cache "
+                         f"({2 * L * layout.attn_cnt * wl.Hkv * wl.smax * 256 / 1e9:.1f} GB) >> 126 MB L2",
+                   "graph": "4 CUDA graphs per step (prepare | L x attention | verify | commit), the tokens-only "
+                            "gather between (NCCL at N > 1)",
+                   "attention_launch": "SPECINFER_ATTN_EARLY_PREFIX on layers >= 1" if early else "plain"},
+        "step_ms": percentiles(step_ms),
         "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
         "gpu_launches": launches_per_step * K, "clocks": clocks,
-        "extra": {"tree_tokens_per_step": tokens_step * ws, "mean_n_accepted_greedy": acc_mean if "greedy" in wl.verify else None,
-                  "mean_n_accepted_mss": acc_mss,
-                  "accepted_tokens_per_s": round(float((na if "greedy" in wl.verify else na2).sum().item()) * ws * K /
-                                                 (total_ms / 1e3), 1),
+        "extra": {"tree_tokens_per_step": tokens_step_global,
+                  "mean_n_accepted": acc, "committed_verifier": step.commit_mode,
+                  "accepted_tokens_per_s_rank0": round(float(na_c.sum().item()) * K / (total_ms / 1e3), 1),
                   "attention_ms_per_step": round(attn_ms_max / K, 4)},
     }
     if rank == 0:
@@ -496,18 +505,16 @@ def run_ours(args, ws, rank, local):
 # ------------------------------------------------------------------------------------------
 # CPU baseline: the fp64 oracle as it stands, on a bounded sample of the same workload
 # ------------------------------------------------------------------------------------------
-def _oracle_sample(wl: Workload, n_req: int, layers=(0,)):
+def _oracle_sample(wl: Workload, n_req: int, layers=(0,), threads=None):
     """Times the fp64 oracle (as it stands) on `n_req` requests of the workload: tree attention of the
-    given layers, then greedy / MSS verification of those requests."""
+    given layers, then greedy / MSS verification of those requests.  Returns (attention s,
+    verification s, threads used)."""
     import oracle
-    cores = len(os.sched_getaffinity(0))
-    os.environ["OMP_NUM_THREADS"] = str(cores)
-    tb = wl.tb
+    cores = threads or len(os.sched_getaffinity(0))
+    oracle.set_num_threads(cores)
+    tb, tbv = wl.tb, wl.tbv
     par, dep = tb.parent[:n_req].cpu(), tb.depth[:n_req].cpu()
     pl, nn_ = tb.prefix_len[:n_req].cpu(), tb.n_nodes[:n_req].cpu()
-    lg = wl.vi.logits[:n_req].cpu().numpy()
-    toks = wl.vi.tree_tokens[:n_req].cpu().numpy()
-    dr = wl.vi.draft_probs[:n_req].cpu().numpy() if "mss" in wl.verify else None
     ta = 0.0
     for l in layers:
         q = wl.ai.q[l, :n_req].cpu()
@@ -516,59 +523,79 @@ def _oracle_sample(wl: Workload, n_req: int, layers=(0,)):
         t0 = time.perf_counter()
         oracle.tree_attention(q, k, v, par, dep, pl, nn_)
         ta += time.perf_counter() - t0
+    nv = min(n_req, tbv.parent.shape[0])
+    pv, nnv = tbv.parent[:nv].cpu().numpy(), tbv.n_nodes[:nv].cpu().numpy()
     t1 = time.perf_counter()
-    if "greedy" in wl.verify:
-        oracle.verify_greedy(lg, toks, par.numpy(), nn_.numpy(), path_len=wl.Dmax + 1)
-    if "mss" in wl.verify:
-        oracle.verify_mss(lg, toks, par.numpy(), nn_.numpy(), dr, seed=1, path_len=wl.Dmax + 1)
+    for m, vi in wl.vi.items():
+        lg, toks = vi.logits[:nv].cpu().numpy(), vi.tree_tokens[:nv].cpu().numpy()
+        if m == "greedy":
+            oracle.verify_greedy(lg, toks, pv, nnv, path_len=wl.Dmax + 1)
+        else:
+            oracle.verify_mss(lg, toks, pv, nnv, vi.draft_probs[:nv].cpu().numpy(), seed=1, path_len=wl.Dmax + 1)
     tv = time.perf_counter() - t1
     return ta, tv, cores
 
 
 def cpu_baseline(wl: Workload, budget_s: float = 12.0):
     """The oracle timed on the host cores on a bounded sample (~10-20 s): every request of the
-    step, as many layers as fit the budget (extrapolated linearly to all layers when fewer)."""
-    import oracle  # noqa: F401  (test infrastructure; only this leg and --impl reference use it)
-    ta1, tv, cores = _oracle_sample(wl, wl.B, layers=(0,))
+    step, as many layers as fit the budget (extrapolated linearly to all layers when fewer); and
+    at ONE thread on one request x one layer (scaled to the step)."""
+    B = wl.tb.parent.shape[0]
+    ta1, tv, cores = _oracle_sample(wl, B, layers=(0,))
     n_layers = int(max(1, min(wl.L, budget_s // max(ta1, 1e-3))))
     if n_layers > 1:
-        ta, tv, cores = _oracle_sample(wl, wl.B, layers=tuple(range(n_layers)))
+        ta, tv, cores = _oracle_sample(wl, B, layers=tuple(range(n_layers)))
     else:
         ta = ta1
     t_step = ta * wl.L / n_layers + tv
     tokens = wl.tree_tokens_per_step()
     extra = "" if n_layers == wl.L else f", x{wl.L / n_layers:.1f} extrapolated to {wl.L} layers"
+    # one thread: one request, one layer (+ its verification), scaled by requests and layers
+    t1a, t1v, _ = _oracle_sample(wl, 1, layers=(0,), threads=1)
+    t_step1 = (t1a * wl.L + t1v) * B
     return {"value": round(tokens / t_step, 3), "unit": UNIT, "cores": cores, "kind": "oracle",
-            "sample": f"all {wl.B} requests, tree attention of {n_layers} of {wl.L} layers "
-                      f"({ta:.1f} s fp64{extra}) + greedy/MSS verification ({tv:.2f} s)"}
+            "sample": f"all {B} requests, tree attention of {n_layers} of {wl.L} layers "
+                      f"({ta:.1f} s fp64{extra}) + greedy/MSS verification ({tv:.2f} s)",
+            "one_thread": {"value": round(tokens / t_step1, 4), "unit": UNIT, "cores": 1,
+                           "sample": f"1 request x 1 layer ({t1a:.2f} s) + its verification ({t1v:.3f} s), "
+                                     f"scaled x{wl.L} layers x {B} requests"}}
 
 
 def run_reference(args, ws, rank, local):
     """Reference arm: the oracle timed on the host cores (there is no reference code; PAPER.md
-    only).  Rank 0 alone runs at N>1."""
+    only).  Rank 0 alone runs at N>1.  One reference step = the oracle's pass over ONE layer of the
+    arm's whole global batch plus its verification (measured; `ms_per_step` is that time), cycling
+    through the layers; `value` extrapolates the layer time to all L layers (labelled)."""
     if rank != 0:
         return
+    from paper_conf_asplos_miaoozcwzwzyssc24_b200 import step as S
     cfg = W.CONFIGS[args.config]
+    Bg = global_batch(cfg, args, ws)
     device = torch.device("cuda", local) if torch.cuda.is_available() else torch.device("cpu")
-    a = argparse.Namespace(**vars(args))
-    a.batch = 1
-    wl = Workload(cfg, a, 0, device)
+    layout = S.make_layout(Bg, 1, 0, cfg.num_q_heads, cfg.num_kv_heads, False)
+    wl = Workload(cfg, args, layout, device)
     for _ in range(args.warmup):
-        _oracle_sample(wl, 1)
-    t_tot = 0.0
-    tokens = 0
-    cores = 1
+        _oracle_sample(wl, Bg, layers=(0,))
+    ta_s, tv_s, cores = [], [], 1
+    w0 = time.perf_counter()
     for it in range(args.steps):
-        ta, tv, cores = _oracle_sample(wl, 1, layers=(it % wl.L,))
-        t_tot += ta * wl.L + tv
-        tokens += int(wl.tb.n_nodes[:1].sum().item())
-    value = tokens / t_tot
-    sample = f"1 request x 1 layer of {cfg.name} tree attention per step (fp64 oracle, x{wl.L} layers extrapolated) + its verification"
+        ta, tv, cores = _oracle_sample(wl, Bg, layers=(it % wl.L,))
+        ta_s.append(ta)
+        tv_s.append(tv)
+    wall = time.perf_counter() - w0
+    tokens = wl.tree_tokens_per_step()
+    t_full = statistics.mean(ta_s) * wl.L + statistics.mean(tv_s)
+    value = tokens / t_full
+    sample = (f"per step: fp64 oracle tree attention of one layer of all {Bg} requests ({statistics.mean(ta_s):.3f} s) "
+              f"+ their verification ({statistics.mean(tv_s):.3f} s); value extrapolates the layer to {wl.L} layers")
     print(json.dumps({
         "impl": "reference", "metric": METRIC, "value": round(value, 3), "unit": UNIT, "n_gpus": ws,
-        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(1e3 * t_tot / args.steps, 3),
-        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-        "config": {"workload": f"{cfg.name}: {cfg.description}"},
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(1e3 * wall / args.steps, 3),
+        "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": f"{cfg.name}: {cfg.description}", "layers": wl.L, "global_batch": Bg,
+                   "prefix": wl.P, "tree_nodes": wl.N, "verify": list(wl.verify)},
+        "extrapolated": {"seconds_per_full_iteration": round(t_full, 3), "layers_measured_per_step": 1,
+                         "layers": wl.L},
         "cpu_baseline": {"value": round(value, 3), "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample},
         "e2e": {"value": round(value, 3), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }), flush=True)

@@ -22,7 +22,9 @@
  * General conventions
  *   - Every data pointer is a DEVICE pointer unless stated otherwise; the caller owns every
  *     buffer (allocation, lifetime, freeing).  The library never allocates device memory and
- *     keeps no global mutable state except a per-device capability cache.
+ *     keeps no global mutable state except a per-device capability cache (sm_100 check, SM
+ *     count, shared-memory limit, and which kernels already carry their shared-memory
+ *     attribute on that device; thread-safe).  The production build has no debug hooks.
  *   - Every call is asynchronous and stream-ordered on `stream` (a cudaStream_t; NULL = the
  *     legacy default stream).  Calls are CUDA-graph capturable.
  *   - Host-checkable errors (NULL pointer, unsupported shape, non-sm_100 device) are returned
@@ -113,11 +115,29 @@ specinfer_status_t specinfer_tree_attention(const specinfer_shape_t *shape, cons
                                             const int32_t *prefix_len, const int32_t *n_nodes,
                                             void *out, void *workspace, specinfer_stream_t stream);
 
+/* specinfer_tree_attention with launch flags (0 = specinfer_tree_attention exactly).
+ * SPECINFER_ATTN_EARLY_PREFIX: the kernel's producers may read the attention schedule in
+ * `workspace` and stage committed-prefix K/V tiles (slots < P_b) BEFORE the programmatic
+ * dependency on the preceding kernel of `stream` resolves (programmatic dependent launch: that
+ * kernel may still be running).  Valid only when the immediately preceding kernel on `stream` wrote
+ * neither those cache slots nor the workspace schedule, i.e. it was not tree_prepare or kv_commit
+ * for this state; the tree slots, q and everything else are still read after the dependency.
+ * Consecutive layers' attention launches qualify (the bench passes it for every layer but the
+ * first).  Unknown flag bits: SPECINFER_ERR_INVALID_ARG.  Results are identical either way. */
+#define SPECINFER_ATTN_EARLY_PREFIX 1u
+specinfer_status_t specinfer_tree_attention_ex(const specinfer_shape_t *shape, const void *q,
+                                               const void *k_cache, const void *v_cache,
+                                               const int32_t *parent, const int32_t *depth,
+                                               const int32_t *prefix_len, const int32_t *n_nodes,
+                                               void *out, void *workspace, uint32_t flags,
+                                               specinfer_stream_t stream);
+
 /* a4 (K4).  VerifyGreedy (Alg. 2): O(u) = lowest token id attaining max logits[u];
  * from the root, repeatedly move to the lowest-index child whose token equals O(u) (R7);
  * finally emit O(u).  Writes accepted_nodes[b] = [0, v1..vL], accepted_tokens[b] =
  * [t_v1..t_vL, O(vL)], n_accepted[b] = L + 1; unused entries -1.  Invalid trees: n_accepted 0.
- * Needs the workspace of tree_prepare for the same tree. */
+ * Needs the workspace of tree_prepare for the same tree.  `logits` must be 16-byte aligned
+ * (rows are read with 128-bit loads when V % 4 == 0), else SPECINFER_ERR_INVALID_ARG. */
 specinfer_status_t specinfer_verify_greedy(const specinfer_shape_t *shape, const float *logits,
                                            const int32_t *tree_tokens, const int32_t *parent,
                                            const int32_t *n_nodes, int32_t *accepted_nodes,
@@ -131,7 +151,8 @@ specinfer_status_t specinfer_verify_greedy(const specinfer_shape_t *shape, const
  * with token x iff p[x] > 0 and r*q_s[x] <= p[x] (q_s = draft_probs[s], the distribution s was
  * drawn from, R12); on reject p <- norm(max(0, p - q_s)) (kept if all zero, R11); after the
  * last rejection (or at a leaf) sample x_next ~ p by an exponential race.  Outputs as for
- * verify_greedy.  temperature > 0.  Needs the workspace of tree_prepare for the same tree. */
+ * verify_greedy.  temperature > 0.  Needs the workspace of tree_prepare for the same tree.
+ * `logits` and `draft_probs` must be 16-byte aligned, else SPECINFER_ERR_INVALID_ARG. */
 specinfer_status_t specinfer_verify_mss(const specinfer_shape_t *shape, const float *logits,
                                         const int32_t *tree_tokens, const int32_t *parent,
                                         const int32_t *n_nodes, const float *draft_probs,
@@ -180,7 +201,7 @@ specinfer_status_t specinfer_kv_commit_paged(const specinfer_shape_t *shape, voi
  * node u on the walk draw x ~ softmax(logits[u]/temperature) by the exponential race of
  * verify_mss step 4 at round 0 (same Philox counters, so a leaf draws the same token under both
  * verifiers); if a child of u carries token x (lowest index, R7) append it and continue, else
- * emit x and stop.  Outputs, workspace and error behaviour as verify_greedy. */
+ * emit x and stop.  Outputs, workspace, alignment and error behaviour as verify_greedy. */
 specinfer_status_t specinfer_verify_ns(const specinfer_shape_t *shape, const float *logits,
                                        const int32_t *tree_tokens, const int32_t *parent,
                                        const int32_t *n_nodes, float temperature, uint64_t seed,
@@ -268,7 +289,13 @@ specinfer_status_t specinfer_sequence_pack(const specinfer_shape_t *shape, int32
 /* a6 (K6).  Depth-first KV-cache commit (L635-644): for every layer l < L, request b with
  * n = n_accepted[b] > 0 and kv-head g: slot P_b + j <- old slot P_b + accepted_nodes[b][j]
  * for j < n (bit copy of K and V rows), then prefix_len[b] += n (device, in/out).
- * k_cache_all/v_cache_all: [L] caches `layer_stride` elements apart. */
+ * k_cache_all/v_cache_all: [L] caches `layer_stride` elements apart (0 = contiguous layers),
+ * 16-byte aligned.  accepted_nodes rows have Dmax+1 entries (the verifiers' output).
+ * Path contract (always met by the verifiers' output): path[0] = 0 (the root), strictly
+ * increasing (hence path[j] >= j, which makes the in-place order safe), P_b + path[j] < Smax.
+ * A caller-built path is committed only up to its first row that breaks the contract, and
+ * n is clamped to Dmax+1: the copy and the prefix_len update use the same clamped count, so the
+ * cache stays consistent (no status is reported: kv_commit takes no workspace). */
 specinfer_status_t specinfer_kv_commit(const specinfer_shape_t *shape, void *k_cache_all,
                                        void *v_cache_all, int32_t *prefix_len,
                                        const int32_t *accepted_nodes, const int32_t *n_accepted,
@@ -284,11 +311,22 @@ specinfer_status_t specinfer_read_device_status(const void *workspace, specinfer
 specinfer_status_t specinfer_philox_debug(const uint32_t *ctr_key, uint32_t *out, int32_t n,
                                           specinfer_stream_t stream);
 
-/* Debug only: when `trace` (device, >= 8*64*8 uint64) is non-NULL, subsequent tree_attention
- * launches record per-tile clock64() timestamps of CTAs 0-7 (trace[cta][tile][event]:
- * 0/1 TMA issue of K/V, 2 S-MMA issue, 3 PV-MMA issue, 4 softmax start, 5 P ready, 6 tile
- * done).  NULL (the default) disables it.  Not thread-safe; process-global. */
+/* Development build only (libspecinfer_debug.so, compiled with -DSPECINFER_DEBUG_HOOKS by
+ * `build_lib.py --debug-hooks`; the production libspecinfer.so compiles every hook out and this
+ * call does nothing there): when `trace` (device, >= 8*64*12 + 4*1024 uint64) is non-NULL,
+ * subsequent tree_attention launches record per-tile clock64() timestamps of CTAs 0-7 and
+ * per-CTA entry / exit / first-load times; the environment variable SPECINFER_DEBUG_FLAGS is
+ * read here (pipeline experiments that invalidate results).  Not thread-safe; process-global. */
 void specinfer_debug_set_trace(void *trace);
+
+/* 1 in the development build (debug hooks compiled in), 0 in the production library. */
+int32_t specinfer_debug_hooks_enabled(void);
+
+/* Measurement only: reads `bytes` (16-byte aligned, multiple of 16) of device memory
+ * at `src` the way tree_attention streams its K/V tiles (32 KB bulk async copies into a 6-deep
+ * shared-memory ring, one CTA per SM, no compute) and discards them: the practical HBM read
+ * ceiling the attention kernel's bandwidth is compared with.  No output. */
+specinfer_status_t specinfer_hbm_read_probe(const void *src, size_t bytes, specinfer_stream_t stream);
 
 /* Number of kernel launches each call issues (for launch accounting in benchmarks). */
 int32_t specinfer_launches_per_call(const char *call_name);

@@ -52,7 +52,14 @@ def lib():
                                           dbl, u64, u64, vp, vp, vp, vp, vp,
                                           i32, vp, vp, vp, vp, vp]
         _lib.oracle_philox4x32_10.argtypes = [vp, vp, vp]
+        _lib.oracle_set_num_threads.argtypes = [i32]
+        _lib.oracle_set_num_threads.restype = None
     return _lib
+
+
+def set_num_threads(n: int) -> None:
+    """OpenMP threads of the oracle's loops (timing only; results do not depend on it)."""
+    lib().oracle_set_num_threads(int(n))
 
 
 def _p(a):

@@ -20,6 +20,9 @@ import torch
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libspecinfer.so")
+# development build with pipeline timestamps / experiment switches (build_lib.py --debug-hooks);
+# tools load it explicitly with load_library(DEBUG_LIB_PATH); tests and the bench never do
+DEBUG_LIB_PATH = os.path.join(_HERE, "libspecinfer_debug.so")
 
 SPECINFER_OK = 0
 STATUS_NAMES = {0: "OK", 1: "ERR_INVALID_ARG", 2: "ERR_UNSUPPORTED", 3: "ERR_CUDA", 4: "ERR_BAD_TREE",
@@ -33,7 +36,9 @@ EXPORTED_SYMBOLS = (
     "specinfer_status_string", "specinfer_leaf_paths", "specinfer_sequence_pack",
     "specinfer_verify_ns", "specinfer_expansion_topology", "specinfer_expand_step", "specinfer_tree_merge",
     "specinfer_tree_attention_paged", "specinfer_kv_commit_paged", "specinfer_tree_rope",
+    "specinfer_debug_hooks_enabled", "specinfer_tree_attention_ex", "specinfer_hbm_read_probe",
 )
+SPECINFER_ATTN_EARLY_PREFIX = 1
 
 
 class SpecInferError(RuntimeError):
@@ -76,6 +81,7 @@ def load_library(path: str = LIB_PATH):
     lib.specinfer_workspace_size.restype = ctypes.c_size_t
     lib.specinfer_tree_prepare.argtypes = [sp, vp, vp, vp, vp, vp, vp]
     lib.specinfer_tree_attention.argtypes = [sp, vp, vp, vp, vp, vp, vp, vp, vp, vp, vp]
+    lib.specinfer_tree_attention_ex.argtypes = [sp, vp, vp, vp, vp, vp, vp, vp, vp, vp, ctypes.c_uint32, vp]
     lib.specinfer_verify_greedy.argtypes = [sp, vp, vp, vp, vp, vp, vp, vp, vp, vp]
     lib.specinfer_verify_mss.argtypes = [sp, vp, vp, vp, vp, vp, f32, u64, u64, vp, vp, vp, vp, vp, vp]
     lib.specinfer_kv_commit.argtypes = [sp, vp, vp, vp, vp, vp, vp]
@@ -92,11 +98,16 @@ def load_library(path: str = LIB_PATH):
     lib.specinfer_sequence_pack.argtypes = [sp, i32, i32] + [vp] * 14 + [vp]
     lib.specinfer_debug_set_trace.argtypes = [vp]
     lib.specinfer_debug_set_trace.restype = None
+    lib.specinfer_hbm_read_probe.argtypes = [vp, ctypes.c_size_t, vp]
+    lib.specinfer_hbm_read_probe.restype = i32
+    lib.specinfer_debug_hooks_enabled.argtypes = []
+    lib.specinfer_debug_hooks_enabled.restype = i32
     lib.specinfer_launches_per_call.argtypes = [ctypes.c_char_p]
     lib.specinfer_launches_per_call.restype = i32
     lib.specinfer_status_string.argtypes = [i32]
     lib.specinfer_status_string.restype = ctypes.c_char_p
-    for name in ("specinfer_tree_prepare", "specinfer_tree_attention", "specinfer_verify_greedy",
+    for name in ("specinfer_tree_prepare", "specinfer_tree_attention", "specinfer_tree_attention_ex",
+                 "specinfer_verify_greedy",
                  "specinfer_verify_mss", "specinfer_kv_commit", "specinfer_read_device_status",
                  "specinfer_philox_debug", "specinfer_leaf_paths", "specinfer_sequence_pack", "specinfer_verify_ns",
                  "specinfer_expansion_topology", "specinfer_expand_step", "specinfer_tree_merge",
@@ -164,7 +175,10 @@ def specinfer_tree_prepare(shape: Shape, parent, depth, prefix_len, n_nodes, wor
 
 
 def specinfer_tree_attention(shape: Shape, q, k_cache, v_cache, parent, depth, prefix_len, n_nodes,
-                             out, workspace):
+                             out, workspace, flags: int = 0):
+    """One layer of tree attention; flags != 0 calls specinfer_tree_attention_ex (include/specinfer.h:
+    SPECINFER_ATTN_EARLY_PREFIX only when the previous kernel on the stream was not tree_prepare or
+    kv_commit of this state)."""
     dev = q.device
     B, N, Hq, Hkv, S = shape.batch, shape.max_nodes, shape.num_q_heads, shape.num_kv_heads, shape.max_seq
     qp = _req("q", q, torch.bfloat16, (B, N, Hq, 128), dev)
@@ -173,8 +187,13 @@ def specinfer_tree_attention(shape: Shape, q, k_cache, v_cache, parent, depth, p
     op = _req("out", out, torch.bfloat16, (B, N, Hq, 128), dev)
     args = _tree_args(shape, parent, depth, prefix_len, n_nodes, dev)
     ws = _req("workspace", workspace, torch.uint8, None, dev)
-    _check("specinfer_tree_attention",
-           load_library().specinfer_tree_attention(ctypes.byref(shape), qp, kp, vp, *args, op, ws, _stream(q)))
+    lib = load_library()
+    if flags:
+        _check("specinfer_tree_attention_ex",
+               lib.specinfer_tree_attention_ex(ctypes.byref(shape), qp, kp, vp, *args, op, ws, int(flags), _stream(q)))
+    else:
+        _check("specinfer_tree_attention",
+               lib.specinfer_tree_attention(ctypes.byref(shape), qp, kp, vp, *args, op, ws, _stream(q)))
 
 
 def specinfer_tree_attention_paged(shape: Shape, q, k_pages, v_pages, page_table, parent, depth, prefix_len, n_nodes,
@@ -409,6 +428,15 @@ def specinfer_debug_set_trace(trace: Optional[torch.Tensor]):
     load_library().specinfer_debug_set_trace(None if trace is None else ctypes.c_void_p(trace.data_ptr()))
 
 
+def specinfer_hbm_read_probe(buf: torch.Tensor):
+    """Streams every byte of the CUDA tensor `buf` through the library's TMA read probe (measurement)."""
+    if not isinstance(buf, torch.Tensor) or not buf.is_cuda or not buf.is_contiguous():
+        raise ValueError("specinfer_hbm_read_probe: needs a contiguous CUDA tensor")
+    nbytes = buf.numel() * buf.element_size()
+    _check("specinfer_hbm_read_probe", load_library().specinfer_hbm_read_probe(
+        ctypes.c_void_p(buf.data_ptr()), ctypes.c_size_t(nbytes), _stream(buf)))
+
+
 def specinfer_launches_per_call(name: str) -> int:
     return int(load_library().specinfer_launches_per_call(name.encode()))
 
@@ -434,9 +462,11 @@ class TreeState:
     def prepare(self):
         specinfer_tree_prepare(self.shape, self.parent, self.depth, self.prefix_len, self.n_nodes, self.workspace)
 
-    def attention(self, q, k, v, out):
+    def attention(self, q, k, v, out, prefetch: bool = False):
+        """prefetch=True: SPECINFER_ATTN_EARLY_PREFIX (the previous kernel on the stream was another
+        attention layer, not prepare / commit)."""
         specinfer_tree_attention(self.shape, q, k, v, self.parent, self.depth, self.prefix_len, self.n_nodes,
-                                 out, self.workspace)
+                                 out, self.workspace, flags=SPECINFER_ATTN_EARLY_PREFIX if prefetch else 0)
 
 
 # ------------------------------------------------------------------------------------------

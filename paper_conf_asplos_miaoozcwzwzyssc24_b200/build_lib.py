@@ -14,6 +14,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libspecinfer.so")
+DEBUG_LIB = os.path.join(HERE, "libspecinfer_debug.so")   # -DSPECINFER_DEBUG_HOOKS (tools only)
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
@@ -25,17 +26,22 @@ def sources():
     return sorted(glob.glob(os.path.join(CSRC, "*.cu")))
 
 
-def _stale() -> bool:
-    if not os.path.exists(LIB):
+def _stale(lib=LIB) -> bool:
+    if not os.path.exists(lib):
         return True
-    t = os.path.getmtime(LIB)
+    t = os.path.getmtime(lib)
     deps = sources() + glob.glob(os.path.join(CSRC, "*.cuh")) + [os.path.join(ROOT, "include", "specinfer.h")]
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def build(force: bool = False, verbose: bool = False, extra=()) -> str:
-    if not force and not _stale():
-        return LIB
+def build(force: bool = False, verbose: bool = False, extra=(), debug_hooks: bool = False) -> str:
+    """Compiles every csrc/*.cu for sm_100a and links libspecinfer.so; with debug_hooks, the
+    development variant libspecinfer_debug.so (pipeline traces, experiment switches)."""
+    target = DEBUG_LIB if debug_hooks else LIB
+    if debug_hooks:
+        extra = tuple(extra) + ("-DSPECINFER_DEBUG_HOOKS",)
+    if not force and not _stale(target):
+        return target
     with tempfile.TemporaryDirectory() as td:
         objs = []
         procs = []
@@ -57,13 +63,13 @@ def build(force: bool = False, verbose: bool = False, extra=()) -> str:
                 sys.stderr.write(f"nvcc failed on {src}\n")
         if failed:
             raise RuntimeError("libspecinfer build failed")
-        tmp = LIB + f".tmp{os.getpid()}"
+        tmp = target + f".tmp{os.getpid()}"
         subprocess.check_call([NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-lcudart_static", "-lrt", "-ldl",
                                "-lpthread"])
-        os.replace(tmp, LIB)
-    return LIB
+        os.replace(tmp, target)
+    return target
 
 
 if __name__ == "__main__":
-    build(force="--force" in sys.argv, verbose="--verbose" in sys.argv)
-    print(LIB)
+    print(build(force="--force" in sys.argv, verbose="--verbose" in sys.argv,
+                debug_hooks="--debug-hooks" in sys.argv))

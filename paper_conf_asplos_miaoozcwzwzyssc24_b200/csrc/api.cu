@@ -17,7 +17,7 @@ cudaError_t launch_tree_prepare(const specinfer_shape_t &s, const WsLayout &w, c
 cudaError_t launch_tree_attention(const specinfer_shape_t &s, const WsLayout &w, const void *q, const void *k,
                                   const void *v, const int32_t *prefix_len, const int32_t *n_nodes, void *out,
                                   char *ws, int num_sms, size_t max_smem, cudaStream_t stream,
-                                  const int32_t *page_table = nullptr, int num_pages = 0);
+                                  const int32_t *page_table = nullptr, int num_pages = 0, uint32_t flags = 0);
 cudaError_t launch_verify_greedy(const specinfer_shape_t &s, const WsLayout &w, const float *logits,
                                  const int32_t *tree_tokens, const int32_t *parent, const int32_t *n_nodes,
                                  int32_t *acc_nodes, int32_t *acc_tokens, int32_t *n_acc, char *ws,
@@ -54,9 +54,12 @@ cudaError_t launch_tree_merge(const specinfer_shape_t &s, int T, int Nin, const 
 cudaError_t launch_tree_rope(const specinfer_shape_t &s, void *q, void *k, const int32_t *prefix_len,
                              const int32_t *depth, const int32_t *n_nodes, float base, cudaStream_t stream);
 cudaError_t launch_philox_debug(const uint32_t *ck, uint32_t *out, int n, cudaStream_t stream);
+cudaError_t launch_hbm_read_probe(const void *src, size_t bytes, int num_sms, cudaStream_t stream);
+#ifdef SPECINFER_DEBUG_HOOKS
 extern unsigned long long *g_attn_trace;
 extern int g_attn_debug_flags;
 extern unsigned long long *g_mss_trace;
+#endif
 }  // namespace specinfer
 
 using namespace specinfer;
@@ -93,6 +96,16 @@ bool device_info(DeviceInfo *out) {
     return true;
 }
 
+// the workspace layout / attention schedule of a shape on this device (the debug build can switch
+// the split-KV cluster mode off: experiment flag 64)
+WsLayout layout(const specinfer_shape_t &s, int num_sms) {
+#ifdef SPECINFER_DEBUG_HOOKS
+    return ws_layout(s, num_sms, !(g_attn_debug_flags & 64));
+#else
+    return ws_layout(s, num_sms);
+#endif
+}
+
 specinfer_status_t check_shape(const specinfer_shape_t *s) {
     if (!s) return SPECINFER_ERR_INVALID_ARG;
     if (s->batch < 1 || s->max_nodes < 1 || s->num_q_heads < 1 || s->num_kv_heads < 1 || s->max_seq < 1 ||
@@ -117,6 +130,11 @@ specinfer_status_t check_ws(const void *ws) {
     return SPECINFER_OK;
 }
 
+// the verifiers read logits / draft rows with 128-bit loads: the row bases must be 16-byte aligned
+bool misaligned16(const void *a, const void *b = nullptr) {
+    return ((reinterpret_cast<uintptr_t>(a) | reinterpret_cast<uintptr_t>(b)) & 15u) != 0;
+}
+
 specinfer_status_t from_cuda(cudaError_t e) { return e == cudaSuccess ? SPECINFER_OK : SPECINFER_ERR_CUDA; }
 
 #define SPI_TRY(x)                                 \
@@ -133,7 +151,7 @@ size_t specinfer_workspace_size(const specinfer_shape_t *shape) {
     if (check_shape(shape) != SPECINFER_OK) return 0;
     DeviceInfo d;
     const int sms = device_info(&d) ? d.num_sms : 148;
-    return ws_layout(*shape, sms > 0 ? sms : 148).total;
+    return layout(*shape, sms > 0 ? sms : 148).total;
 }
 
 specinfer_status_t specinfer_tree_prepare(const specinfer_shape_t *shape, const int32_t *parent,
@@ -144,29 +162,38 @@ specinfer_status_t specinfer_tree_prepare(const specinfer_shape_t *shape, const 
     SPI_TRY(check_ws(workspace));
     DeviceInfo d;
     SPI_TRY(check_device(&d));
-    const WsLayout w = ws_layout(*shape, d.num_sms);
+    const WsLayout w = layout(*shape, d.num_sms);
     return from_cuda(launch_tree_prepare(*shape, w, parent, depth, prefix_len, n_nodes,
                                          reinterpret_cast<char *>(workspace), w.grid,
                                          (cudaStream_t)stream));
 }
 
-specinfer_status_t specinfer_tree_attention(const specinfer_shape_t *shape, const void *q, const void *k_cache,
-                                            const void *v_cache, const int32_t *parent, const int32_t *depth,
-                                            const int32_t *prefix_len, const int32_t *n_nodes, void *out,
-                                            void *workspace, specinfer_stream_t stream) {
+specinfer_status_t specinfer_tree_attention_ex(const specinfer_shape_t *shape, const void *q, const void *k_cache,
+                                               const void *v_cache, const int32_t *parent, const int32_t *depth,
+                                               const int32_t *prefix_len, const int32_t *n_nodes, void *out,
+                                               void *workspace, uint32_t flags, specinfer_stream_t stream) {
     SPI_TRY(check_shape(shape));
     if (!q || !k_cache || !v_cache || !parent || !depth || !prefix_len || !n_nodes || !out)
         return SPECINFER_ERR_INVALID_ARG;
     if ((reinterpret_cast<uintptr_t>(q) | reinterpret_cast<uintptr_t>(k_cache) |
          reinterpret_cast<uintptr_t>(v_cache) | reinterpret_cast<uintptr_t>(out)) & 15u)
         return SPECINFER_ERR_INVALID_ARG;
+    if (flags & ~(uint32_t)SPECINFER_ATTN_EARLY_PREFIX) return SPECINFER_ERR_INVALID_ARG;
     SPI_TRY(check_ws(workspace));
     DeviceInfo d;
     SPI_TRY(check_device(&d));
-    const WsLayout w = ws_layout(*shape, d.num_sms);
+    const WsLayout w = layout(*shape, d.num_sms);
     return from_cuda(launch_tree_attention(*shape, w, q, k_cache, v_cache, prefix_len, n_nodes, out,
                                            reinterpret_cast<char *>(workspace), w.grid, d.max_smem,
-                                           (cudaStream_t)stream));
+                                           (cudaStream_t)stream, nullptr, 0, flags));
+}
+
+specinfer_status_t specinfer_tree_attention(const specinfer_shape_t *shape, const void *q, const void *k_cache,
+                                            const void *v_cache, const int32_t *parent, const int32_t *depth,
+                                            const int32_t *prefix_len, const int32_t *n_nodes, void *out,
+                                            void *workspace, specinfer_stream_t stream) {
+    return specinfer_tree_attention_ex(shape, q, k_cache, v_cache, parent, depth, prefix_len, n_nodes, out, workspace,
+                                       0u, stream);
 }
 
 specinfer_status_t specinfer_tree_attention_paged(const specinfer_shape_t *shape, const void *q, const void *k_pages,
@@ -185,7 +212,7 @@ specinfer_status_t specinfer_tree_attention_paged(const specinfer_shape_t *shape
     SPI_TRY(check_ws(workspace));
     DeviceInfo d;
     SPI_TRY(check_device(&d));
-    const WsLayout w = ws_layout(*shape, d.num_sms);
+    const WsLayout w = layout(*shape, d.num_sms);
     return from_cuda(launch_tree_attention(*shape, w, q, k_pages, v_pages, prefix_len, n_nodes, out,
                                            reinterpret_cast<char *>(workspace), w.grid, d.max_smem,
                                            (cudaStream_t)stream, page_table, num_pages));
@@ -226,10 +253,11 @@ specinfer_status_t specinfer_verify_greedy(const specinfer_shape_t *shape, const
     if (shape->vocab < 1) return SPECINFER_ERR_INVALID_ARG;
     if (!logits || !tree_tokens || !parent || !n_nodes || !accepted_nodes || !accepted_tokens || !n_accepted)
         return SPECINFER_ERR_INVALID_ARG;
+    if (misaligned16(logits)) return SPECINFER_ERR_INVALID_ARG;
     SPI_TRY(check_ws(workspace));
     DeviceInfo d;
     SPI_TRY(check_device(&d));
-    const WsLayout w = ws_layout(*shape, d.num_sms);
+    const WsLayout w = layout(*shape, d.num_sms);
     return from_cuda(launch_verify_greedy(*shape, w, logits, tree_tokens, parent, n_nodes, accepted_nodes,
                                           accepted_tokens, n_accepted, reinterpret_cast<char *>(workspace),
                                           (cudaStream_t)stream));
@@ -246,10 +274,11 @@ specinfer_status_t specinfer_verify_mss(const specinfer_shape_t *shape, const fl
     if (!logits || !tree_tokens || !parent || !n_nodes || !draft_probs || !accepted_nodes || !accepted_tokens ||
         !n_accepted)
         return SPECINFER_ERR_INVALID_ARG;
+    if (misaligned16(logits, draft_probs)) return SPECINFER_ERR_INVALID_ARG;
     SPI_TRY(check_ws(workspace));
     DeviceInfo d;
     SPI_TRY(check_device(&d));
-    const WsLayout w = ws_layout(*shape, d.num_sms);
+    const WsLayout w = layout(*shape, d.num_sms);
     return from_cuda(launch_verify_mss(*shape, w, logits, tree_tokens, parent, n_nodes, draft_probs, temperature,
                                        seed, offset, request_ids, accepted_nodes, accepted_tokens, n_accepted,
                                        reinterpret_cast<char *>(workspace), (cudaStream_t)stream));
@@ -265,10 +294,11 @@ specinfer_status_t specinfer_verify_ns(const specinfer_shape_t *shape, const flo
     if (shape->vocab < 1 || !(temperature > 0.f) || !isfinite(temperature)) return SPECINFER_ERR_INVALID_ARG;
     if (!logits || !tree_tokens || !parent || !n_nodes || !accepted_nodes || !accepted_tokens || !n_accepted)
         return SPECINFER_ERR_INVALID_ARG;
+    if (misaligned16(logits)) return SPECINFER_ERR_INVALID_ARG;
     SPI_TRY(check_ws(workspace));
     DeviceInfo d;
     SPI_TRY(check_device(&d));
-    const WsLayout w = ws_layout(*shape, d.num_sms);
+    const WsLayout w = layout(*shape, d.num_sms);
     return from_cuda(launch_verify_ns(*shape, w, logits, tree_tokens, parent, n_nodes, temperature, seed, offset,
                                       request_ids, accepted_nodes, accepted_tokens, n_accepted,
                                       reinterpret_cast<char *>(workspace), (cudaStream_t)stream));
@@ -394,19 +424,41 @@ specinfer_status_t specinfer_philox_debug(const uint32_t *ctr_key, uint32_t *out
     return from_cuda(launch_philox_debug(ctr_key, out, n, (cudaStream_t)stream));
 }
 
+specinfer_status_t specinfer_hbm_read_probe(const void *src, size_t bytes, specinfer_stream_t stream) {
+    if (bytes > 0 && !src) return SPECINFER_ERR_INVALID_ARG;
+    if ((reinterpret_cast<uintptr_t>(src) | bytes) & 15u) return SPECINFER_ERR_INVALID_ARG;
+    DeviceInfo d;
+    SPI_TRY(check_device(&d));
+    return from_cuda(launch_hbm_read_probe(src, bytes, d.num_sms, (cudaStream_t)stream));
+}
+
 void specinfer_debug_set_trace(void *trace) {
+#ifdef SPECINFER_DEBUG_HOOKS
+    // development build only (libspecinfer_debug.so): pipeline timestamps and experiment switches
+    // (flags 1/2/4/8 make results invalid); the production library compiles all of it out
     g_attn_trace = reinterpret_cast<unsigned long long *>(trace);
     g_mss_trace = getenv("SPECINFER_TRACE_MSS") ? reinterpret_cast<unsigned long long *>(trace) : nullptr;
     if (g_mss_trace) g_attn_trace = nullptr;
-    // experiment switches for pipeline studies (results invalid when set); never set in production
     const char *f = getenv("SPECINFER_DEBUG_FLAGS");
     g_attn_debug_flags = f ? atoi(f) : 0;
+#else
+    (void)trace;
+#endif
+}
+
+int32_t specinfer_debug_hooks_enabled(void) {
+#ifdef SPECINFER_DEBUG_HOOKS
+    return 1;
+#else
+    return 0;
+#endif
 }
 
 int32_t specinfer_launches_per_call(const char *name) {
     if (!name) return -1;
     if (!strcmp(name, "tree_prepare")) return 2;     // validate+bitsets, schedule (+1 memset)
     if (!strcmp(name, "tree_attention")) return 1;   // split combine fused (last piece merges)
+    if (!strcmp(name, "tree_attention_ex")) return 1;
     if (!strcmp(name, "verify_greedy")) return 1;    // argmax + walk fused (last CTA walks)
     if (!strcmp(name, "verify_mss")) return 1;
     if (!strcmp(name, "kv_commit")) return 2;        // copy, prefix update
@@ -419,6 +471,7 @@ int32_t specinfer_launches_per_call(const char *name) {
     if (!strcmp(name, "tree_merge")) return 1;         // race-argmax + walk fused (last CTA walks)
     if (!strcmp(name, "sequence_pack")) return 1;
     if (!strcmp(name, "tree_rope")) return 1;
+    if (!strcmp(name, "hbm_read_probe")) return 1;
     return -1;
 }
 

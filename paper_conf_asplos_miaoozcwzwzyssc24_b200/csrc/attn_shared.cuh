@@ -3,6 +3,8 @@
 // kernel for wider trees / GQA groups): launch parameters, schedule helpers, TMA helpers,
 // tensor-map encoding, debug tracing.
 #pragma once
+#include <atomic>
+
 #include "common.cuh"
 
 namespace specinfer {
@@ -21,6 +23,8 @@ struct AttnParams {
     __nv_bfloat16 *out;
     int B, Nmax, Hq, Hkv, G, Smax, chunks, npc, n_items, nk_slots, nv_slots;
     int splitk;  // > 1: split-KV mode (cluster of splitk CTAs per item, DSMEM merge)
+    int early_prefix;  // SPECINFER_ATTN_EARLY_PREFIX: the producers read the schedule and stage the
+                       // first committed-prefix tiles before the programmatic dependency resolves
     int lanes;  // CTAs per lock-step group (schedule_kernel); 1 = plain stream-K over items
     // paged KV (NEXT-4): page_table[b][t] = page holding keys [128 t, 128 t + 128) of request b;
     // a page is [Hkv][128][128] bf16.  nullptr = contiguous [B][Hkv][Smax][128] caches.
@@ -31,22 +35,34 @@ struct AttnParams {
     int debug_flags;            // experiments only: 1 = skip K/V TMA, 2 = skip MMAs (results invalid)
 };
 
+// Debug hooks (pipeline timestamps, experiment switches) exist only in a library built with
+// -DSPECINFER_DEBUG_HOOKS (build_lib.py --debug-hooks -> libspecinfer_debug.so, development tools);
+// the production build compiles them out: no trace stores, every experiment branch constant-false.
+#ifdef SPECINFER_DEBUG_HOOKS
+#define SPI_FLAGS(p) ((p).debug_flags)
+#define SPI_TRACING(p) ((p).trace != nullptr)
+#else
+#define SPI_FLAGS(p) 0
+#define SPI_TRACING(p) false
+#endif
+
 // debug timestamps: trace[cta][tile][event], CTAs < kTraceCtas, tiles < kTraceTiles
-constexpr int kTraceCtas = 8, kTraceTiles = 64, kTraceEv = 12;
+constexpr int kTraceCtas = 8, kTraceTiles = 64, kTraceEv = 16;
 __device__ __forceinline__ unsigned long long globaltimer_ns() {
     unsigned long long t;
     asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
     return t;
 }
-// kernel-level timestamps of every CTA (ns): [entry, exit, first K issue, 0]
+// kernel-level timestamps of every CTA (ns), 8 slots: 0 entry, 1 exit, 2 first K issue, 3 split-KV
+// cluster barrier, 4 prologue done, 5 dependency wait passed, 6 schedule read, 7 first S ready
 #define SPI_TRACE_K(slot)                                                                                  \
     do {                                                                                                   \
-        if (p.trace != nullptr)                                                                            \
-            p.trace[(size_t)kTraceCtas * kTraceTiles * kTraceEv + blockIdx.x * 4 + (slot)] = globaltimer_ns(); \
+        if (SPI_TRACING(p))                                                                                \
+            p.trace[(size_t)kTraceCtas * kTraceTiles * kTraceEv + blockIdx.x * 8 + (slot)] = globaltimer_ns(); \
     } while (0)
 #define SPI_TRACE(ev)                                                                               \
     do {                                                                                            \
-        if (p.trace != nullptr && blockIdx.x < kTraceCtas && lt < kTraceTiles)                      \
+        if (SPI_TRACING(p) && blockIdx.x < kTraceCtas && lt < kTraceTiles)                          \
             p.trace[((size_t)blockIdx.x * kTraceTiles + lt) * kTraceEv + (ev)] = clock64();         \
     } while (0)
 
@@ -146,6 +162,21 @@ static PFN_encodeTiled_t get_encode_fn() {
             fn = reinterpret_cast<PFN_encodeTiled_t>(ptr);
     }
     return fn;
+}
+
+// cudaFuncAttributeMaxDynamicSharedMemorySize is per device (context): one bit per attention kernel
+// variant and device, set once (part of the per-device capability cache, include/specinfer.h).
+// Racing first calls both set the attribute, which is idempotent.
+inline cudaError_t ensure_max_smem_attr(const void *func, int variant, size_t max_smem) {
+    static std::atomic<uint32_t> done[64];
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    const uint32_t bit = 1u << variant;
+    if (dev >= 0 && dev < 64 && (done[dev].load(std::memory_order_acquire) & bit)) return cudaSuccess;
+    e = cudaFuncSetAttribute(func, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)max_smem);
+    if (e == cudaSuccess && dev >= 0 && dev < 64) done[dev].fetch_or(bit, std::memory_order_acq_rel);
+    return e;
 }
 
 static bool encode_2d(CUtensorMap *m, const void *base, uint64_t rows, uint32_t box_rows) {

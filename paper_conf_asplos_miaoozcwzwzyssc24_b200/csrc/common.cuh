@@ -64,7 +64,7 @@ inline int choose_nt(int G, int nmax) {
     return kRowsBlock;
 }
 
-inline WsLayout ws_layout(const specinfer_shape_t &s, int num_sms) {
+inline WsLayout ws_layout(const specinfer_shape_t &s, int num_sms, bool allow_split_kv = true) {
     WsLayout w{};
     const int B = s.batch, N = s.max_nodes;
     const int G = s.num_q_heads / s.num_kv_heads;
@@ -79,7 +79,7 @@ inline WsLayout ws_layout(const specinfer_shape_t &s, int num_sms) {
     w.splitk = 1;
     // (only when an item can span enough 128-key tiles for the split to pay for the cluster merge:
     // the schedule keeps items shorter than 12 tiles whole on rank 0)
-    if (w.nt != kRowsBlock && w.lanes == 1 && (s.max_seq + 127) / 128 >= 12) {
+    if (allow_split_kv && w.nt != kRowsBlock && w.lanes == 1 && (s.max_seq + 127) / 128 >= 12) {
         int k = 1;
         // rank 0 gathers the k partials ([nt][128] + 2 [nt] floats each) in its K/V rings (>= 160 KB)
         const int kmax = w.nt == 64 ? 4 : 8;

@@ -253,32 +253,38 @@ __global__ void __launch_bounds__(128) tree_merge_kernel(int T, int Nin, const i
         s_bad = bad;
     }
     __syncthreads();
+    // depths (and the Dmax check) BEFORE any output is written: a merged tree deeper than Dmax is
+    // reported like every other bad input (n_nodes 0, padding rows, node_map -1).  s_stack is free.
     const int nm = s_n;
+    for (int u = threadIdx.x; u < nm; u += blockDim.x) {
+        int dep = 0;
+        for (int x = s_par[u]; x >= 0; x = s_par[x]) ++dep;
+        s_stack[u] = dep;
+        if (dep > Dmax) atomicOr(&s_bad, 1);
+    }
+    __syncthreads();
+    const int nw = s_bad ? 0 : nm;
     for (int i = threadIdx.x; i < Nmax; i += blockDim.x) {
         parent[(size_t)b * Nmax + i] = -1;
         depth[(size_t)b * Nmax + i] = 0;
         tokens[(size_t)b * Nmax + i] = -1;
     }
     __syncthreads();
-    for (int u = threadIdx.x; u < nm; u += blockDim.x) {
+    for (int u = threadIdx.x; u < nw; u += blockDim.x) {
         const int d = s_dfs[u];
-        int dep = 0;
-        for (int x = s_par[u]; x >= 0; x = s_par[x]) ++dep;
-        if (dep > Dmax) atomicOr(&s_bad, 1);
         parent[(size_t)b * Nmax + d] = s_par[u] >= 0 ? s_dfs[s_par[u]] : -1;
-        depth[(size_t)b * Nmax + d] = dep;
+        depth[(size_t)b * Nmax + d] = s_stack[u];
         tokens[(size_t)b * Nmax + d] = s_tok[u];
     }
     // node_map: trie ids -> DFS ids
     for (int idx = threadIdx.x; idx < T * Nin; idx += blockDim.x) {
         int32_t *m = node_map + (size_t)b * T * Nin + idx;
         const int v = *m;
-        if (!s_n) *m = -1;
+        if (!nw) *m = -1;
         else if (v >= 0) *m = s_dfs[v];
     }
-    __syncthreads();
     if (threadIdx.x == 0) {
-        n_nodes[b] = s_bad ? 0 : nm;
+        n_nodes[b] = nw;
         if (s_bad && status) atomicOr(status, kStatusBadTree);
     }
 }

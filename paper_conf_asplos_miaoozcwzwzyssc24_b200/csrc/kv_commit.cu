@@ -13,6 +13,23 @@
 
 namespace specinfer {
 
+// Number of path rows of request b that can be committed: n_acc clamped to the path row length,
+// then to the longest prefix of the path that is a valid DFS commit (path[0] = 0, strictly
+// increasing, so path[j] >= j, and P + path[j] < Smax).  The verifiers always produce valid paths;
+// a caller-built path that breaks the contract is committed only up to its first bad row, by the
+// copy and the prefix update alike (include/specinfer.h).
+__device__ __forceinline__ int commit_len(const int32_t *path, int n, int P, int Smax, int path_len) {
+    n = min(n, path_len);
+    if (n <= 0) return 0;
+    if (path[0] != 0 || P >= Smax) return 0;
+    int j = 1;
+    for (; j < n; ++j) {
+        const int src = path[j];
+        if (src <= path[j - 1] || P + src >= Smax) break;
+    }
+    return j;
+}
+
 // paged KV (NEXT-4): slot s of request b, kv-head g lives at row (page_table[b][s/128] Hkv + g) 128
 // + s % 128 of the layer's [num_pages][Hkv][128][128] pages; page_table == nullptr: contiguous.
 __global__ void __launch_bounds__(256) kv_commit_copy_kernel(
@@ -25,9 +42,10 @@ __global__ void __launch_bounds__(256) kv_commit_copy_kernel(
     const int g = (int)(item % Hkv);
     const int b = (int)((item / Hkv) % B);
     const int l = (int)(item / ((long long)Hkv * B));
-    const int n = n_acc[b];
-    if (n <= 1) return;
     const int P = prefix_len[b];
+    const int32_t *path = acc_nodes + (size_t)b * path_len;
+    const int n = commit_len(path, n_acc[b], P, Smax, path_len);
+    if (n <= 1) return;
     __nv_bfloat16 *layer = (lane < 16 ? k_all : v_all) + (size_t)l * layer_stride;
     const int col = (lane & 15) * 8;  // 8 bf16 = 16 bytes
     auto row = [&](int slot) -> __nv_bfloat16 * {
@@ -35,7 +53,6 @@ __global__ void __launch_bounds__(256) kv_commit_copy_kernel(
         const int page = page_table[(size_t)b * max_pages + slot / kKeyTile];
         return layer + (((size_t)page * Hkv + g) * kKeyTile + slot % kKeyTile) * kHeadDim + col;
     };
-    const int32_t *path = acc_nodes + (size_t)b * path_len;
     for (int j = 1; j < n; ++j) {
         const int src = path[j];
         if (src == j) continue;
@@ -44,9 +61,10 @@ __global__ void __launch_bounds__(256) kv_commit_copy_kernel(
     }
 }
 
-__global__ void kv_commit_prefix_kernel(int32_t *__restrict__ prefix_len, const int32_t *__restrict__ n_acc, int B) {
+__global__ void kv_commit_prefix_kernel(int32_t *__restrict__ prefix_len, const int32_t *__restrict__ acc_nodes,
+                                        const int32_t *__restrict__ n_acc, int B, int Smax, int path_len) {
     const int b = blockIdx.x * blockDim.x + threadIdx.x;
-    if (b < B && n_acc[b] > 0) prefix_len[b] += n_acc[b];
+    if (b < B) prefix_len[b] += commit_len(acc_nodes + (size_t)b * path_len, n_acc[b], prefix_len[b], Smax, path_len);
 }
 
 cudaError_t launch_kv_commit(const specinfer_shape_t &s, void *k_all, void *v_all, int32_t *prefix_len,
@@ -68,7 +86,8 @@ cudaError_t launch_kv_commit(const specinfer_shape_t &s, void *k_all, void *v_al
         cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return e;
     }
-    kv_commit_prefix_kernel<<<(s.batch + 255) / 256, 256, 0, stream>>>(prefix_len, n_acc, s.batch);
+    kv_commit_prefix_kernel<<<(s.batch + 255) / 256, 256, 0, stream>>>(prefix_len, acc_nodes, n_acc, s.batch,
+                                                                       s.max_seq, s.max_depth + 1);
     return cudaGetLastError();
 }
 

@@ -35,6 +35,7 @@ namespace specinfer {
 template <int NT>
 struct SmemPlan {
     static constexpr int kQBuf = 2 * NT * 128;         // one Q buffer: 2 halves x NT rows x 128 B
+    static constexpr int kNQ = 2;                      // Q buffers (segment s uses s % kNQ)
     static constexpr int kPBuf = kKeyTile * NT * 2;    // one P^T buffer: 128 keys x NT bf16
     // P^T buffers: two (softmax(t) overlaps PV(t-1)) except at NT = 64, where the second 16 KB
     // would cost a K/V ring slot (measured: width-5 C2 tree 1% slower with two)
@@ -88,7 +89,7 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
     uint8_t *s_k = smem;
     uint8_t *s_v = s_k + (size_t)NK * kSlotBytes;
     uint8_t *s_q = s_v + (size_t)NV * kSlotBytes;
-    uint8_t *s_p = s_q + 2 * Plan::kQBuf;
+    uint8_t *s_p = s_q + Plan::kNQ * Plan::kQBuf;
     SmemMisc *misc = reinterpret_cast<SmemMisc *>(s_p + Plan::kNP * Plan::kPBuf);
 
     const int warp = threadIdx.x >> 5;
@@ -132,7 +133,7 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
     }
     if (warp >= 3) {
         // Q rows beyond a chunk's G*npc rows are never written by TMA: keep them zero
-        for (int i = threadIdx.x - 96; i < 2 * Plan::kQBuf / 16; i += kSoft)
+        for (int i = threadIdx.x - 96; i < Plan::kNQ * Plan::kQBuf / 16; i += kSoft)
             reinterpret_cast<uint4 *>(s_q)[i] = make_uint4(0, 0, 0, 0);
         // V rows past a request's last key are never loaded: they must hold finite data (0 * NaN)
         for (int i = threadIdx.x - 96; i < NV * kSlotBytes / 16; i += kSoft)
@@ -145,25 +146,71 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
     tc_fence_after();
     const uint32_t tmem = misc->tmem_base;
     const uint32_t tm_S0 = tmem, tm_O = tmem + 2 * NT;
+    if (threadIdx.x == 0) SPI_TRACE_K(4);
 
     // Programmatic dependent launch: everything above overlapped the previous kernel's tail;
-    // from here on we read inputs it may have produced.
-    grid_dependency_wait();
+    // from here on we read inputs it may have produced.  With early_prefix (the caller guarantees
+    // that neither the committed prefix of the caches nor the schedule in the workspace was written
+    // by the immediately preceding kernel), the two producer lanes first stage the committed-prefix
+    // tiles of their first segment and only then wait; every other warp waits here.
+    // (the whole producer warp skips this wait: a wait on lanes 2-31 alone would hold lanes 0-1 at the
+    // warp's reconvergence point; lanes 0-1 wait after staging, lanes 2-31 read nothing)
+    const bool early = p.early_prefix != 0 && warp == 0;
+    if (!early) grid_dependency_wait();
+    if (threadIdx.x == 0) SPI_TRACE_K(5);
     // this CTA's slice of the tile sequence (precomputed by tree_prepare for this grid)
     const int4 ci = __ldg(p.cta_info + 2 * blockIdx.x);
     const int4 first_info = __ldg(p.cta_info + 2 * blockIdx.x + 1);
     const int t0 = ci.x, t1 = ci.y, x_first = ci.z, T = ci.w;
     const int ntiles = t1 - t0;
+    if (threadIdx.x == 0 && ntiles > -1000000) SPI_TRACE_K(6);
 
     if (ntiles <= 0) {
         // no work for this CTA (fewer tiles than CTAs)
+        if (early) grid_dependency_wait();
     } else if (warp == 0) {
         // ============================ TMA producers ============================
         const uint64_t pol = l2_evict_first_policy();
+        // one K (lane 0) or V (lane 1) tile of segment d into ring slot lt % NS
+        auto issue = [&](const SegDesc &d, int t, int lt, bool is_v) {
+            const int key0 = (t - d.ib) * kKeyTile;
+            const int nv = min(kKeyTile, d.P + d.n - key0);
+            const int row0 = kv_tile_row(p, d.b, d.g, key0);
+            const int NS = is_v ? NV : NK;
+            const int slot = lt % NS, f = lt / NS;
+            if (f >= 1) mbar_wait(is_v ? &misc->v_empty[slot] : &misc->k_empty[slot], (f - 1) & 1);
+            if (!is_v) {
+                SPI_TRACE(0);
+                if (lt == 0) SPI_TRACE_K(2);
+            } else {
+                SPI_TRACE(1);
+            }
+            uint8_t *dst = (is_v ? s_v : s_k) + (size_t)slot * kSlotBytes;
+            uint64_t *bar = is_v ? &misc->v_full[slot] : &misc->k_full[slot];
+            const CUtensorMap *m = is_v ? &tm_v : &tm_k;
+            if (SPI_FLAGS(p) & 1) {
+                mbar_arrive(bar);
+            } else if (nv == kKeyTile) {
+                mbar_arrive_expect_tx(bar, kSlotBytes);
+                tma_load_2d(dst, m, bar, 0, row0, pol);
+                tma_load_2d(dst + kHalfBytes, m, bar, 64, row0, pol);
+            } else if (is_v) {
+                tma_load_rows(dst, bar, nv, row0, pol, &tm_v16, &tm_v4, &tm_v1);
+            } else {
+                tma_load_rows(dst, bar, nv, row0, pol, &tm_k16, &tm_k4, &tm_k1);
+            }
+        };
+        // committed-prefix tiles of the first segment that fit the free ring slots (early mode)
+        auto n_early = [&](const SegDesc &d, int NS) {
+            int c = 0;
+            while (c < NS && d.begin + c < d.end && (d.begin + c - d.ib + 1) * kKeyTile <= d.P) ++c;
+            return c;
+        };
         if (lane == 0) {
             // segment descriptors for every role, Q, and the K tiles
             int lt = 0, ls = 0;
             int4 next_info = first_info;
+            SPI_TRACE(12);
             for (int x = x_first; lt < ntiles; ++x) {
                 const int4 info = next_info;  // {first tile, end tile, P, n}
                 next_info = __ldg(p.item_info + x + 1);  // prefetched a segment ahead (sentinel-safe)
@@ -181,35 +228,24 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
                 d.P = info.z;
                 d.n = info.w;
                 misc->seg[ls % kSegRing] = d;
+                if (ls == 0) SPI_TRACE(13);
                 mbar_arrive(&misc->seg_full[ls % kSegRing]);  // release: descriptor visible
-                const int Kend = d.P + d.n;
-                const int qb = ls & 1;
-                if (ls >= 2) mbar_wait(&misc->q_empty[qb], ((ls >> 1) - 1) & 1);
+                int pre = 0;
+                if (early && ls == 0) {
+                    pre = n_early(d, NK);
+                    for (int i = 0; i < pre; ++i) issue(d, d.begin + i, i, false);
+                    grid_dependency_wait();   // q, tree keys and everything else: after the dependency
+                }
+                const int qb = ls % Plan::kNQ;
+                if (ls >= Plan::kNQ) mbar_wait(&misc->q_empty[qb], ((ls / Plan::kNQ) - 1) & 1);
                 mbar_arrive_expect_tx(&misc->q_full[qb], 2u * (uint32_t)(p.G * p.npc) * 128u);
                 uint8_t *qdst = s_q + qb * Plan::kQBuf;
                 const int node0 = d.b * p.Nmax + d.c * p.npc;
                 tma_load_3d(qdst, &tm_q, &misc->q_full[qb], 0, d.g * p.G, node0);
                 tma_load_3d(qdst + NT * 128, &tm_q, &misc->q_full[qb], 64, d.g * p.G, node0);
-                for (int t = d.begin; t < d.end; ++t, ++lt) {
-                    const int key0 = (t - d.ib) * kKeyTile;
-                    const int nv = min(kKeyTile, Kend - key0);
-                    const int row0 = kv_tile_row(p, d.b, d.g, key0);
-                    const int slot = lt % NK, f = lt / NK;
-                    if (f >= 1) mbar_wait(&misc->k_empty[slot], (f - 1) & 1);
-                    SPI_TRACE(0);
-                    if (lt == 0) SPI_TRACE_K(2);
-                    uint8_t *dst = s_k + (size_t)slot * kSlotBytes;
-                    uint64_t *bar = &misc->k_full[slot];
-                    if (p.debug_flags & 1) {
-                        mbar_arrive(bar);
-                    } else if (nv == kKeyTile) {
-                        mbar_arrive_expect_tx(bar, kSlotBytes);
-                        tma_load_2d(dst, &tm_k, bar, 0, row0, pol);
-                        tma_load_2d(dst + kHalfBytes, &tm_k, bar, 64, row0, pol);
-                    } else {
-                        tma_load_rows(dst, bar, nv, row0, pol, &tm_k16, &tm_k4, &tm_k1);
-                    }
-                }
+                if (ls == 0) SPI_TRACE(14);
+                lt += pre;
+                for (int t = d.begin + pre; t < d.end; ++t, ++lt) issue(d, t, lt, false);
                 ++ls;
             }
             grid_launch_dependents();  // all of this CTA's K loads are issued
@@ -219,26 +255,14 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
             while (lt < ntiles) {
                 mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
                 const SegDesc d = misc->seg[ls % kSegRing];
-                const int Kend = d.P + d.n;
-                for (int t = d.begin; t < d.end; ++t, ++lt) {
-                    const int key0 = (t - d.ib) * kKeyTile;
-                    const int nv = min(kKeyTile, Kend - key0);
-                    const int row0 = kv_tile_row(p, d.b, d.g, key0);
-                    const int slot = lt % NV, f = lt / NV;
-                    if (f >= 1) mbar_wait(&misc->v_empty[slot], (f - 1) & 1);
-                    SPI_TRACE(1);
-                    uint8_t *dst = s_v + (size_t)slot * kSlotBytes;
-                    uint64_t *bar = &misc->v_full[slot];
-                    if (p.debug_flags & 1) {
-                        mbar_arrive(bar);
-                    } else if (nv == kKeyTile) {
-                        mbar_arrive_expect_tx(bar, kSlotBytes);
-                        tma_load_2d(dst, &tm_v, bar, 0, row0, pol);
-                        tma_load_2d(dst + kHalfBytes, &tm_v, bar, 64, row0, pol);
-                    } else {
-                        tma_load_rows(dst, bar, nv, row0, pol, &tm_v16, &tm_v4, &tm_v1);
-                    }
+                int pre = 0;
+                if (early && ls == 0) {
+                    pre = n_early(d, NV);
+                    for (int i = 0; i < pre; ++i) issue(d, d.begin + i, i, true);
+                    grid_dependency_wait();
                 }
+                lt += pre;
+                for (int t = d.begin + pre; t < d.end; ++t, ++lt) issue(d, t, lt, true);
                 ++ls;
             }
         }
@@ -252,8 +276,8 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
             while (lt < ntiles) {
                 mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
                 const SegDesc d = misc->seg[ls % kSegRing];
-                const int qb = ls & 1;
-                mbar_wait(&misc->q_full[qb], (ls >> 1) & 1);
+                const int qb = ls % Plan::kNQ;
+                mbar_wait(&misc->q_full[qb], (ls / Plan::kNQ) & 1);
                 for (int t = d.begin; t < d.end; ++t, ++lt) {
                     const int slot = lt % NK;
                     mbar_wait(&misc->k_full[slot], (lt / NK) & 1);
@@ -269,7 +293,7 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
                         const uint32_t qoff = (kk >> 2) * (NT * 128) + (kk & 3) * 32;
                         const uint64_t adesc = make_smem_desc(kbase + koff, 16, 1024, kSw128);
                         const uint64_t bdesc = make_smem_desc(qbase + qoff, 16, 1024, kSw128);
-                        if (!(p.debug_flags & 2)) umma_bf16_ss(tm_S0 + sb * NT, adesc, bdesc, idesc_s, kk > 0 ? 1u : 0u);
+                        if (!(SPI_FLAGS(p) & 2)) umma_bf16_ss(tm_S0 + sb * NT, adesc, bdesc, idesc_s, kk > 0 ? 1u : 0u);
                     }
                     umma_commit(&misc->s_full[sb]);
                     umma_commit(&misc->k_empty[slot]);
@@ -300,7 +324,7 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
                         const uint64_t adesc = make_smem_desc(vbase + kk * 16 * 128, kHalfBytes, 1024, kSw128);
                         const uint64_t bdesc = make_smem_desc(p_addr + (lt % Plan::kNP) * Plan::kPBuf + kk * 16 * (NT * 2), Plan::kPBuf,
                                                               8 * NT * 2, Plan::kPSwizzle);
-                        if (!(p.debug_flags & 2)) umma_bf16_ss(tm_O, adesc, bdesc, idesc_o, (first && kk == 0) ? 0u : 1u);
+                        if (!(SPI_FLAGS(p) & 2)) umma_bf16_ss(tm_O, adesc, bdesc, idesc_o, (first && kk == 0) ? 0u : 1u);
                     }
                     umma_commit(&misc->p_empty[lt % Plan::kNP]);
                     umma_commit(&misc->v_empty[slot]);
@@ -357,6 +381,7 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
                 mbar_wait(&misc->s_full[sb], (lt >> 1) & 1);
                 tc_fence_after();
                 if (st == 0) SPI_TRACE(4);
+                if (st == 0 && lt == 0) SPI_TRACE_K(7);
                 float xv[NTH];
                 {
                     uint32_t r16[NTH / 16][16];
@@ -585,7 +610,7 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
                             __threadfence();
 // merge-phase trace points go to the (unused) row of tile lt + 1: 0 start, 1 pieces issued,
 // 2 staged, 3 weights, 4 accumulated, 5 stored
-#define SPI_TRACE2(ev) do { if (st == 0 && p.trace != nullptr && blockIdx.x < kTraceCtas && lt + 1 < kTraceTiles) \
+#define SPI_TRACE2(ev) do { if (st == 0 && SPI_TRACING(p) && blockIdx.x < kTraceCtas && lt + 1 < kTraceTiles) \
     p.trace[((size_t)blockIdx.x * kTraceTiles + lt + 1) * kTraceEv + (ev)] = clock64(); } while (0)
                             SPI_TRACE2(0);
                             float acc[NTH];
@@ -599,7 +624,7 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
                             float *so = reinterpret_cast<float *>(s_k);
                             if (st == 0) {
                                 int npcs = -1;
-                                if (sd.end == t1 && !(p.debug_flags & 32)) {  // no tile follows: rings idle (32: test the fallback)
+                                if (sd.end == t1 && !(SPI_FLAGS(p) & 32)) {  // no tile follows: rings idle (32: test the fallback)
                                     npcs = 0;
                                     const int cf = cta_of_tile(sd.ib, T, NC), cl2 = cta_of_tile(sd.ie - 1, T, NC);
                                     for (int cc = cf; cc <= cl2 && npcs <= kCombineBatch; ++cc) {
@@ -806,7 +831,7 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
             const int n = info.w, G = p.G, rc = G * p.npc;
             const int c = x % p.chunks, g = (x / p.chunks) % p.Hkv, b = x / (p.chunks * p.Hkv);
             const int node0 = c * p.npc;
-            float *cmb_w = reinterpret_cast<float *>(s_p);  // [K][NT] weights
+            float *cmb_w = so + (size_t)K * kPart;  // [K][NT] merge weights, after the staged partials
             if (st < NT) {
                 float M = -INFINITY;
                 for (int k = 0; k < K; ++k) M = fmaxf(M, so[(size_t)k * kPart + NT * kHeadDim + st]);
@@ -857,7 +882,16 @@ template <int NT>
 static size_t attn_smem_bytes(int num_slots) {
     using Plan = SmemPlan<NT>;
     static_assert(3 * kCombineBatch * NT * 4 <= Plan::kPBuf, "combine staging must fit the P buffer");
-    return 1024 + (size_t)num_slots * kSlotBytes + 2 * Plan::kQBuf + Plan::kNP * Plan::kPBuf + sizeof(SmemMisc);
+    return 1024 + (size_t)num_slots * kSlotBytes + Plan::kNQ * Plan::kQBuf + Plan::kNP * Plan::kPBuf +
+           sizeof(SmemMisc);
+}
+
+// bytes rank 0 of a split-KV cluster can stage partials in: its K/V rings, Q and P^T buffers
+// (contiguous, all idle once its tiles are done)
+template <int NT>
+static size_t split_stage_bytes(int num_slots) {
+    using Plan = SmemPlan<NT>;
+    return (size_t)num_slots * kSlotBytes + Plan::kNQ * Plan::kQBuf + Plan::kNP * Plan::kPBuf;
 }
 
 template <int NT>
@@ -874,20 +908,18 @@ static cudaError_t launch_nt(const AttnParams &prm0, const void *q, const void *
         return cudaErrorInvalidValue;
     int ns = 2 * kMaxSlots;
     while (ns > 2 && attn_smem_bytes<NT>(ns) > max_smem) --ns;
-    // split-KV mode: rank 0 gathers every part's partial in its (contiguous) K/V rings
-    if (prm0.splitk > 1 && (size_t)prm0.splitk * (NT * kHeadDim + 2 * NT) * 4 > (size_t)ns * kSlotBytes)
+    // split-KV mode: rank 0 gathers every part's partial (and the merge weights) in its idle buffers
+    if (prm0.splitk > 1 && (size_t)prm0.splitk * (NT * kHeadDim + 3 * NT) * 4 > split_stage_bytes<NT>(ns))
         return cudaErrorInvalidConfiguration;
     // K tiles are released right after S = K Q^T; V tiles are held until PV: give V the extra slot
     ns = min(ns, 6);
     prm.nk_slots = ns / 2;
     prm.nv_slots = ns - ns / 2;
     const size_t smem = attn_smem_bytes<NT>(ns);
-    static bool attr_set = false;
-    if (!attr_set) {
-        cudaError_t e = cudaFuncSetAttribute(tree_attn_kernel<NT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             (int)max_smem);
+    {
+        const cudaError_t e = ensure_max_smem_attr((const void *)tree_attn_kernel<NT>, NT == 16 ? 0 : (NT == 32 ? 1 : 2),
+                                                   max_smem);
         if (e != cudaSuccess) return e;
-        attr_set = true;
     }
     // programmatic dependent launch: the prologue (barrier init, TMEM alloc, smem zeroing) of
     // this grid overlaps the tail of the previous kernel on the stream
@@ -914,15 +946,18 @@ static cudaError_t launch_nt(const AttnParams &prm0, const void *q, const void *
 cudaError_t launch_tree_attention_rows(const AttnParams &prm0, const void *q, const void *k, const void *v,
                                        int num_ctas, size_t max_smem, cudaStream_t stream);
 
-unsigned long long *g_attn_trace = nullptr;  // debug only (specinfer_debug_set_trace)
-int g_attn_debug_flags = 0;                   // debug only (SPECINFER_DEBUG_FLAGS, experiments)
+#ifdef SPECINFER_DEBUG_HOOKS
+unsigned long long *g_attn_trace = nullptr;  // debug build only (specinfer_debug_set_trace)
+int g_attn_debug_flags = 0;                   // debug build only (SPECINFER_DEBUG_FLAGS, experiments)
+#endif
 
 cudaError_t launch_tree_attention(const specinfer_shape_t &s, const WsLayout &w, const void *q,
                                   const void *k, const void *v, const int32_t *prefix_len,
                                   const int32_t *n_nodes, void *out, char *ws, int num_sms,
                                   size_t max_smem, cudaStream_t stream, const int32_t *page_table,
-                                  int num_pages) {
+                                  int num_pages, uint32_t flags) {
     AttnParams prm{};
+    prm.early_prefix = (flags & SPECINFER_ATTN_EARLY_PREFIX) ? 1 : 0;
     prm.page_table = page_table;
     prm.max_pages = (s.max_seq + kKeyTile - 1) / kKeyTile;
     prm.n_pages = num_pages;
@@ -949,8 +984,10 @@ cudaError_t launch_tree_attention(const specinfer_shape_t &s, const WsLayout &w,
     prm.lanes = w.lanes;
     const float sm_scale = s.sm_scale > 0.f ? s.sm_scale : 1.0f / sqrtf((float)s.head_dim);
     prm.scale_log2 = sm_scale * 1.4426950408889634f;
+#ifdef SPECINFER_DEBUG_HOOKS
     prm.trace = g_attn_trace;
     prm.debug_flags = g_attn_debug_flags;
+#endif
     prm.splitk = w.splitk;
     const int grid = w.grid;  // persistent one CTA per SM, or n_items x splitk in split-KV mode
     switch (w.nt) {

@@ -263,7 +263,7 @@ __global__ void __launch_bounds__(352, 1)
                 uint8_t *dst = s_ring + (size_t)slot * kSlotBytes;
                 uint64_t *bar = &misc->full[slot];
                 const CUtensorMap *m = is_v ? &tm_v : &tm_k;
-                if (p.debug_flags & 1) {  // experiment: no K/V traffic (results invalid)
+                if (SPI_FLAGS(p) & 1) {  // experiment: no K/V traffic (results invalid)
                     mbar_arrive(bar);
                 } else if (nv == kKeyTile) {
                     mbar_arrive_expect_tx(bar, kSlotBytes);
@@ -335,7 +335,7 @@ __global__ void __launch_bounds__(352, 1)
                         const uint64_t adesc = make_smem_desc(qbase + off, 16, 1024, kSw128);
                         const uint64_t bdesc = make_smem_desc(kbase + (kk >> 2) * kHalfBytes + (kk & 3) * 32, 16,
                                                               1024, kSw128);
-                        if (!(p.debug_flags & 2))
+                        if (!(SPI_FLAGS(p) & 2))
                             umma_bf16_ss(tmem + kColS + sb * 128, adesc, bdesc, idesc_s, kk > 0 ? 1u : 0u);
                     }
                     umma_commit(&misc->s_full[sb]);
@@ -378,7 +378,7 @@ __global__ void __launch_bounds__(352, 1)
 #pragma unroll
                     for (int kk = 0; kk < kKeyTile / 16; ++kk) {
                         const uint64_t bdesc = make_smem_desc(vbase + kk * 16 * 128, kHalfBytes, 1024, kSw128);
-                        if (!(p.debug_flags & 2))
+                        if (!(SPI_FLAGS(p) & 2))
                             umma_bf16_ts(tmem + kColO + pb * 128, tmem + kColS + pb * 128 + kk * 8, bdesc, idesc_o,
                                          (first && kk == 0) ? 0u : 1u);
                     }
@@ -454,7 +454,7 @@ __global__ void __launch_bounds__(352, 1)
                 // pass 1: tile row max (unmasked tiles, the common case, take the select-free path)
                 float tm4[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
                 if (masked) tile_max<true>(s_col, vis, tm4);
-                else if (p.debug_flags & 4) tm4[0] = 1.f;  // experiment: no S loads (results invalid)
+                else if (SPI_FLAGS(p) & 4) tm4[0] = 1.f;  // experiment: no S loads (results invalid)
                 else tile_max<false>(s_col, vis, tm4);
                 const float tm = fmaxf(fmaxf(tm4[0], tm4[1]), fmaxf(tm4[2], tm4[3])) * p.scale_log2;
                 // stale running max: move it only when this tile exceeds it by more than 2^8
@@ -488,7 +488,7 @@ __global__ void __launch_bounds__(352, 1)
                 // (keys 32 q .. 32 q + 31 -> columns 16 q .. 16 q + 15: always already read)
                 float l4[4] = {0.f, 0.f, 0.f, 0.f};
                 if (masked) tile_exp<true>(s_col, vis, p.scale_log2, mref, l4);
-                else if (p.debug_flags & 8) l4[0] = 1.f;  // experiment: no softmax work (results invalid)
+                else if (SPI_FLAGS(p) & 8) l4[0] = 1.f;  // experiment: no softmax work (results invalid)
                 else tile_exp<false>(s_col, vis, p.scale_log2, mref, l4);
                 l += (l4[0] + l4[1]) + (l4[2] + l4[3]);
                 tmem_st_wait();
@@ -676,12 +676,9 @@ cudaError_t launch_tree_attention_rows(const AttnParams &prm0, const void *q, co
     prm.nk_slots = ns;  // unified K/V ring
     prm.nv_slots = 0;
     const size_t smem = rows_smem_bytes(ns);
-    static bool attr_set = false;
-    if (!attr_set) {
-        cudaError_t e = cudaFuncSetAttribute(tree_attn_rows_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             (int)max_smem);
+    {
+        const cudaError_t e = ensure_max_smem_attr((const void *)tree_attn_rows_kernel, 3, max_smem);
         if (e != cudaSuccess) return e;
-        attr_set = true;
     }
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(num_ctas);

@@ -668,7 +668,11 @@ __global__ void __launch_bounds__(kMssThreads) verify_mss_kernel(
     cluster_sync_all();  // no CTA leaves while others may still read its DSMEM slots
 }
 
-unsigned long long *g_mss_trace = nullptr;  // debug only (specinfer_debug_set_trace with SPECINFER_TRACE_MSS)
+#ifdef SPECINFER_DEBUG_HOOKS
+unsigned long long *g_mss_trace = nullptr;  // debug build only (specinfer_debug_set_trace + SPECINFER_TRACE_MSS)
+#else
+static unsigned long long *const g_mss_trace = nullptr;  // production: no MSS timestamps
+#endif
 
 cudaError_t launch_verify_greedy(const specinfer_shape_t &s, const WsLayout &w, const float *logits,
                                  const int32_t *tree_tokens, const int32_t *parent, const int32_t *n_nodes,

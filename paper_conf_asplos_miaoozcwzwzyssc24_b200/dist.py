@@ -56,10 +56,13 @@ def unpack_accepted(buf: torch.Tensor):
 
 
 def gather_accepted(packed: torch.Tensor, out: torch.Tensor = None) -> torch.Tensor:
-    """All-gather the per-rank packed rows (equal request counts per rank) into [world·B][2Lp+1]."""
+    """All-gather the per-rank packed rows (EQUAL row counts per rank) into [world·rows][2Lp+1].
+    Uneven request shards go through `GatherPlan` (padding rows with n = 0)."""
     world = torch.distributed.get_world_size()
     if out is None:
         out = torch.empty((world * packed.shape[0], packed.shape[1]), dtype=packed.dtype, device=packed.device)
+    if out.shape[0] != world * packed.shape[0]:
+        raise ValueError(f"gather_accepted: out has {out.shape[0]} rows, expected {world} x {packed.shape[0]}")
     if torch.distributed.get_backend() == "nccl":
         torch.distributed.all_gather_into_tensor(out, packed)
     else:
@@ -68,3 +71,37 @@ def gather_accepted(packed: torch.Tensor, out: torch.Tensor = None) -> torch.Ten
         if parts[0].data_ptr() != out.data_ptr():
             out.copy_(torch.cat(parts, 0))
     return out
+
+
+class GatherPlan:
+    """The tokens-only exchange (a7) for `batch_global` requests split by `shard_requests` over
+    `world` ranks: every rank contributes ceil(B / world) rows (its requests, then padding rows with
+    n = 0, which every consumer treats as 'nothing accepted'), one all-gather, and `rows_of_all`
+    gives the global requests in order (padding dropped)."""
+
+    def __init__(self, batch_global: int, world: int, path_len: int, device):
+        self.world, self.B, self.Lp = world, batch_global, path_len
+        self.pad = -(-batch_global // world)
+        self.counts = [shard_requests(batch_global, world, r)[1] for r in range(world)]
+        idx = [r * self.pad + i for r in range(world) for i in range(self.counts[r])]
+        self.index = torch.tensor(idx, dtype=torch.long, device=device)
+        self.send = torch.zeros((self.pad, 2 * path_len + 1), dtype=torch.int32, device=device)
+        self.recv = torch.zeros((world * self.pad, 2 * path_len + 1), dtype=torch.int32, device=device)
+
+    def pack(self, n_accepted, accepted_tokens, accepted_nodes):
+        cnt = n_accepted.shape[0]
+        self.send[:cnt, 0] = n_accepted
+        self.send[:cnt, 1:1 + self.Lp] = accepted_tokens
+        self.send[:cnt, 1 + self.Lp:] = accepted_nodes
+        return self.send
+
+    def exchange(self):
+        if self.world > 1:
+            gather_accepted(self.send, self.recv)
+        else:
+            self.recv.copy_(self.send)
+        return self.recv
+
+    def rows_of_all(self) -> torch.Tensor:
+        """[batch_global][2Lp+1] packed rows of every request in global order."""
+        return self.recv.index_select(0, self.index)

@@ -166,3 +166,17 @@ def test_tree_merge_invalid():
     (par, dep, tok), nn, nmap, bits = _merge_gpu(reqs, 5)
     assert nn.tolist() == [0, 3, 0] and bits & 1
     assert (nmap[0] == -1).all() and (nmap[2] == -1).all()
+
+
+def test_tree_merge_depth_beyond_dmax():
+    """A merged tree deeper than Dmax is reported like every other bad input (header contract):
+    n_nodes 0, node_map -1, padding rows (parent -1, depth 0, token -1), BAD_TREE; other requests of
+    the batch are unaffected."""
+    reqs = [[([-1, 0, 1, 2], [1, 2, 3, 4])],              # depth 3 > Dmax 2
+            [([-1, 0, 1], [1, 2, 3]), ([-1, 0], [1, 5])]]  # depth 2: fine
+    (par, dep, tok), nn, nmap, bits = _merge_gpu(reqs, 8, Dmax=2)
+    assert nn.tolist() == [0, 4] and bits & 1
+    assert (nmap[0] == -1).all()
+    assert (par[0] == -1).all() and (dep[0] == 0).all() and (tok[0] == -1).all()
+    rp, rt, rd, _ = oracle.tree_merge(reqs[1])
+    assert list(par[1, :4]) == rp and list(tok[1, :4]) == rt and list(dep[1, :4]) == rd

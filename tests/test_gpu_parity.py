@@ -140,28 +140,32 @@ def test_attention_split_kv_clusters(Hq, Hkv, pls):
         assert torch.isnan(out[b, n[b]:].float()).all()
 
 
-@pytest.mark.parametrize("force_fallback", [False, True])
-def test_attention_split_merge_paths(force_fallback, monkeypatch):
-    """Stream-K split items (units cut by CTA boundaries): the merge through the bulk-staged path
-    and, forced with debug flag 32, the batched-load fallback path give the oracle's result."""
-    import os
-    if force_fallback:
-        monkeypatch.setenv("SPECINFER_DEBUG_FLAGS", "32")
-    spi.specinfer_debug_set_trace(None)  # (re-reads SPECINFER_DEBUG_FLAGS)
-    try:
-        # 24 units x ~24 tiles over 148 CTAs: stream-K (a unit exceeds an even share by > 16 tiles),
+@pytest.mark.parametrize("case", ["staged", "batched"])
+def test_attention_split_merge_paths(case):
+    """Stream-K split items (units cut by CTA boundaries) and both merge paths of the last piece:
+    'staged' = every piece's (O, m, l) bulk-copied into the idle K/V rings (at most 8 pieces);
+    'batched' = one request whose KV stream spans far more than 8 CTAs' shares, so its merge runs
+    the batched-load path (pieces read 8 at a time)."""
+    if case == "staged":
+        # 24 units x ~24 tiles over 148 CTAs: stream-K (a unit exceeds an even share by > 8 tiles),
         # every unit cut into ~6 pieces
         B, Hq, Hkv, P = 3, 8, 8, 3000
         parent, depth = W.expansion_tree((1, 1, 3, 1, 1, 1, 1, 1))
-        tb = W.make_tree_batch([(parent, depth)] * B, list(W.ragged_prefix(P, B)), device=DEV, max_depth=8)
-        smax = P + tb.max_nodes + 3
-        ai = W.make_attention_inputs(tb, 1, Hq, Hkv, smax, seed=77, device=DEV, poison=True)
-        out, _ = _gpu_attention(tb, ai, Hq, Hkv)
-        ref = _oracle_attention(ai, tb)
-        _check_rows(out, ref, tb)
-    finally:
-        monkeypatch.delenv("SPECINFER_DEBUG_FLAGS", raising=False)
-        spi.specinfer_debug_set_trace(None)
+        pls = list(W.ragged_prefix(P, B))
+        trees = [(parent, depth)] * B
+    else:
+        # 40 single-head requests, one of them with a 40000-key prefix (~313 tiles = ~130 CTAs'
+        # shares of the ~350-tile stream): that item is cut into far more than 8 pieces
+        B, Hq, Hkv = 40, 2, 1
+        parent, depth = W.expansion_tree((1, 2, 2))
+        pls = [40000] + [5 + 3 * b for b in range(B - 1)]
+        trees = [(parent, depth)] * B
+    tb = W.make_tree_batch(trees, pls, device=DEV, max_depth=8)
+    smax = max(pls) + tb.max_nodes + 3
+    ai = W.make_attention_inputs(tb, 1, Hq, Hkv, smax, seed=77, device=DEV, poison=True)
+    out, _ = _gpu_attention(tb, ai, Hq, Hkv)
+    ref = _oracle_attention(ai, tb)
+    _check_rows(out, ref, tb)
 
 
 @pytest.mark.parametrize("peaky", [False, True])
@@ -515,3 +519,43 @@ def test_kv_commit_parity(L, Hkv):
         assert np.array_equal(kh[:, b, :, :e], kg[:, b, :, :e])
         assert np.array_equal(vh[:, b, :, :e], vg[:, b, :, :e])
     assert int(na.cpu().numpy()[[0, 1, 3]].max()) >= 2  # some request committed a moved path
+
+
+@pytest.mark.parametrize("B,Hq,Hkv,expansion,P", [(2, 32, 32, (1, 1, 3, 1, 1, 1, 1, 1), 2048),   # split-KV
+                                                  (6, 8, 8, (1, 2, 2), 3000),                    # stream-K
+                                                  (3, 16, 2, (1, 2, 2, 2), 700)])                # rows kernel
+def test_attention_early_prefix_bit_identical(B, Hq, Hkv, expansion, P):
+    """SPECINFER_ATTN_EARLY_PREFIX (committed-prefix tiles staged before the programmatic dependency
+    resolves) on layers >= 1 of a CUDA-graph chain gives bit-identical outputs to plain launches,
+    and matches the oracle."""
+    parent, depth = W.expansion_tree(expansion)
+    tb = W.make_tree_batch([(parent, depth)] * B, list(W.ragged_prefix(P, B)), device=DEV, max_depth=8)
+    smax = P + tb.max_nodes + 2
+    L = 4
+    ai = W.make_attention_inputs(tb, L, Hq, Hkv, smax, seed=31, device=DEV, poison=True)
+    shape = _shape(tb, Hq, Hkv, smax)
+    outs = []
+    for early in (False, True):
+        st = spi.TreeState.create(shape, tb.parent, tb.depth, tb.prefix_len, tb.n_nodes)
+        out = torch.full(ai.q.shape, float("nan"), dtype=torch.bfloat16, device=DEV)
+        s = torch.cuda.Stream()
+        s.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.stream(s):
+            st.prepare()
+            for l in range(L):
+                st.attention(ai.q[l], ai.k_cache[l], ai.v_cache[l], out[l], prefetch=early and l > 0)
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=s):
+            st.prepare()
+            for l in range(L):
+                st.attention(ai.q[l], ai.k_cache[l], ai.v_cache[l], out[l], prefetch=early and l > 0)
+        out.fill_(float("nan"))
+        g.replay()
+        g.replay()
+        torch.cuda.synchronize()
+        outs.append(out)
+    n = tb.n_nodes.cpu().numpy()
+    for b in range(B):
+        assert torch.equal(outs[0][:, b, :n[b]], outs[1][:, b, :n[b]])
+    _check_rows(outs[1][L - 1], _oracle_attention(ai, tb, layer=L - 1), tb)

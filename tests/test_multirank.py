@@ -6,6 +6,7 @@ import os
 import socket
 
 import numpy as np
+import pytest
 import torch
 import torch.multiprocessing as mp
 
@@ -175,3 +176,110 @@ def test_bench_reference_arm_two_ranks_prints_one_line():
     assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["value"] == d["value"]
     assert d["e2e"] == {"value": d["value"], "unit": d["unit"], "h2d_bytes_per_step": 0,
                         "d2h_bytes_per_step": 0}
+
+
+# ---------------------------------------------------------------------------------------------
+# the bench's step plumbing (paper_conf_asplos_miaoozcwzwzyssc24_b200/step.py + bench.Workload)
+# end to end at world size 2 under gloo, with the oracle standing in for the device calls: both
+# layouts, an uneven request split (5 requests over 2 ranks), strong scaling; every rank's accepted
+# paths, attention outputs and committed cache equal the world-size-1 run's share bit for bit
+# ---------------------------------------------------------------------------------------------
+
+class OracleOps:
+    """Host stand-in for step.DeviceOps (same call signatures) backed by the fp64 oracle."""
+
+    class St:
+        def __init__(self, shape, parent, depth, prefix_len, n_nodes):
+            self.shape, self.parent, self.depth, self.prefix_len, self.n_nodes = shape, parent, depth, prefix_len, n_nodes
+
+    def state(self, shape, parent, depth, prefix_len, n_nodes):
+        return self.St(shape, parent, depth, prefix_len, n_nodes)
+
+    def prepare(self, st):
+        pass
+
+    def attention(self, st, q, k, v, out, prefetch):
+        r = oracle.tree_attention(q, k, v, st.parent, st.depth, st.prefix_len, st.n_nodes)
+        out.copy_(torch.from_numpy(np.nan_to_num(r)).to(torch.bfloat16))
+
+    def verify_greedy(self, shape, st, logits, tokens, parent, n_nodes, an, at, na):
+        r = oracle.verify_greedy(logits.numpy(), tokens.numpy(), parent.numpy(), n_nodes.numpy(), path_len=an.shape[1])
+        for dst, src in zip((an, at, na), r):
+            dst.copy_(torch.from_numpy(src))
+
+    def verify_mss(self, shape, st, logits, tokens, parent, n_nodes, draft, temperature, seed, offset, rids, an, at, na):
+        r = oracle.verify_mss(logits.numpy(), tokens.numpy(), parent.numpy(), n_nodes.numpy(), draft.numpy(),
+                              temperature=temperature, seed=seed, offset=offset, request_ids=rids.numpy(),
+                              path_len=an.shape[1])
+        for dst, src in zip((an, at, na), r[:3]):
+            dst.copy_(torch.from_numpy(src))
+
+    def kv_commit(self, shape, k_all, v_all, prefix_len, an, na):
+        kb = k_all.view(torch.int16).numpy().view(np.uint16)
+        vb = v_all.view(torch.int16).numpy().view(np.uint16)
+        oracle.kv_commit(kb, vb, prefix_len.numpy(), an.numpy(), na.numpy())
+
+
+STEP_CFG = W.Config("T", 2, 5, 4, 2, 40, (1, 2, 2), 50, ("greedy", "mss"), 7, "test config (GQA 4/2)")
+
+
+def _run_step(world, rank, kv_shard):
+    import argparse
+    import bench
+    from paper_conf_asplos_miaoozcwzwzyssc24_b200 import step as S
+    args = argparse.Namespace(layers=None, prefix=None, verify=None, batch=None, scaling="strong")
+    cfg = STEP_CFG
+    layout = S.make_layout(cfg.batch, world, rank, cfg.num_q_heads, cfg.num_kv_heads, kv_shard)
+    wl = bench.Workload(cfg, args, layout, "cpu")
+    shape_v = object() if kv_shard else None
+    tree = (wl.tb.parent, wl.tb.depth, wl.tb.prefix_len, wl.tb.n_nodes)
+    tree_v = (wl.tbv.parent, wl.tbv.depth, wl.tbv.prefix_len, wl.tbv.n_nodes) if kv_shard else tree
+    shape = object()
+    step = S.VerifyStep(OracleOps(), layout, shape, shape_v if kv_shard else shape, tree, tree_v, wl.verify,
+                        wl.Dmax + 1, "cpu")
+    out = torch.empty_like(wl.ai.q)
+    step.prepare()
+    for l in range(wl.L):
+        step.attention(wl.ai.q[l], wl.ai.k_cache[l], wl.ai.v_cache[l], out[l], layer=l)
+    inputs = {m: (wl.vi[m].logits, wl.vi[m].tree_tokens, wl.vi[m].draft_probs) for m in wl.verify}
+    step.verify(inputs, seed=cfg.seed, offset=3)
+    step.gather()
+    step.commit(wl.ai.k_cache, wl.ai.v_cache)
+    return (layout, step.accepted_all().numpy(), out.float().numpy(),
+            wl.ai.k_cache.view(torch.int16).numpy().copy(), wl.tb.prefix_len.numpy().copy(), wl.tb.n_nodes.numpy())
+
+
+def _step_worker(rank, world, port, kv_shard, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    torch.distributed.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        q.put((rank, _run_step(world, rank, kv_shard)))
+    finally:
+        torch.distributed.destroy_process_group()
+
+
+@pytest.mark.parametrize("kv_shard", [False, True])
+def test_step_plumbing_two_ranks_equals_one(kv_shard):
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_step_worker, args=(r, world, port, kv_shard, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = dict(q.get(timeout=300) for _ in range(world))
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    lay1, acc1, out1, k1, pl1, n1 = _run_step(1, 0, False)
+    assert acc1[:, 0].min() >= 1                                   # every request accepted its root at least
+    assert (acc1[:, 0] > 1).any()                                  # and some a longer path (rows really moved)
+    for r in range(world):
+        lay, acc, out, k, pl, n = res[r]
+        np.testing.assert_array_equal(acc, acc1)                   # the gathered accepted rows, global order
+        a = slice(lay.attn_lo, lay.attn_lo + lay.attn_cnt)
+        np.testing.assert_array_equal(pl, pl1[a])                  # committed prefix lengths
+        for i, b in enumerate(range(lay.attn_lo, lay.attn_lo + lay.attn_cnt)):
+            P = pl1[b]
+            np.testing.assert_array_equal(k[:, i, :, :P], k1[:, b, lay.kv0:lay.kv0 + lay.nkv, :P])
+            np.testing.assert_array_equal(out[:, i, :n1[b]], out1[:, b, :n1[b], lay.q0:lay.q0 + lay.nq])

@@ -32,6 +32,9 @@ def main():
     a = ap.parse_args()
     if a.lib:
         spi.load_library(a.lib)
+    elif a.trace or a.flags:
+        from paper_conf_asplos_miaoozcwzwzyssc24_b200 import build_lib
+        spi.load_library(build_lib.build(debug_hooks=True))  # hooks exist only in the development build
     cfg = W.CONFIGS[a.config]
     dev = torch.device("cuda:0")
     B = a.batch or cfg.batch
@@ -74,14 +77,14 @@ def main():
     res = {"flags": a.flags, "config": a.config, "B": B, "P": P, "us_per_launch": round(us, 2), "GBps": round(byts / us / 1e3, 1)}
     print(json.dumps(res), flush=True)
     if a.trace:
-        tr = torch.zeros(8 * 64 * 12 + 4 * 1024, dtype=torch.int64, device=dev)
+        tr = torch.zeros(8 * 64 * 16 + 8 * 1024, dtype=torch.int64, device=dev)
         spi.specinfer_debug_set_trace(tr)
         st.attention(ai.q[0], ai.k_cache[0], ai.v_cache[0], out[0])
         torch.cuda.synchronize()
         spi.specinfer_debug_set_trace(None)
         allt = tr.cpu().numpy().astype(np.int64)
-        t = allt[:8 * 64 * 12].reshape(8, 64, 12)
-        kt = allt[8 * 64 * 12:].reshape(-1, 4)
+        t = allt[:8 * 64 * 16].reshape(8, 64, 16)
+        kt = allt[8 * 64 * 16:].reshape(-1, 8)
         kt = kt[kt[:, 0] > 0]
         t0 = kt[:, 0].min() if len(kt) else 0
         if len(kt): print(f"kernel-level (us from first CTA entry) over {len(kt)} CTAs: entry max {(kt[:,0].max()-t0)/1e3:.2f}; "

@@ -5,13 +5,18 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np
 import torch
 import paper_conf_asplos_miaoozcwzwzyssc24_b200 as spi
+from paper_conf_asplos_miaoozcwzwzyssc24_b200 import build_lib
+spi.load_library(build_lib.build(debug_hooks=True))  # traces exist only in the development build
 import workloads as W
 
 ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="C2")
 ap.add_argument("--batch", type=int, default=1)
 ap.add_argument("--prefix", type=int, default=None)
+ap.add_argument("--flags", type=int, default=0, help="debug flags (64: no split-KV clusters)")
 a = ap.parse_args()
+os.environ["SPECINFER_DEBUG_FLAGS"] = str(a.flags)
+spi.specinfer_debug_set_trace(None)
 cfg = W.CONFIGS[a.config]
 dev = torch.device("cuda:0")
 P = a.prefix or cfg.prefix
@@ -26,13 +31,13 @@ out = torch.empty_like(ai.q[0])
 for _ in range(3):
     st.attention(ai.q[0], ai.k_cache[0], ai.v_cache[0], out)
 torch.cuda.synchronize()
-tr = torch.zeros(8 * 64 * 12 + 4 * 1024, dtype=torch.int64, device=dev)
+tr = torch.zeros(8 * 64 * 16 + 8 * 1024, dtype=torch.int64, device=dev)
 spi.specinfer_debug_set_trace(tr)
 torch.cuda.synchronize()
 st.attention(ai.q[0], ai.k_cache[0], ai.v_cache[0], out)
 torch.cuda.synchronize()
 spi.specinfer_debug_set_trace(None)
-kt = tr.cpu().numpy().astype(np.int64)[8 * 64 * 12:].reshape(-1, 4)[:148]
+kt = tr.cpu().numpy().astype(np.int64)[8 * 64 * 16:].reshape(-1, 8)[:148]
 kt = kt[kt[:, 0] > 0]  # CTAs of this launch (the grid may be smaller than 148)
 t0 = kt[:, 0].min()
 ex = (kt[:, 1] - t0) / 1e3
@@ -46,7 +51,7 @@ print("earliest 5:", [(int(c), round(float(ex[c]), 2)) for c in order[:5]])
 if (kt[:, 3] > 0).any():
     s3 = (kt[:, 3] - t0) / 1e3
     print("split-KV: first cluster barrier passed (us) min/median/max:", np.percentile(s3[kt[:, 3] > 0], [0, 50, 100]).round(2))
-t = tr.cpu().numpy().astype(np.int64)[:8 * 64 * 12].reshape(8, 64, 12)
+t = tr.cpu().numpy().astype(np.int64)[:8 * 64 * 16].reshape(8, 64, 16)
 for c in range(8):
     x = t[c]
     nv = int((x[:, 0] > 0).sum())
@@ -55,4 +60,4 @@ for c in range(8):
           "K-iss V-iss S-mma PV-mma 4..11")
     show = list(range(min(nv + 1, 8))) + [i for i in range(max(8, nv - 3), min(nv + 2, 64))]
     for i in show:
-        print(f"  {i:3d} " + " ".join(f"{(v - base) if v else -1:7d}" for v in x[i, :12]))
+        print(f"  {i:3d} " + " ".join(f"{(v - base) if v else -1:7d}" for v in x[i, :16]))

@@ -3,6 +3,8 @@ import argparse, os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np, torch
 import paper_conf_asplos_miaoozcwzwzyssc24_b200 as spi
+from paper_conf_asplos_miaoozcwzwzyssc24_b200 import build_lib
+spi.load_library(build_lib.build(debug_hooks=True))  # traces exist only in the development build
 import workloads as W
 
 ap = argparse.ArgumentParser()

@@ -298,3 +298,68 @@ def random_tree_batch(B: int, n: int, P: int, seed: int, max_depth: int = 8, max
         # depth <= 8 with fanout <= 8 can hold at most 1 + 8 + ... nodes; clamp fanout need
         trees.append(random_tree(nb, max_depth, max_fanout, rng))
     return make_tree_batch(trees, [P] * B, max_nodes=n, max_depth=max_depth, device=device)
+
+
+# --------------------------------------------------------------------------------------------
+# per-request generation (multi-GPU bench): every request's tensors come from their own seeded
+# generator, so a rank can materialise exactly its share of a GLOBAL problem (request range and /
+# or kv-head range) and the values equal the N = 1 run's bit for bit (strong scaling)
+# --------------------------------------------------------------------------------------------
+
+def request_seed(seed: int, tensor_id: int, layer: int, rid: int) -> int:
+    ss = np.random.SeedSequence([int(seed), int(tensor_id), int(layer), int(rid)])
+    return int(ss.generate_state(1, np.uint64)[0] & np.uint64(2**63 - 1))
+
+
+def make_request_attention_inputs(tree: TreeBatch, request_ids: Sequence[int], layers: int, num_q_heads: int,
+                                  num_kv_heads: int, smax: int, seed: int, q_heads: Tuple[int, int] = None,
+                                  kv_heads: Tuple[int, int] = None, device="cpu") -> AttnInputs:
+    """q, K, V ~ N(0,1) -> bf16 for the global requests ``request_ids`` (rows of ``tree`` in the same
+    order), keeping q-heads [q0, q0 + nq) and kv-heads [kv0, kv0 + nkv) of the global head counts."""
+    B, Nmax = tree.parent.shape
+    assert len(request_ids) == B
+    q0, nq = q_heads or (0, num_q_heads)
+    kv0, nkv = kv_heads or (0, num_kv_heads)
+    D = HEAD_DIM
+    q = torch.empty((layers, B, Nmax, nq, D), dtype=torch.bfloat16, device=device)
+    k = torch.empty((layers, B, nkv, smax, D), dtype=torch.bfloat16, device=device)
+    v = torch.empty_like(k)
+    for l in range(layers):
+        for i, rid in enumerate(request_ids):
+            q[l, i] = randn_bf16((Nmax, num_q_heads, D), request_seed(seed, 1, l, rid), device)[:, q0:q0 + nq]
+            k[l, i] = randn_bf16((num_kv_heads, smax, D), request_seed(seed, 2, l, rid), device)[kv0:kv0 + nkv]
+            v[l, i] = randn_bf16((num_kv_heads, smax, D), request_seed(seed, 3, l, rid), device)[kv0:kv0 + nkv]
+    return AttnInputs(q, k, v, tree, smax)
+
+
+def make_request_verify_inputs(tree: TreeBatch, request_ids: Sequence[int], vocab: int, seed: int, mode: str,
+                               device="cpu", tau: Optional[float] = None,
+                               logit_scale: float = LOGIT_SCALE) -> VerifyInputs:
+    """make_verify_inputs with one generator per global request (same recipe)."""
+    B, Nmax = tree.parent.shape
+    if tau is None:
+        tau = TAU_GREEDY if mode == "greedy" else TAU_MSS
+    parent = tree.parent.cpu().numpy()
+    n_nodes = tree.n_nodes.cpu().numpy()
+    logits = torch.empty((B, Nmax, vocab), dtype=torch.float32, device=device)
+    draft = torch.zeros((B, Nmax, vocab), dtype=torch.float32, device=device)
+    tokens = np.zeros((B, Nmax), np.int32)
+    for i, rid in enumerate(request_ids):
+        g = _gen(request_seed(seed, 7 if mode == "greedy" else 9, 0, rid), device)
+        lg = torch.randn((Nmax, vocab), generator=g, device=device, dtype=torch.float32).mul_(logit_scale)
+        noise = torch.randn((Nmax, vocab), generator=g, device=device, dtype=torch.float32)
+        q = torch.softmax(lg + tau * noise, dim=-1)
+        logits[i] = lg
+        gs = _gen(request_seed(seed, 8, 0, rid), device)
+        kids = {}
+        for c in range(1, int(n_nodes[i])):
+            kids.setdefault(int(parent[i, c]), []).append(c)
+        for u, cs in kids.items():
+            if mode == "greedy":
+                toks = torch.topk(q[u], len(cs)).indices.cpu().numpy()
+            else:
+                toks = torch.multinomial(q[u], len(cs), replacement=True, generator=gs).cpu().numpy()
+            for c, t in zip(cs, toks):
+                tokens[i, c] = int(t)
+                draft[i, c] = q[u]
+    return VerifyInputs(logits, draft, torch.from_numpy(tokens).to(device))
