@@ -183,6 +183,12 @@ class Workload:
         # MSS's distributional guarantee), so each verifier gets the tree tokens of its own mode
         self.vi = {m: W.make_request_verify_inputs(self.tbv, list(layout.verify_ids), self.V, cfg.seed, m,
                                                    device=device) for m in self.verify}
+        if len(self.vi) > 1:
+            # the same LLM logits and SSM distributions (only the tree tokens differ): one copy in HBM
+            first = self.vi[self.verify[0]]
+            for m in self.verify[1:]:
+                assert torch.equal(self.vi[m].logits, first.logits)
+                self.vi[m] = W.VerifyInputs(first.logits, first.draft_probs, self.vi[m].tree_tokens)
         self.bytes_launch = self.attn_bytes_per_launch()
         self.flops_launch = self.attn_flops_per_launch()
 
@@ -384,17 +390,17 @@ def run_ours(args, ws, rank, local):
     if not args.no_e2e:
         h_q = torch.empty_like(wl.ai.q, device="cpu").pin_memory()
         h_q.copy_(wl.ai.q)
-        h_in = {m: [t.cpu().pin_memory() for t in (wl.vi[m].logits, wl.vi[m].tree_tokens)] +
-                ([wl.vi[m].draft_probs.cpu().pin_memory()] if m == "mss" else []) for m in wl.verify}
-        d_in = {m: [wl.vi[m].logits, wl.vi[m].tree_tokens] + ([wl.vi[m].draft_probs] if m == "mss" else [])
-                for m in wl.verify}
+        # the step's inputs once each: the LLM logits (shared by the verifiers), the draft
+        # probabilities (MSS), every verifier's tree tokens
+        d_list = [wl.vi[wl.verify[0]].logits] + ([wl.vi["mss"].draft_probs] if "mss" in wl.verify else []) + \
+            [wl.vi[m].tree_tokens for m in wl.verify]
+        h_list = [t.cpu().pin_memory() for t in d_list]
         tree_dev = [wl.tb.parent, wl.tb.depth, wl.tb.n_nodes, prefix0]
         h_tree = [t.cpu().pin_memory() for t in tree_dev]
         res_a, res_n = step.res[step.commit_mode][1], step.res[step.commit_mode][2]
         h_res_a = torch.empty(tuple(res_a.shape), dtype=torch.int32).pin_memory()
         h_res_n = torch.empty(tuple(res_n.shape), dtype=torch.int32).pin_memory()
-        h2d = h_q.numel() * 2 + sum(t.numel() * t.element_size() for v in h_in.values() for t in v) + \
-            sum(t.numel() * 4 for t in h_tree)
+        h2d = h_q.numel() * 2 + sum(t.numel() * t.element_size() for t in h_list) + sum(t.numel() * 4 for t in h_tree)
         d2h = h_res_a.numel() * 4 + h_res_n.numel() * 4
 
         # One CUDA graph per step: the H2D copies run on a copy stream (pinned memory, the copy
@@ -414,9 +420,8 @@ def run_ours(args, ws, rank, local):
                 for l in range(L):
                     wl.ai.q[l].copy_(h_q[l], non_blocking=True)
                     ev_q[l].record(copy_s)
-                for m in wl.verify:
-                    for d, h in zip(d_in[m], h_in[m]):
-                        d.copy_(h, non_blocking=True)
+                for d, h in zip(d_list, h_list):
+                    d.copy_(h, non_blocking=True)
                 ev_lg.record(copy_s)
             s.wait_event(ev_tree)
             seg_prepare()
@@ -463,10 +468,10 @@ def run_ours(args, ws, rank, local):
         e2e = {"value": round(tokens_step_global * K / (e2e_ms / 1e3), 1), "unit": UNIT,
                "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
                "ms_per_step": round(e2e_ms / K, 4),
-               "inputs": "per step from pinned host memory: tree arrays, q of every layer, logits + tree tokens"
-                         + (" + draft probabilities" if "mss" in wl.verify else "")
-                         + " of each verifier; result read back: accepted tokens + counts; H2D on a copy stream "
-                           "overlapping the attention of earlier layers"}
+               "inputs": "per step from pinned host memory: tree arrays, q of every layer, the LLM logits"
+                         + (", draft probabilities" if "mss" in wl.verify else "")
+                         + ", each verifier's tree tokens; result read back: accepted tokens + counts; H2D on a copy "
+                           "stream overlapping the attention of earlier layers"}
 
     cpu = None
     if rank == 0 and ws == 1 and not args.no_cpu:

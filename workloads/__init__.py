@@ -335,7 +335,9 @@ def make_request_attention_inputs(tree: TreeBatch, request_ids: Sequence[int], l
 def make_request_verify_inputs(tree: TreeBatch, request_ids: Sequence[int], vocab: int, seed: int, mode: str,
                                device="cpu", tau: Optional[float] = None,
                                logit_scale: float = LOGIT_SCALE) -> VerifyInputs:
-    """make_verify_inputs with one generator per global request (same recipe)."""
+    """make_verify_inputs with one generator per global request (same recipe).  The LLM logits and the
+    SSM distributions of a request do not depend on `mode`; only the drafting policy does (greedy:
+    top-k children, MSS: i.i.d. draws), so both verifiers of a config see the same model outputs."""
     B, Nmax = tree.parent.shape
     if tau is None:
         tau = TAU_GREEDY if mode == "greedy" else TAU_MSS
@@ -345,7 +347,7 @@ def make_request_verify_inputs(tree: TreeBatch, request_ids: Sequence[int], voca
     draft = torch.zeros((B, Nmax, vocab), dtype=torch.float32, device=device)
     tokens = np.zeros((B, Nmax), np.int32)
     for i, rid in enumerate(request_ids):
-        g = _gen(request_seed(seed, 7 if mode == "greedy" else 9, 0, rid), device)
+        g = _gen(request_seed(seed, 7, 0, rid), device)
         lg = torch.randn((Nmax, vocab), generator=g, device=device, dtype=torch.float32).mul_(logit_scale)
         noise = torch.randn((Nmax, vocab), generator=g, device=device, dtype=torch.float32)
         q = torch.softmax(lg + tau * noise, dim=-1)
