@@ -62,6 +62,9 @@ def parse():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-early", action="store_true", help="plain attention launches (no EARLY_PREFIX)")
     ap.add_argument("--verify", default=None, help="comma list overriding the config's verify modes")
+    ap.add_argument("--gather", default="p2p", choices=["p2p", "nccl"],
+                    help="tokens-only exchange: fused into the verifier with peer stores (NEXT-4a, default) or an "
+                         "NCCL all-gather between the verify and commit graphs (the baseline)")
     ap.add_argument("--shard", default="auto", choices=["auto", "request", "kv"],
                     help="layout: request sharding, or kv-head sharding (GQA; auto for G > 1 at N > 1)")
     return ap.parse_args()
@@ -234,7 +237,17 @@ def run_ours(args, ws, rank, local):
                if kv_shard else shape)
     tree = (wl.tb.parent, wl.tb.depth, wl.tb.prefix_len, wl.tb.n_nodes)
     tree_v = (wl.tbv.parent, wl.tbv.depth, wl.tbv.prefix_len, wl.tbv.n_nodes) if kv_shard else tree
-    step = S.VerifyStep(S.DeviceOps(), layout, shape, shape_v, tree, tree_v, wl.verify, Lp, device)
+    from paper_conf_asplos_miaoozcwzwzyssc24_b200 import dist as D
+    p2p, gather_note = None, "NCCL all_gather_into_tensor between the verify and commit graphs" if ws > 1 else \
+        "local copy (N = 1)"
+    if args.gather == "p2p":
+        try:
+            p2p = D.P2PGather(Bg, ws, rank, Lp, device, exchange=D.all_gather_object_exchange if ws > 1 else None)
+            gather_note = ("fused into the committed verifier: peer stores of every request's row + epoch flags "
+                           "(CUDA IPC over NVLink), device-side wait in the verify graph")
+        except Exception as exc:   # (setup only: no IPC between the ranks' GPUs) -> the NCCL baseline
+            gather_note = f"p2p setup failed ({type(exc).__name__}: {exc}); NCCL all-gather"
+    step = S.VerifyStep(S.DeviceOps(), layout, shape, shape_v, tree, tree_v, wl.verify, Lp, device, p2p=p2p)
     inputs = {m: (wl.vi[m].logits, wl.vi[m].tree_tokens, wl.vi[m].draft_probs if m == "mss" else None)
               for m in wl.verify}
     out = torch.empty_like(wl.ai.q)
@@ -251,6 +264,12 @@ def run_ours(args, ws, rank, local):
 
     def seg_verify():
         step.verify(inputs, seed=cfg.seed, offset=0)
+        if p2p is not None:
+            step.gather()    # device-side wait for every rank's rows (graph-capturable)
+
+    def gather_between():
+        if p2p is None:
+            step.gather()    # NCCL / local copy: eager, between the verify and commit graphs
 
     def seg_commit():
         step.commit(wl.ai.k_cache, wl.ai.v_cache)
@@ -259,14 +278,15 @@ def run_ours(args, ws, rank, local):
                          L * spi.specinfer_launches_per_call("tree_attention") +
                          ("greedy" in wl.verify) * spi.specinfer_launches_per_call("verify_greedy") +
                          ("mss" in wl.verify) * spi.specinfer_launches_per_call("verify_mss") +
-                         spi.specinfer_launches_per_call("kv_commit"))
+                         spi.specinfer_launches_per_call("kv_commit") +
+                         (spi.specinfer_launches_per_call("gather_wait") if p2p is not None else 0))
 
     # ---- capture the segments as CUDA graphs (one launch each per step; the gather stays eager) ----
     s = torch.cuda.Stream(device)
     s.wait_stream(torch.cuda.current_stream(device))
     with torch.cuda.stream(s):
         for _ in range(2):  # eager warm-up (lazy init, tensor-map encode, func attributes)
-            seg_prepare(); seg_attention(); seg_verify(); step.gather(); seg_commit()
+            seg_prepare(); seg_attention(); seg_verify(); gather_between(); seg_commit()
     torch.cuda.synchronize(device)
     graphs = []
     for fn in (seg_prepare, seg_attention, seg_verify, seg_commit):
@@ -278,7 +298,7 @@ def run_ours(args, ws, rank, local):
 
     with torch.cuda.stream(s):
         for _ in range(args.warmup):
-            graphs[0].replay(); graphs[1].replay(); graphs[2].replay(); step.gather(); graphs[3].replay()
+            graphs[0].replay(); graphs[1].replay(); graphs[2].replay(); gather_between(); graphs[3].replay()
     torch.cuda.synchronize(device)
     K = args.steps
     ev = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(K)]
@@ -298,7 +318,7 @@ def run_ours(args, ws, rank, local):
             graphs[1].replay()
             ev[k][2].record(s)
             graphs[2].replay()
-            step.gather()
+            gather_between()
             graphs[3].replay()
         e_all[1].record(s)
     torch.cuda.synchronize(device)
@@ -430,7 +450,7 @@ def run_ours(args, ws, rank, local):
                 step.attention(wl.ai.q[l], wl.ai.k_cache[l], wl.ai.v_cache[l], out[l], layer=l if early else 0)
             s.wait_event(ev_lg)
             seg_verify()
-            step.gather()
+            gather_between()
             seg_commit()
             h_res_a.copy_(res_a, non_blocking=True)
             h_res_n.copy_(res_n, non_blocking=True)
@@ -492,8 +512,8 @@ def run_ours(args, ws, rank, local):
                                    else f"request-sharded x{ws}") if ws > 1 else "single GPU",
                    "l2": "no flush: every step streams this GPU's KV cache "
                          f"({2 * L * layout.attn_cnt * wl.Hkv * wl.smax * 256 / 1e9:.1f} GB) >> 126 MB L2",
-                   "graph": "4 CUDA graphs per step (prepare | L x attention | verify | commit), the tokens-only "
-                            "gather between (NCCL at N > 1)",
+                   "graph": "4 CUDA graphs per step (prepare | L x attention | verify | commit)",
+                   "gather": gather_note,
                    "attention_launch": "SPECINFER_ATTN_EARLY_PREFIX on layers >= 1" if early else "plain"},
         "step_ms": percentiles(step_ms),
         "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,

@@ -161,6 +161,49 @@ specinfer_status_t specinfer_verify_mss(const specinfer_shape_t *shape, const fl
                                         int32_t *accepted_tokens, int32_t *n_accepted,
                                         void *workspace, specinfer_stream_t stream);
 
+/* NEXT-4a: the tokens-only exchange after verification (a7) fused into the
+ * verifier.  Every rank r of `world` allocates (device memory, zero-initialised, owned by the
+ * caller) a receive table recv_r int32 [2][world * rows_per_rank][row_len] (double-buffered by
+ * step parity), arrival flags flags_r uint32 [world] and a local state uint32 [2]; the descriptor
+ * holds EVERY rank's recv / flags pointers as mapped in this process (CUDA IPC / peer access over
+ * NVLink; recv[rank] / flags[rank] are this rank's own) and this rank's state.  row_len =
+ * 2 (Dmax + 1) + 1: a row is [n_accepted | accepted_tokens | accepted_nodes] of one request; request
+ * b of rank r goes to row r * rows_per_rank + b (rows_per_rank >= every rank's batch; rows of absent
+ * requests stay as the caller initialised them, zero = nothing accepted).
+ * specinfer_verify_greedy_ex / specinfer_verify_mss_ex (gather NULL = the plain call): the CTA
+ * that finishes a request stores its row into every rank's table (peer stores), the last request
+ * of the rank releases the step's epoch on every rank's flag (system scope).
+ * specinfer_gather_wait: waits (acquire) until every rank released this step's epoch to us, copies
+ * the step's table to table_out int32 [world * rows_per_rank][row_len] (device, may be NULL) and
+ * advances the local epoch.  Calls of one rank must alternate verify_*_ex, gather_wait on one stream
+ * (graph-capturable: the epoch lives in `state`).  A rank that never publishes makes the others'
+ * gather_wait trap after a watchdog timeout (launch failure).  Errors: INVALID_ARG for world
+ * outside [1, SPECINFER_MAX_PEERS], rank >= world, rows_per_rank < batch, wrong row_len, NULL
+ * pointers. */
+#define SPECINFER_MAX_PEERS 8
+typedef struct {
+    int32_t world, rank, rows_per_rank, row_len;
+    int32_t *recv[SPECINFER_MAX_PEERS];
+    uint32_t *flags[SPECINFER_MAX_PEERS];
+    uint32_t *state;
+} specinfer_gather_t;
+specinfer_status_t specinfer_verify_greedy_ex(const specinfer_shape_t *shape, const float *logits,
+                                              const int32_t *tree_tokens, const int32_t *parent,
+                                              const int32_t *n_nodes, int32_t *accepted_nodes,
+                                              int32_t *accepted_tokens, int32_t *n_accepted,
+                                              void *workspace, const specinfer_gather_t *gather,
+                                              specinfer_stream_t stream);
+specinfer_status_t specinfer_verify_mss_ex(const specinfer_shape_t *shape, const float *logits,
+                                           const int32_t *tree_tokens, const int32_t *parent,
+                                           const int32_t *n_nodes, const float *draft_probs,
+                                           float temperature, uint64_t seed, uint64_t offset,
+                                           const int32_t *request_ids, int32_t *accepted_nodes,
+                                           int32_t *accepted_tokens, int32_t *n_accepted,
+                                           void *workspace, const specinfer_gather_t *gather,
+                                           specinfer_stream_t stream);
+specinfer_status_t specinfer_gather_wait(const specinfer_gather_t *gather, int32_t *table_out,
+                                         specinfer_stream_t stream);
+
 /* NEXT-4: rotary position encoding of the tree (reading A4: node i of request b is token number
  * depth[i] after the committed prefix of S_u, Def. 4.1, so it is encoded at position
  * P_b + depth[i]; siblings share a position).  In place, one launch:

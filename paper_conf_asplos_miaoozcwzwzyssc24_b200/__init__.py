@@ -37,7 +37,9 @@ EXPORTED_SYMBOLS = (
     "specinfer_verify_ns", "specinfer_expansion_topology", "specinfer_expand_step", "specinfer_tree_merge",
     "specinfer_tree_attention_paged", "specinfer_kv_commit_paged", "specinfer_tree_rope",
     "specinfer_debug_hooks_enabled", "specinfer_tree_attention_ex", "specinfer_hbm_read_probe",
+    "specinfer_verify_greedy_ex", "specinfer_verify_mss_ex", "specinfer_gather_wait",
 )
+MAX_PEERS = 8
 SPECINFER_ATTN_EARLY_PREFIX = 1
 
 
@@ -55,6 +57,13 @@ class Shape(ctypes.Structure):
 
     def __repr__(self):
         return "Shape(" + ", ".join(f"{n}={getattr(self, n)}" for n, _ in self._fields_) + ")"
+
+
+class GatherDesc(ctypes.Structure):
+    """specinfer_gather_t (NEXT-4a fused verify -> gather; include/specinfer.h)."""
+    _fields_ = [("world", ctypes.c_int32), ("rank", ctypes.c_int32), ("rows_per_rank", ctypes.c_int32),
+                ("row_len", ctypes.c_int32), ("recv", ctypes.c_void_p * MAX_PEERS),
+                ("flags", ctypes.c_void_p * MAX_PEERS), ("state", ctypes.c_void_p)]
 
 
 def make_shape(batch, max_nodes, num_q_heads, num_kv_heads, max_seq, *, num_layers=1, vocab=0,
@@ -98,6 +107,12 @@ def load_library(path: str = LIB_PATH):
     lib.specinfer_sequence_pack.argtypes = [sp, i32, i32] + [vp] * 14 + [vp]
     lib.specinfer_debug_set_trace.argtypes = [vp]
     lib.specinfer_debug_set_trace.restype = None
+    gp = ctypes.POINTER(GatherDesc)
+    lib.specinfer_verify_greedy_ex.argtypes = [sp, vp, vp, vp, vp, vp, vp, vp, vp, gp, vp]
+    lib.specinfer_verify_mss_ex.argtypes = [sp, vp, vp, vp, vp, vp, f32, u64, u64, vp, vp, vp, vp, vp, gp, vp]
+    lib.specinfer_gather_wait.argtypes = [gp, vp, vp]
+    for name in ("specinfer_verify_greedy_ex", "specinfer_verify_mss_ex", "specinfer_gather_wait"):
+        getattr(lib, name).restype = i32
     lib.specinfer_hbm_read_probe.argtypes = [vp, ctypes.c_size_t, vp]
     lib.specinfer_hbm_read_probe.restype = i32
     lib.specinfer_debug_hooks_enabled.argtypes = []
@@ -251,7 +266,9 @@ def specinfer_tree_rope(shape: Shape, q, k_cache, prefix_len, depth, n_nodes, ro
 
 
 def specinfer_verify_greedy(shape: Shape, logits, tree_tokens, parent, n_nodes, accepted_nodes,
-                            accepted_tokens, n_accepted, workspace):
+                            accepted_tokens, n_accepted, workspace, gather: Optional[GatherDesc] = None):
+    """VerifyGreedy; with `gather` (NEXT-4a) the accepted rows also go to every rank's receive table
+    (specinfer_verify_greedy_ex)."""
     dev = logits.device
     B, N, V, Lp = shape.batch, shape.max_nodes, shape.vocab, shape.max_depth + 1
     args = (_req("logits", logits, torch.float32, (B, N, V), dev),
@@ -261,12 +278,18 @@ def specinfer_verify_greedy(shape: Shape, logits, tree_tokens, parent, n_nodes, 
             _req("accepted_tokens", accepted_tokens, torch.int32, (B, Lp), dev),
             _req("n_accepted", n_accepted, torch.int32, (B,), dev),
             _req("workspace", workspace, torch.uint8, None, dev))
-    _check("specinfer_verify_greedy",
-           load_library().specinfer_verify_greedy(ctypes.byref(shape), *args, _stream(logits)))
+    lib = load_library()
+    if gather is not None:
+        _check("specinfer_verify_greedy_ex",
+               lib.specinfer_verify_greedy_ex(ctypes.byref(shape), *args, ctypes.byref(gather), _stream(logits)))
+    else:
+        _check("specinfer_verify_greedy", lib.specinfer_verify_greedy(ctypes.byref(shape), *args, _stream(logits)))
 
 
 def specinfer_verify_mss(shape: Shape, logits, tree_tokens, parent, n_nodes, draft_probs, temperature,
-                         seed, offset, request_ids, accepted_nodes, accepted_tokens, n_accepted, workspace):
+                         seed, offset, request_ids, accepted_nodes, accepted_tokens, n_accepted, workspace,
+                         gather: Optional[GatherDesc] = None):
+    """VerifyStochastic (MSS); with `gather` the rows are also published (specinfer_verify_mss_ex)."""
     dev = logits.device
     B, N, V, Lp = shape.batch, shape.max_nodes, shape.vocab, shape.max_depth + 1
     if not (temperature > 0):
@@ -280,11 +303,28 @@ def specinfer_verify_mss(shape: Shape, logits, tree_tokens, parent, n_nodes, dra
          _req("accepted_tokens", accepted_tokens, torch.int32, (B, Lp), dev),
          _req("n_accepted", n_accepted, torch.int32, (B,), dev),
          _req("workspace", workspace, torch.uint8, None, dev))
-    _check("specinfer_verify_mss",
-           load_library().specinfer_verify_mss(ctypes.byref(shape), *a, ctypes.c_float(temperature),
-                                               ctypes.c_uint64(int(seed) & (2**64 - 1)),
-                                               ctypes.c_uint64(int(offset) & (2**64 - 1)), rid, *o,
-                                               _stream(logits)))
+    lib = load_library()
+    sc = (ctypes.c_float(temperature), ctypes.c_uint64(int(seed) & (2**64 - 1)),
+          ctypes.c_uint64(int(offset) & (2**64 - 1)), rid)
+    if gather is not None:
+        _check("specinfer_verify_mss_ex",
+               lib.specinfer_verify_mss_ex(ctypes.byref(shape), *a, *sc, *o, ctypes.byref(gather), _stream(logits)))
+    else:
+        _check("specinfer_verify_mss", lib.specinfer_verify_mss(ctypes.byref(shape), *a, *sc, *o, _stream(logits)))
+
+
+def specinfer_gather_wait(gather: GatherDesc, table_out: Optional[torch.Tensor] = None, stream_of=None):
+    """NEXT-4a: wait for every rank's rows of this step, copy them to `table_out` (int32
+    [world * rows_per_rank][row_len], CUDA), advance the epoch.  Stream: the current stream of
+    `table_out`'s device (or of `stream_of`)."""
+    ref = table_out if table_out is not None else stream_of
+    if ref is None:
+        raise ValueError("specinfer_gather_wait: pass table_out or stream_of (a CUDA tensor)")
+    tp = None
+    if table_out is not None:
+        tp = _req("table_out", table_out, torch.int32, (gather.world * gather.rows_per_rank, gather.row_len),
+                  table_out.device)
+    _check("specinfer_gather_wait", load_library().specinfer_gather_wait(ctypes.byref(gather), tp, _stream(ref)))
 
 
 def specinfer_verify_ns(shape: Shape, logits, tree_tokens, parent, n_nodes, temperature, seed, offset, request_ids,

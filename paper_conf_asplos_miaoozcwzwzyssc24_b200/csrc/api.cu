@@ -9,6 +9,7 @@
 #include <mutex>
 
 #include "common.cuh"
+#include "gather.cuh"
 
 namespace specinfer {
 cudaError_t launch_tree_prepare(const specinfer_shape_t &s, const WsLayout &w, const int32_t *parent,
@@ -21,12 +22,13 @@ cudaError_t launch_tree_attention(const specinfer_shape_t &s, const WsLayout &w,
 cudaError_t launch_verify_greedy(const specinfer_shape_t &s, const WsLayout &w, const float *logits,
                                  const int32_t *tree_tokens, const int32_t *parent, const int32_t *n_nodes,
                                  int32_t *acc_nodes, int32_t *acc_tokens, int32_t *n_acc, char *ws,
-                                 cudaStream_t stream);
+                                 cudaStream_t stream, const GatherDev *gather);
+cudaError_t launch_gather_wait(const GatherDev &g, int32_t *table_out, cudaStream_t stream);
 cudaError_t launch_verify_mss(const specinfer_shape_t &s, const WsLayout &w, const float *logits,
                               const int32_t *tree_tokens, const int32_t *parent, const int32_t *n_nodes,
                               const float *draft_probs, float temperature, uint64_t seed, uint64_t offset,
                               const int32_t *request_ids, int32_t *acc_nodes, int32_t *acc_tokens,
-                              int32_t *n_acc, char *ws, cudaStream_t stream);
+                              int32_t *n_acc, char *ws, cudaStream_t stream, const GatherDev *gather);
 cudaError_t launch_verify_ns(const specinfer_shape_t &s, const WsLayout &w, const float *logits,
                              const int32_t *tree_tokens, const int32_t *parent, const int32_t *n_nodes,
                              float temperature, uint64_t seed, uint64_t offset, const int32_t *request_ids,
@@ -133,6 +135,27 @@ specinfer_status_t check_ws(const void *ws) {
 // the verifiers read logits / draft rows with 128-bit loads: the row bases must be 16-byte aligned
 bool misaligned16(const void *a, const void *b = nullptr) {
     return ((reinterpret_cast<uintptr_t>(a) | reinterpret_cast<uintptr_t>(b)) & 15u) != 0;
+}
+
+// host validation of a gather descriptor (NEXT-4a) against the verify shape
+specinfer_status_t gather_dev(const specinfer_gather_t *g, const specinfer_shape_t &s, GatherDev *out) {
+    if (g->world < 1 || g->world > SPECINFER_MAX_PEERS || g->rank < 0 || g->rank >= g->world) return SPECINFER_ERR_INVALID_ARG;
+    if (g->rows_per_rank < s.batch || g->row_len != 2 * (s.max_depth + 1) + 1 || !g->state)
+        return SPECINFER_ERR_INVALID_ARG;
+    GatherDev d{};
+    for (int r = 0; r < g->world; ++r) {
+        if (!g->recv[r] || !g->flags[r]) return SPECINFER_ERR_INVALID_ARG;
+        d.recv[r] = g->recv[r];
+        d.flags[r] = g->flags[r];
+    }
+    d.state = g->state;
+    d.world = g->world;
+    d.rank = g->rank;
+    d.rows_per_rank = g->rows_per_rank;
+    d.row_len = g->row_len;
+    d.nreq = s.batch;
+    *out = d;
+    return SPECINFER_OK;
 }
 
 specinfer_status_t from_cuda(cudaError_t e) { return e == cudaSuccess ? SPECINFER_OK : SPECINFER_ERR_CUDA; }
@@ -245,22 +268,57 @@ specinfer_status_t specinfer_tree_rope(const specinfer_shape_t *shape, void *q, 
     return from_cuda(launch_tree_rope(*shape, q, k_cache, prefix_len, depth, n_nodes, rope_base, (cudaStream_t)stream));
 }
 
-specinfer_status_t specinfer_verify_greedy(const specinfer_shape_t *shape, const float *logits,
-                                           const int32_t *tree_tokens, const int32_t *parent, const int32_t *n_nodes,
-                                           int32_t *accepted_nodes, int32_t *accepted_tokens, int32_t *n_accepted,
-                                           void *workspace, specinfer_stream_t stream) {
+specinfer_status_t specinfer_verify_greedy_ex(const specinfer_shape_t *shape, const float *logits,
+                                              const int32_t *tree_tokens, const int32_t *parent,
+                                              const int32_t *n_nodes, int32_t *accepted_nodes,
+                                              int32_t *accepted_tokens, int32_t *n_accepted, void *workspace,
+                                              const specinfer_gather_t *gather, specinfer_stream_t stream) {
     SPI_TRY(check_shape(shape));
     if (shape->vocab < 1) return SPECINFER_ERR_INVALID_ARG;
     if (!logits || !tree_tokens || !parent || !n_nodes || !accepted_nodes || !accepted_tokens || !n_accepted)
         return SPECINFER_ERR_INVALID_ARG;
     if (misaligned16(logits)) return SPECINFER_ERR_INVALID_ARG;
+    GatherDev g{};
+    if (gather) SPI_TRY(gather_dev(gather, *shape, &g));
     SPI_TRY(check_ws(workspace));
     DeviceInfo d;
     SPI_TRY(check_device(&d));
     const WsLayout w = layout(*shape, d.num_sms);
     return from_cuda(launch_verify_greedy(*shape, w, logits, tree_tokens, parent, n_nodes, accepted_nodes,
                                           accepted_tokens, n_accepted, reinterpret_cast<char *>(workspace),
-                                          (cudaStream_t)stream));
+                                          (cudaStream_t)stream, gather ? &g : nullptr));
+}
+
+specinfer_status_t specinfer_verify_greedy(const specinfer_shape_t *shape, const float *logits,
+                                           const int32_t *tree_tokens, const int32_t *parent, const int32_t *n_nodes,
+                                           int32_t *accepted_nodes, int32_t *accepted_tokens, int32_t *n_accepted,
+                                           void *workspace, specinfer_stream_t stream) {
+    return specinfer_verify_greedy_ex(shape, logits, tree_tokens, parent, n_nodes, accepted_nodes, accepted_tokens,
+                                      n_accepted, workspace, nullptr, stream);
+}
+
+specinfer_status_t specinfer_verify_mss_ex(const specinfer_shape_t *shape, const float *logits,
+                                           const int32_t *tree_tokens, const int32_t *parent, const int32_t *n_nodes,
+                                           const float *draft_probs, float temperature, uint64_t seed, uint64_t offset,
+                                           const int32_t *request_ids, int32_t *accepted_nodes,
+                                           int32_t *accepted_tokens, int32_t *n_accepted, void *workspace,
+                                           const specinfer_gather_t *gather, specinfer_stream_t stream) {
+    SPI_TRY(check_shape(shape));
+    if (shape->vocab < 1 || !(temperature > 0.f) || !isfinite(temperature)) return SPECINFER_ERR_INVALID_ARG;
+    if (!logits || !tree_tokens || !parent || !n_nodes || !draft_probs || !accepted_nodes || !accepted_tokens ||
+        !n_accepted)
+        return SPECINFER_ERR_INVALID_ARG;
+    if (misaligned16(logits, draft_probs)) return SPECINFER_ERR_INVALID_ARG;
+    GatherDev g{};
+    if (gather) SPI_TRY(gather_dev(gather, *shape, &g));
+    SPI_TRY(check_ws(workspace));
+    DeviceInfo d;
+    SPI_TRY(check_device(&d));
+    const WsLayout w = layout(*shape, d.num_sms);
+    return from_cuda(launch_verify_mss(*shape, w, logits, tree_tokens, parent, n_nodes, draft_probs, temperature,
+                                       seed, offset, request_ids, accepted_nodes, accepted_tokens, n_accepted,
+                                       reinterpret_cast<char *>(workspace), (cudaStream_t)stream,
+                                       gather ? &g : nullptr));
 }
 
 specinfer_status_t specinfer_verify_mss(const specinfer_shape_t *shape, const float *logits,
@@ -269,19 +327,22 @@ specinfer_status_t specinfer_verify_mss(const specinfer_shape_t *shape, const fl
                                         const int32_t *request_ids, int32_t *accepted_nodes,
                                         int32_t *accepted_tokens, int32_t *n_accepted, void *workspace,
                                         specinfer_stream_t stream) {
-    SPI_TRY(check_shape(shape));
-    if (shape->vocab < 1 || !(temperature > 0.f) || !isfinite(temperature)) return SPECINFER_ERR_INVALID_ARG;
-    if (!logits || !tree_tokens || !parent || !n_nodes || !draft_probs || !accepted_nodes || !accepted_tokens ||
-        !n_accepted)
-        return SPECINFER_ERR_INVALID_ARG;
-    if (misaligned16(logits, draft_probs)) return SPECINFER_ERR_INVALID_ARG;
-    SPI_TRY(check_ws(workspace));
+    return specinfer_verify_mss_ex(shape, logits, tree_tokens, parent, n_nodes, draft_probs, temperature, seed, offset,
+                                   request_ids, accepted_nodes, accepted_tokens, n_accepted, workspace, nullptr,
+                                   stream);
+}
+
+specinfer_status_t specinfer_gather_wait(const specinfer_gather_t *gather, int32_t *table_out,
+                                         specinfer_stream_t stream) {
+    if (!gather) return SPECINFER_ERR_INVALID_ARG;
+    specinfer_shape_t s{};
+    s.batch = 1;
+    s.max_depth = (gather->row_len - 3) / 2;
+    GatherDev g{};
+    SPI_TRY(gather_dev(gather, s, &g));
     DeviceInfo d;
     SPI_TRY(check_device(&d));
-    const WsLayout w = layout(*shape, d.num_sms);
-    return from_cuda(launch_verify_mss(*shape, w, logits, tree_tokens, parent, n_nodes, draft_probs, temperature,
-                                       seed, offset, request_ids, accepted_nodes, accepted_tokens, n_accepted,
-                                       reinterpret_cast<char *>(workspace), (cudaStream_t)stream));
+    return from_cuda(launch_gather_wait(g, table_out, (cudaStream_t)stream));
 }
 
 specinfer_status_t specinfer_verify_ns(const specinfer_shape_t *shape, const float *logits,
@@ -461,6 +522,8 @@ int32_t specinfer_launches_per_call(const char *name) {
     if (!strcmp(name, "tree_attention_ex")) return 1;
     if (!strcmp(name, "verify_greedy")) return 1;    // argmax + walk fused (last CTA walks)
     if (!strcmp(name, "verify_mss")) return 1;
+    if (!strcmp(name, "verify_greedy_ex") || !strcmp(name, "verify_mss_ex")) return 1;  // gather fused
+    if (!strcmp(name, "gather_wait")) return 1;
     if (!strcmp(name, "kv_commit")) return 2;        // copy, prefix update
     if (!strcmp(name, "leaf_paths")) return 1;
     if (!strcmp(name, "verify_ns")) return 1;

@@ -18,6 +18,7 @@
 // counters from the global request id, node, round, offset; readings R9, R15) makes the result
 // independent of batching and GPU count.
 #include "common.cuh"
+#include "gather.cuh"
 
 namespace specinfer {
 
@@ -199,7 +200,7 @@ __global__ void __launch_bounds__(kGreedyThreads) verify_greedy_kernel(
     const int32_t *__restrict__ parent, const int32_t *__restrict__ n_nodes,
     const int32_t *__restrict__ req_ok, int32_t *__restrict__ argmax_ws,
     uint32_t *__restrict__ counter, int32_t *__restrict__ acc_nodes, int32_t *__restrict__ acc_tokens,
-    int32_t *__restrict__ n_acc, int Nmax, int V, int path_len, NsParams ns) {
+    int32_t *__restrict__ n_acc, int Nmax, int V, int path_len, NsParams ns, GatherDev g) {
     const int u = blockIdx.x, b = blockIdx.y;
     const int n = n_nodes[b];
     __shared__ ArgMax sh[32];
@@ -211,6 +212,9 @@ __global__ void __launch_bounds__(kGreedyThreads) verify_greedy_kernel(
                 acc_tokens[(size_t)b * path_len + j] = -1;
             }
             if (threadIdx.x == 0) n_acc[b] = 0;
+            __syncthreads();
+            if (threadIdx.x < 32)   // an invalid request still publishes its (empty) row
+                gather_publish(g, b, 0, acc_nodes + (size_t)b * path_len, acc_tokens + (size_t)b * path_len, path_len);
         }
         return;
     }
@@ -289,6 +293,8 @@ __global__ void __launch_bounds__(kGreedyThreads) verify_greedy_kernel(
         n_acc[b] = cnt + 1;
         counter[b] = 0u;  // reusable by the next call on this workspace
     }
+    __syncwarp();
+    gather_publish(g, b, cnt + 1, an, at, path_len);   // NEXT-4a (no-op without a gather)
 }
 
 // ------------------------------------------------------------------------------------------
@@ -435,7 +441,8 @@ __global__ void __launch_bounds__(kMssThreads) verify_mss_kernel(
     const float *__restrict__ draft_probs, const int32_t *__restrict__ req_ok, float temperature,
     uint32_t seed_lo, uint32_t seed_hi, uint32_t off, const int32_t *__restrict__ request_ids,
     float *__restrict__ pbuf_all, int32_t *__restrict__ acc_nodes, int32_t *__restrict__ acc_tokens,
-    int32_t *__restrict__ n_acc, int Nmax, int V, int path_len, unsigned long long *__restrict__ trace) {
+    int32_t *__restrict__ n_acc, int Nmax, int V, int path_len, unsigned long long *__restrict__ trace,
+    GatherDev g) {
     const int b = blockIdx.y;
     const int tid = threadIdx.x;
     __shared__ MssPart s_slot[2], s_result;
@@ -462,7 +469,11 @@ __global__ void __launch_bounds__(kMssThreads) verify_mss_kernel(
             at[j] = -1;
         }
     if (!req_ok[b]) {  // uniform over the cluster
-        if (leader && tid == 0) n_acc[b] = 0;
+        if (leader) {
+            if (tid == 0) n_acc[b] = 0;
+            __syncthreads();
+            if (tid < 32) gather_publish(g, b, 0, an, at, path_len);   // its (empty) row
+        }
         return;
     }
     const int n = n_nodes[b];
@@ -665,6 +676,10 @@ __global__ void __launch_bounds__(kMssThreads) verify_mss_kernel(
     }
     if (leader && tid == 0) n_acc[b] = cnt + 1;
     TR(63);
+    if (leader) {
+        __syncthreads();
+        if (tid < 32) gather_publish(g, b, cnt + 1, an, at, path_len);   // NEXT-4a (no-op without a gather)
+    }
     cluster_sync_all();  // no CTA leaves while others may still read its DSMEM slots
 }
 
@@ -677,12 +692,12 @@ static unsigned long long *const g_mss_trace = nullptr;  // production: no MSS t
 cudaError_t launch_verify_greedy(const specinfer_shape_t &s, const WsLayout &w, const float *logits,
                                  const int32_t *tree_tokens, const int32_t *parent, const int32_t *n_nodes,
                                  int32_t *acc_nodes, int32_t *acc_tokens, int32_t *n_acc, char *ws,
-                                 cudaStream_t stream) {
+                                 cudaStream_t stream, const GatherDev *gather) {
     dim3 grid(s.max_nodes, s.batch);
     verify_greedy_kernel<false><<<grid, kGreedyThreads, 0, stream>>>(
         logits, tree_tokens, parent, n_nodes, reinterpret_cast<const int32_t *>(ws + w.req_ok),
         reinterpret_cast<int32_t *>(ws + w.argmax), reinterpret_cast<uint32_t *>(ws + w.verify_cnt), acc_nodes,
-        acc_tokens, n_acc, s.max_nodes, s.vocab, s.max_depth + 1, NsParams{});
+        acc_tokens, n_acc, s.max_nodes, s.vocab, s.max_depth + 1, NsParams{}, gather ? *gather : GatherDev{});
     return cudaGetLastError();
 }
 
@@ -696,7 +711,7 @@ cudaError_t launch_verify_ns(const specinfer_shape_t &s, const WsLayout &w, cons
     verify_greedy_kernel<true><<<grid, kGreedyThreads, 0, stream>>>(
         logits, tree_tokens, parent, n_nodes, reinterpret_cast<const int32_t *>(ws + w.req_ok),
         reinterpret_cast<int32_t *>(ws + w.argmax), reinterpret_cast<uint32_t *>(ws + w.verify_cnt), acc_nodes,
-        acc_tokens, n_acc, s.max_nodes, s.vocab, s.max_depth + 1, ns);
+        acc_tokens, n_acc, s.max_nodes, s.vocab, s.max_depth + 1, ns, GatherDev{});
     return cudaGetLastError();
 }
 
@@ -704,7 +719,7 @@ cudaError_t launch_verify_mss(const specinfer_shape_t &s, const WsLayout &w, con
                               const int32_t *tree_tokens, const int32_t *parent, const int32_t *n_nodes,
                               const float *draft_probs, float temperature, uint64_t seed, uint64_t offset,
                               const int32_t *request_ids, int32_t *acc_nodes, int32_t *acc_tokens,
-                              int32_t *n_acc, char *ws, cudaStream_t stream) {
+                              int32_t *n_acc, char *ws, cudaStream_t stream, const GatherDev *gather) {
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(kMssCluster, s.batch);
     cfg.blockDim = dim3(kMssThreads);
@@ -721,7 +736,39 @@ cudaError_t launch_verify_mss(const specinfer_shape_t &s, const WsLayout &w, con
                               reinterpret_cast<const int32_t *>(ws + w.req_ok), temperature, (uint32_t)seed,
                               (uint32_t)(seed >> 32), (uint32_t)offset, request_ids,
                               reinterpret_cast<float *>(ws + w.mss_p), acc_nodes, acc_tokens, n_acc, s.max_nodes,
-                              s.vocab, s.max_depth + 1, g_mss_trace);
+                              s.vocab, s.max_depth + 1, g_mss_trace, gather ? *gather : GatherDev{});
+}
+
+// NEXT-4a: waits until every rank published this epoch's rows here, copies the table to table_out
+// (a fixed address for the consumers: the buffer alternates by epoch parity) and advances the epoch
+__global__ void __launch_bounds__(256) gather_wait_kernel(GatherDev g, int32_t *__restrict__ table_out) {
+    const uint32_t e = ld_volatile_u32(g.state) + 1u;
+    if ((int)threadIdx.x < g.world) {
+        const uint32_t *f = g.flags[g.rank] + threadIdx.x;
+        if (ld_acquire_sys(f) < e) {
+            const long long t0 = clock64();
+            while (ld_acquire_sys(f) < e) {
+                if (clock64() - t0 > SPECINFER_WATCHDOG_CYCLES) {
+                    printf("specinfer: gather_wait timeout rank %d waiting for rank %d epoch %u\n", g.rank,
+                           (int)threadIdx.x, e);
+                    __trap();
+                }
+            }
+        }
+    }
+    __syncthreads();
+    __threadfence_system();
+    const size_t n = (size_t)g.world * g.rows_per_rank * g.row_len;
+    const int32_t *src = g.recv[g.rank] + (size_t)((e - 1u) & 1u) * n;
+    if (table_out != nullptr)
+        for (size_t i = threadIdx.x; i < n; i += blockDim.x) table_out[i] = __ldcv(src + i);
+    __syncthreads();
+    if (threadIdx.x == 0) g.state[0] = e;
+}
+
+cudaError_t launch_gather_wait(const GatherDev &g, int32_t *table_out, cudaStream_t stream) {
+    gather_wait_kernel<<<1, 256, 0, stream>>>(g, table_out);
+    return cudaGetLastError();
 }
 
 cudaError_t launch_philox_debug(const uint32_t *ck, uint32_t *out, int n, cudaStream_t stream) {

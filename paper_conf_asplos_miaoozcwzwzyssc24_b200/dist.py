@@ -105,3 +105,54 @@ class GatherPlan:
     def rows_of_all(self) -> torch.Tensor:
         """[batch_global][2Lp+1] packed rows of every request in global order."""
         return self.recv.index_select(0, self.index)
+
+
+class P2PGather:
+    """NEXT-4a: one rank's buffers for the verifier-fused gather (include/specinfer.h,
+    specinfer_gather_t) and the peer mappings of every other rank's buffers (CUDA IPC: over
+    NVLink / NVSwitch between GPUs, plain device memory between processes on one GPU).
+
+    `exchange(obj) -> [obj of rank 0, ..., obj of rank world-1]` shares picklable objects between the
+    ranks (torch.distributed.all_gather_object, or queues in a test).  The row layout is GatherPlan's:
+    request b of rank r at row r * pad + b, so GatherPlan.index selects the global requests."""
+
+    def __init__(self, batch_global: int, world: int, rank: int, path_len: int, device, exchange=None):
+        from torch.multiprocessing.reductions import reduce_tensor
+        import paper_conf_asplos_miaoozcwzwzyssc24_b200 as spi
+        if world > spi.MAX_PEERS:
+            raise ValueError(f"P2PGather: at most {spi.MAX_PEERS} ranks")
+        self.world, self.rank, self.B = world, rank, batch_global
+        self.pad = -(-batch_global // world)
+        self.row_len = 2 * path_len + 1
+        i32 = dict(dtype=torch.int32, device=device)
+        self.recv = torch.zeros((2, world * self.pad, self.row_len), **i32)
+        self.flags = torch.zeros((world,), **i32)
+        self.state = torch.zeros((2,), **i32)
+        self.table = torch.zeros((world * self.pad, self.row_len), **i32)
+        if world > 1:
+            objs = exchange((reduce_tensor(self.recv), reduce_tensor(self.flags)))
+            self.peers = []
+            for r, ((f1, a1), (f2, a2)) in enumerate(objs):
+                self.peers.append((self.recv, self.flags) if r == rank else (f1(*a1), f2(*a2)))
+        else:
+            self.peers = [(self.recv, self.flags)]
+        d = spi.GatherDesc()
+        d.world, d.rank, d.rows_per_rank, d.row_len = world, rank, self.pad, self.row_len
+        for r, (rv, fl) in enumerate(self.peers):
+            d.recv[r] = rv.data_ptr()
+            d.flags[r] = fl.data_ptr()
+        d.state = self.state.data_ptr()
+        self.desc = d
+        self.spi = spi
+
+    def wait(self):
+        """Device-side wait for this step's rows of every rank; returns the table (global order via
+        GatherPlan.index)."""
+        self.spi.specinfer_gather_wait(self.desc, self.table)
+        return self.table
+
+
+def all_gather_object_exchange(obj):
+    out = [None] * torch.distributed.get_world_size()
+    torch.distributed.all_gather_object(out, obj)
+    return out

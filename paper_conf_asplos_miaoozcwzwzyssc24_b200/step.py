@@ -77,13 +77,14 @@ class DeviceOps:
     def attention(self, st, q, k, v, out, prefetch: bool):
         st.attention(q, k, v, out, prefetch=prefetch)
 
-    def verify_greedy(self, shape, st, logits, tokens, parent, n_nodes, an, at, na):
-        self.spi.specinfer_verify_greedy(shape, logits, tokens, parent, n_nodes, an, at, na, st.workspace)
+    def verify_greedy(self, shape, st, logits, tokens, parent, n_nodes, an, at, na, gather=None):
+        self.spi.specinfer_verify_greedy(shape, logits, tokens, parent, n_nodes, an, at, na, st.workspace,
+                                         gather=gather)
 
     def verify_mss(self, shape, st, logits, tokens, parent, n_nodes, draft, temperature, seed, offset, rids, an, at,
-                   na):
+                   na, gather=None):
         self.spi.specinfer_verify_mss(shape, logits, tokens, parent, n_nodes, draft, temperature, seed, offset, rids,
-                                      an, at, na, st.workspace)
+                                      an, at, na, st.workspace, gather=gather)
 
     def kv_commit(self, shape, k_all, v_all, prefix_len, an, na):
         self.spi.specinfer_kv_commit(shape, k_all, v_all, prefix_len, an, na)
@@ -95,7 +96,10 @@ class VerifyStep:
     verification batch (layout.verify_ids); with request sharding they are the same tensors."""
 
     def __init__(self, ops, layout: Layout, shape_attn, shape_verify, attn_tree: Tuple, verify_tree: Tuple,
-                 modes: Sequence[str], path_len: int, device, commit_mode: Optional[str] = None):
+                 modes: Sequence[str], path_len: int, device, commit_mode: Optional[str] = None,
+                 p2p: Optional["D.P2PGather"] = None):
+        """p2p: NEXT-4a, the committed verifier publishes its rows to every rank itself (peer stores +
+        flags) and gather() is a device-side wait; None: the NCCL / gloo all-gather (GatherPlan)."""
         self.ops, self.layout = ops, layout
         self.shape_attn, self.shape_verify = shape_attn, shape_verify
         self.attn_tree, self.verify_tree = attn_tree, verify_tree
@@ -112,6 +116,7 @@ class VerifyStep:
                         torch.zeros((B,), **i32)) for m in self.modes}   # (nodes, tokens, n) per verifier
         self.rids = torch.arange(layout.req_lo, layout.req_lo + B, **i32)
         self.plan = D.GatherPlan(layout.batch_global, layout.world, path_len, device)
+        self.p2p = p2p
         self.an_all = torch.zeros((layout.batch_global, path_len), **i32)
         self.na_all = torch.zeros((layout.batch_global,), **i32)
         self._layer = 0
@@ -138,25 +143,29 @@ class VerifyStep:
         for m in self.modes:
             an, at, na = self.res[m]
             logits, tokens, draft = inputs[m]
+            kw = {"gather": self.p2p.desc} if (self.p2p is not None and m == self.commit_mode) else {}
             if m == "greedy":
-                self.ops.verify_greedy(self.shape_verify, self.st_v, logits, tokens, parent, n_nodes, an, at, na)
+                self.ops.verify_greedy(self.shape_verify, self.st_v, logits, tokens, parent, n_nodes, an, at, na, **kw)
             else:
                 self.ops.verify_mss(self.shape_verify, self.st_v, logits, tokens, parent, n_nodes, draft,
-                                    temperature, seed, offset, self.rids, an, at, na)
+                                    temperature, seed, offset, self.rids, an, at, na, **kw)
 
     # ---- a7 ----
     def gather(self):
         """Tokens-only all-gather of the committed verifier's rows (n | tokens | nodes); at N = 1 a
         copy, so the kv-sharded path is exercised on one GPU too."""
-        an, at, na = self.res[self.commit_mode]
-        self.plan.pack(na, at, an)
-        self.plan.exchange()
+        if self.p2p is not None:
+            table = self.p2p.wait()          # the verifier already stored the rows on every rank
+        else:
+            an, at, na = self.res[self.commit_mode]
+            self.plan.pack(na, at, an)
+            table = self.plan.exchange()
         if self.layout.kv_shard:
-            rows = self.plan.rows_of_all()
+            rows = table.index_select(0, self.plan.index)
             n_all, _, nodes_all = D.unpack_accepted(rows)
             self.na_all.copy_(n_all)
             self.an_all.copy_(nodes_all)
-        return self.plan.recv
+        return table
 
     # ---- a6 ----
     def commit(self, k_all, v_all):
@@ -175,4 +184,5 @@ class VerifyStep:
 
     def accepted_all(self) -> torch.Tensor:
         """Packed rows of every global request after gather() (global order)."""
-        return self.plan.rows_of_all()
+        table = self.p2p.table if self.p2p is not None else self.plan.recv
+        return table.index_select(0, self.plan.index)
