@@ -2,20 +2,22 @@
 // per kv-head), sm_100a.  Same computation and schedule as tree_attention.cu (Def. 4.1
 // L594-598, Eq. 1-4, topology-aware mask L645-674), different tiling:
 //  * a work item is (request, kv-head, block of 128 query rows); the UMMA M dimension is the query
-//    rows (one TMEM lane per row), N = 128 keys for S = Q K^T and N = 128 dims for O += P V, so the
-//    MMAs run at full rate (N = 128) instead of the A-read-bound N <= 64 of the swapped kernel;
-//  * two softmax groups of 4 warps own alternate KV tiles (tile parity), each with its own S
-//    buffer, O accumulator and running (m, l) per row, merged by log-sum-exp at the segment end:
-//    the groups run out of phase, so one group's TMEM / barrier latency hides behind the other's
-//    exponentials; every row's softmax is thread-local (exact tile max, stale running max with a
-//    2^8 tolerance, O row rescaled in TMEM by its own thread when it moves);
-//  * P (bf16 pairs) is written over the first 64 columns of its own S buffer and feeds the PV
-//    MMA as the A operand ("TS" form): TMEM = S0 S1 O0 O1, smem holds only Q and the K / V rings;
+//    rows (one TMEM lane per row), N = 128 keys for S = Q K^T and N = 128 dims for O += P V;
+//  * TMEM = S0 | S1 | O | P0 | P1 (128 + 128 + 128 + 64 + 64 columns): S double-buffered, ONE O
+//    accumulator, P (bf16 pairs) in its own columns, so the S buffer of tile t is free as soon as
+//    the softmax has loaded it and S(t + 2) never waits for PV(t) (round 1 aliased P over S and the
+//    chain S -> softmax -> PV -> S(t + 2) bounded the kernel);
+//  * 8 softmax warps, two per TMEM lane quarter: thread (row r, half h) owns keys [64 h, 64 h + 64)
+//    of every tile and dims [64 h, 64 h + 64) of O; the two halves of a row exchange their partial
+//    tile maxima through shared memory (one 64-thread barrier per tile), so both hold the same
+//    stale running max; O is rescaled in TMEM (after PV(t - 1)) only when a tile raises a row's
+//    max by more than 2^8;
+//  * K and V in separate TMA rings fed by two producer lanes; S issuer and PV issuer threads;
 //  * lane mode (schedule_kernel): the row blocks of one (request, kv-head) run on `lanes` CTAs in
 //    lock-step over the same tile range, so each KV tile is read from HBM once;
 //  * tree keys are masked with the ancestor-or-self bitset of the row's node (tree_prepare);
-//  * the stream-K schedule, producers, segment ring, row-exact tail loads, split combine and PDL
-//    are shared with the swapped kernel (attn_shared.cuh).
+//  * the stream-K schedule, segment descriptors, row-exact tail loads, split combine and PDL are
+//    shared with the swapped kernel (attn_shared.cuh).
 #include "attn_shared.cuh"
 
 namespace specinfer {
@@ -24,21 +26,22 @@ namespace rows {
 
 constexpr int RB = kRowsBlock;              // 128 query rows per item
 constexpr int kQBuf = 2 * RB * 128;          // one Q buffer: 2 halves x 128 rows x 128 B
-constexpr int kTmemCols = 512;               // S0 S1 (P aliased over S) | O0 O1
-constexpr int kColS = 0, kColO = 256;
-
-constexpr int kMaxRing = 6;                  // unified K/V tile ring (slots of 32 KB)
+constexpr int kTmemCols = 512;
+constexpr int kColS = 0, kColO = 256, kColP = 384;
+constexpr int kMaxK = 4, kMaxV = 4;          // ring slots (the launch picks 3 K + 2 V)
 
 struct Misc {
-    uint64_t full[kMaxRing], empty[kMaxRing];
+    uint64_t k_full[kMaxK], k_empty[kMaxK];
+    uint64_t v_full[kMaxV], v_empty[kMaxV];
     uint64_t q_full[2], q_empty[2];
-    uint64_t s_full[2];
-    uint64_t p_full[2], p_empty[2];
+    uint64_t s_full[2], s_free[2];           // S(t) ready / S buffer t & 1 loaded by the softmax
+    uint64_t p_full[2], pv_done[2];          // P(t) written / PV(t) complete (P buffer free, O advanced)
+    uint64_t o_free;                         // the epilogue has read O (next segment may overwrite it)
     uint64_t seg_full[kSegRing];
     SegDesc seg[kSegRing];
     uint32_t tmem_base;
     int32_t bcast;
-    float2 xch[RB];        // [row] (m, l) exchange between the two softmax groups at a segment's end
+    float xm[2][2][RB];                      // [0][0]: row references; [1][0] / [1][1]: segment-end hand-over
 };
 
 __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
@@ -63,64 +66,65 @@ __device__ __forceinline__ void umma_bf16_ts(uint32_t d_tmem, uint32_t a_tmem, u
         : "memory");
 }
 
-// Row max of one 128-key S tile (this thread's TMEM lane), optionally under the visibility mask.
-template <bool kMask>
-__device__ __forceinline__ void tile_max(uint32_t s_col, const uint32_t (&vis)[4], float (&tm4)[4]) {
-#pragma unroll
-    for (int h = 0; h < 2; ++h) {
-        uint32_t v[2][32];
-        tmem_ld32(s_col + h * 64, v[0]);
-        tmem_ld32(s_col + h * 64 + 32, v[1]);
-        tmem_ld_wait();
-#pragma unroll
-        for (int q = 0; q < 2; ++q) {
-#pragma unroll
-            for (int i = 0; i < 32; ++i) {
-                float x = __uint_as_float(v[q][i]);
-                if (kMask) x = ((vis[2 * h + q] >> i) & 1u) ? x : -INFINITY;
-                tm4[i & 3] = fmaxf(tm4[i & 3], x);
-            }
-        }
-    }
+// 2^x for a pair of x <= 8 on the FMA/ALU pipes (round-to-nearest split x = n + f, f in [-1/2, 1/2],
+// degree-4 Taylor polynomial of 2^f: relative error < 5e-5, far below the bf16 rounding of P)
+__device__ __forceinline__ uint64_t exp2_poly2(uint64_t x2) {
+    const float x0 = fmaxf(__uint_as_float((uint32_t)x2), -126.f);
+    const float x1 = fmaxf(__uint_as_float((uint32_t)(x2 >> 32)), -126.f);
+    const uint64_t xm = f2_bits(x0, x1);
+    const uint64_t magic = f2_bits(12582912.f, 12582912.f);   // 1.5 * 2^23: rint via the fp adder
+    const uint64_t t = fadd2(xm, magic);
+    const uint64_t nf = fadd2(t, f2_bits(-12582912.f, -12582912.f));
+    const uint64_t f = fadd2(xm, nf ^ 0x8000000080000000ull);   // x - n
+    uint64_t q = f2_bits(0.009618129f, 0.009618129f);
+    q = ffma2(q, f, f2_bits(0.05550411f, 0.05550411f));
+    q = ffma2(q, f, f2_bits(0.2402265f, 0.2402265f));
+    q = ffma2(q, f, f2_bits(0.6931472f, 0.6931472f));
+    q = ffma2(q, f, f2_bits(1.f, 1.f));
+    const uint32_t n0 = (uint32_t)t - 0x4B400000u, n1 = (uint32_t)(t >> 32) - 0x4B400000u;
+    return (uint64_t)((uint32_t)q + (n0 << 23)) | ((uint64_t)((uint32_t)(q >> 32) + (n1 << 23)) << 32);
 }
 
-// P = 2^(s * scale_log2 - mref) of one S tile, packed to bf16 pairs over the first 64 columns of the
-// same TMEM buffer; accumulates the fp32 row sum.
-template <bool kMask>
-__device__ __forceinline__ void tile_exp(uint32_t s_col, const uint32_t (&vis)[4], float scale_log2, float mref,
-                                         float (&l4)[4]) {
-    const uint64_t sc2 = f2_bits(scale_log2, scale_log2), nm2 = f2_bits(-mref, -mref);
-    uint64_t la = f2_bits(0.f, 0.f), lb = f2_bits(0.f, 0.f);  // paired row-sum accumulators
+// P = 2^(s * scale_log2 - mref) of 32 keys as 16 bf16 pairs (into w, not yet stored); returns the fp32
+// sum of the bf16-ROUNDED values, so the normalisation matches the numerator the PV MMA computes.
+// kMax: also the max of the (raw) s values, for the deferred stale-max check.
+template <bool kMax>
+__device__ __forceinline__ float exp32(const uint32_t (&v)[32], uint64_t sc2, uint64_t nm2, uint32_t (&w)[16],
+                                       float &pm) {
+    uint64_t la = f2_bits(0.f, 0.f), lb = f2_bits(0.f, 0.f);
+    float m2[2] = {-INFINITY, -INFINITY};
 #pragma unroll
-    for (int h = 0; h < 2; ++h) {
-        uint32_t v[2][32];
-        tmem_ld32(s_col + h * 64, v[0]);
-        tmem_ld32(s_col + h * 64 + 32, v[1]);
-        tmem_ld_wait();
-#pragma unroll
-        for (int q = 0; q < 2; ++q) {
-            uint32_t w16[16];
-#pragma unroll
-            for (int i = 0; i < 16; ++i) {
-                float x0 = __uint_as_float(v[q][2 * i]), x1 = __uint_as_float(v[q][2 * i + 1]);
-                if (kMask) {
-                    x0 = ((vis[2 * h + q] >> (2 * i)) & 1u) ? x0 : -INFINITY;
-                    x1 = ((vis[2 * h + q] >> (2 * i + 1)) & 1u) ? x1 : -INFINITY;
-                }
-                const uint64_t y = ffma2(f2_bits(x0, x1), sc2, nm2);
-                const float e0 = ex2(__uint_as_float((uint32_t)y));
-                const float e1 = ex2(__uint_as_float((uint32_t)(y >> 32)));
-                w16[i] = pack_bf16x2(e0, e1);
-                if (i & 1) lb = fadd2(lb, f2_bits(e0, e1));
-                else la = fadd2(la, f2_bits(e0, e1));
-            }
-            tmem_st16(s_col + (2 * h + q) * 16, w16);
+    for (int i = 0; i < 16; ++i) {
+        const float x0 = __uint_as_float(v[2 * i]), x1 = __uint_as_float(v[2 * i + 1]);
+        if (kMax) m2[i & 1] = fmaxf(m2[i & 1], fmaxf(x0, x1));
+        const uint64_t y = ffma2(f2_bits(x0, x1), sc2, nm2);
+        float e0, e1;
+#ifdef ROWS_POLY_EXP
+        if ((i & 3) == 3) {   // a quarter of the exponentials on the FMA pipe (MUFU relief)
+            const uint64_t e = exp2_poly2(y);
+            e0 = __uint_as_float((uint32_t)e);
+            e1 = __uint_as_float((uint32_t)(e >> 32));
+        } else
+#endif
+        {
+            e0 = ex2(__uint_as_float((uint32_t)y));
+            e1 = ex2(__uint_as_float((uint32_t)(y >> 32)));
         }
+        w[i] = pack_bf16x2(e0, e1);
+        const uint64_t r2 = f2_bits(__uint_as_float(w[i] << 16), __uint_as_float(w[i] & 0xFFFF0000u));
+        if (i & 1) lb = fadd2(lb, r2);
+        else la = fadd2(la, r2);
     }
-    l4[0] += __uint_as_float((uint32_t)la);
-    l4[1] += __uint_as_float((uint32_t)(la >> 32));
-    l4[2] += __uint_as_float((uint32_t)lb);
-    l4[3] += __uint_as_float((uint32_t)(lb >> 32));
+    if (kMax) pm = fmaxf(pm, fmaxf(m2[0], m2[1]));
+    const uint64_t s = fadd2(la, lb);
+    return __uint_as_float((uint32_t)s) + __uint_as_float((uint32_t)(s >> 32));
+}
+
+// masks 32 S values in place (invisible -> -inf)
+__device__ __forceinline__ void mask32(uint32_t (&v)[32], uint32_t vis) {
+#pragma unroll
+    for (int i = 0; i < 32; ++i)
+        if (!((vis >> i) & 1u)) v[i] = __float_as_uint(-INFINITY);
 }
 
 }  // namespace rows
@@ -136,9 +140,10 @@ __global__ void __launch_bounds__(352, 1)
     // the launch budgets no alignment slack, so a misaligned base is a hard error
     extern __shared__ __align__(1024) uint8_t smem[];
     if ((smem_u32(smem) & 1023u) != 0u) __trap();
-    const int NS = p.nk_slots;                 // unified ring: K and V tiles in MMA consumption order
-    uint8_t *s_ring = smem;
-    uint8_t *s_q = s_ring + (size_t)NS * kSlotBytes;
+    const int NK = p.nk_slots, NV = p.nv_slots;
+    uint8_t *s_k = smem;
+    uint8_t *s_v = s_k + (size_t)NK * kSlotBytes;
+    uint8_t *s_q = s_v + (size_t)NV * kSlotBytes;
     Misc *misc = reinterpret_cast<Misc *>(s_q + 2 * kQBuf);
 
     const int warp = threadIdx.x >> 5;
@@ -148,17 +153,23 @@ __global__ void __launch_bounds__(352, 1)
     if (threadIdx.x == 0) SPI_TRACE_K(0);
 
     if (threadIdx.x == 0) {
-        for (int i = 0; i < NS; ++i) {
-            mbar_init(&misc->full[i], 1);
-            mbar_init(&misc->empty[i], 1);
+        for (int i = 0; i < NK; ++i) {
+            mbar_init(&misc->k_full[i], 1);
+            mbar_init(&misc->k_empty[i], 1);
+        }
+        for (int i = 0; i < NV; ++i) {
+            mbar_init(&misc->v_full[i], 1);
+            mbar_init(&misc->v_empty[i], 1);
         }
         for (int i = 0; i < 2; ++i) {
             mbar_init(&misc->q_full[i], 1);
             mbar_init(&misc->q_empty[i], 1);
             mbar_init(&misc->s_full[i], 1);
+            mbar_init(&misc->s_free[i], 4);
             mbar_init(&misc->p_full[i], 4);
-            mbar_init(&misc->p_empty[i], 1);
+            mbar_init(&misc->pv_done[i], 1);
         }
+        mbar_init(&misc->o_free, 4);
         for (int i = 0; i < kSegRing; ++i) mbar_init(&misc->seg_full[i], 1);
         fence_barrier_init();
     }
@@ -172,8 +183,8 @@ __global__ void __launch_bounds__(352, 1)
         for (int i = threadIdx.x - 96; i < 2 * kQBuf / 16; i += 256)
             reinterpret_cast<uint4 *>(s_q)[i] = make_uint4(0, 0, 0, 0);
         // rows past a request's last key are never loaded: slots must hold finite data (0 * NaN)
-        for (int i = threadIdx.x - 96; i < NS * kSlotBytes / 16; i += 256)
-            reinterpret_cast<uint4 *>(s_ring)[i] = make_uint4(0, 0, 0, 0);
+        for (int i = threadIdx.x - 96; i < (NK + NV) * kSlotBytes / 16; i += 256)
+            reinterpret_cast<uint4 *>(s_k)[i] = make_uint4(0, 0, 0, 0);
         fence_proxy_async_smem();
     }
     if (warp == 1) tmem_alloc<kTmemCols>(&misc->tmem_base);
@@ -182,32 +193,59 @@ __global__ void __launch_bounds__(352, 1)
     tc_fence_after();
     const uint32_t tmem = misc->tmem_base;
 
-    grid_dependency_wait();
+    // Programmatic dependent launch (see tree_attention.cu): the producer warp may stage
+    // committed-prefix tiles of its first segment before the dependency resolves (early_prefix)
+    const bool early = p.early_prefix != 0 && warp == 0;
+    if (!early) grid_dependency_wait();
     const int4 ci = __ldg(p.cta_info + 2 * blockIdx.x);
     const int4 first_info = __ldg(p.cta_info + 2 * blockIdx.x + 1);
     const int t0 = ci.x, t1 = ci.y, x_first = ci.z, T = ci.w;
     const int ntiles = t1 - t0;
 
     if (ntiles <= 0) {
-        // no work for this CTA
+        if (early) grid_dependency_wait();
     } else if (warp == 0) {
-        // ============================ TMA producer (one thread) ============================
-        // Loads K and V tiles into one ring in exactly the order the MMA issuer consumes them:
-        // K(0), K(1), then V(j), K(j + 2) for j = 0, 1, ...  (S(lt + 2) follows PV(lt)).  The K
-        // cursor publishes the segment descriptors and loads each segment's Q; the V cursor follows
-        // the published descriptors.
-        // lane mode: the other chunks of the unit read the same tiles shortly after, from L2
+        // ============================ TMA producers ============================
+        // lane 0: segment descriptors, Q and the K ring; lane 1: the V ring (follows the descriptors)
         const uint64_t pol = p.lanes > 1 ? l2_evict_normal_policy() : l2_evict_first_policy();
+        auto issue = [&](const SegDesc &d, int t, int lt, bool is_v) {
+            const int key0 = (t - d.ib) * kKeyTile;
+            const int nv = min(kKeyTile, d.P + d.n - key0);
+            const int row0 = kv_tile_row(p, d.b, d.g, key0);
+            const int NS = is_v ? NV : NK;
+            const int slot = lt % NS, f = lt / NS;
+            if (f >= 1) mbar_wait(is_v ? &misc->v_empty[slot] : &misc->k_empty[slot], (f - 1) & 1);
+            if (!is_v) {
+                SPI_TRACE(0);
+                if (lt == 0) SPI_TRACE_K(2);
+            } else {
+                SPI_TRACE(1);
+            }
+            uint8_t *dst = (is_v ? s_v : s_k) + (size_t)slot * kSlotBytes;
+            uint64_t *bar = is_v ? &misc->v_full[slot] : &misc->k_full[slot];
+            const CUtensorMap *m = is_v ? &tm_v : &tm_k;
+            if (SPI_FLAGS(p) & 1) {  // experiment: no K/V traffic (results invalid)
+                mbar_arrive(bar);
+            } else if (nv == kKeyTile) {
+                mbar_arrive_expect_tx(bar, kSlotBytes);
+                tma_load_2d(dst, m, bar, 0, row0, pol);
+                tma_load_2d(dst + kHalfBytes, m, bar, 64, row0, pol);
+            } else if (is_v) {
+                tma_load_rows(dst, bar, nv, row0, pol, &tm_v16, &tm_v4, &tm_v1);
+            } else {
+                tma_load_rows(dst, bar, nv, row0, pol, &tm_k16, &tm_k4, &tm_k1);
+            }
+        };
+        auto n_early = [&](const SegDesc &d, int NS) {
+            int c = 0;
+            while (c < NS && d.begin + c < d.end && (d.begin + c - d.ib + 1) * kKeyTile <= d.P) ++c;
+            return c;
+        };
         if (lane == 0) {
-            int x = x_first;
+            int x = x_first, ls = 0, lt = 0;
             int4 next_info = first_info;
-            int lsk = 0, lsv = 0;           // segments opened by the K / V cursors
-            int li = 0;                     // ring loads issued
-            SegDesc dk{}, dv{};
-            int tk = 0, tv = 0;
-            bool kdone = false, vdone = false;
-            // next non-empty segment of this CTA's range -> ring slot lsk (terminal if none)
-            auto publish = [&]() {
+            for (;;) {
+                // next non-empty segment of this CTA's range (terminal descriptor if none)
                 SegDesc d{};
                 d.x = -1;
                 for (;; x += p.lanes) {
@@ -229,105 +267,71 @@ __global__ void __launch_bounds__(352, 1)
                     x += p.lanes;
                     break;
                 }
-                misc->seg[lsk % kSegRing] = d;
-                mbar_arrive(&misc->seg_full[lsk % kSegRing]);
-                if (d.x >= 0) {
-                    const int qb = lsk & 1;
-                    if (lsk >= 2) mbar_wait(&misc->q_empty[qb], ((lsk >> 1) - 1) & 1);
-                    mbar_arrive_expect_tx(&misc->q_full[qb], 2u * (uint32_t)(p.G * p.npc) * 128u);
-                    uint8_t *qdst = s_q + qb * kQBuf;
-                    const int node0 = d.b * p.Nmax + d.c * p.npc;
-                    tma_load_3d(qdst, &tm_q, &misc->q_full[qb], 0, d.g * p.G, node0);
-                    tma_load_3d(qdst + RB * 128, &tm_q, &misc->q_full[qb], 64, d.g * p.G, node0);
+                misc->seg[ls % kSegRing] = d;
+                mbar_arrive(&misc->seg_full[ls % kSegRing]);
+                if (d.x < 0) {
+                    if (early && ls == 0) grid_dependency_wait();
+                    break;
                 }
-                dk = d;
-                tk = d.begin;
-                kdone = d.x < 0;
-                ++lsk;
-            };
-            auto open_v = [&]() {
-                dv = misc->seg[lsv % kSegRing];  // published earlier by this thread
-                tv = dv.begin;
-                vdone = dv.x < 0;
-                ++lsv;
-            };
-            // one tile of K (is_v = 0) or V (1) of segment d, tile t, into the next ring slot
-            auto load = [&](const SegDesc &d, int t, bool is_v) {
-                const int Kend = d.P + d.n;
-                const int key0 = (t - d.ib) * kKeyTile;
-                const int nv = min(kKeyTile, Kend - key0);
-                const int row0 = kv_tile_row(p, d.b, d.g, key0);
-                const int slot = li % NS, f = li / NS;
-                if (f >= 1) mbar_wait(&misc->empty[slot], (f - 1) & 1);
-                if (li == 0) SPI_TRACE_K(2);
-                uint8_t *dst = s_ring + (size_t)slot * kSlotBytes;
-                uint64_t *bar = &misc->full[slot];
-                const CUtensorMap *m = is_v ? &tm_v : &tm_k;
-                if (SPI_FLAGS(p) & 1) {  // experiment: no K/V traffic (results invalid)
-                    mbar_arrive(bar);
-                } else if (nv == kKeyTile) {
-                    mbar_arrive_expect_tx(bar, kSlotBytes);
-                    tma_load_2d(dst, m, bar, 0, row0, pol);
-                    tma_load_2d(dst + kHalfBytes, m, bar, 64, row0, pol);
-                } else if (is_v) {
-                    tma_load_rows(dst, bar, nv, row0, pol, &tm_v16, &tm_v4, &tm_v1);
-                } else {
-                    tma_load_rows(dst, bar, nv, row0, pol, &tm_k16, &tm_k4, &tm_k1);
+                int pre = 0;
+                if (early && ls == 0) {
+                    pre = n_early(d, NK);
+                    for (int i = 0; i < pre; ++i) issue(d, d.begin + i, i, false);
+                    grid_dependency_wait();
                 }
-                ++li;
-            };
-            int lt_k = 0, lt_v = 0;
-            auto step_k = [&]() {
-                {
-                    const int lt = lt_k;
-                    SPI_TRACE(0);
-                }
-                load(dk, tk, false);
-                ++lt_k;
-                if (++tk == dk.end) publish();
-            };
-            auto step_v = [&]() {
-                {
-                    const int lt = lt_v;
-                    SPI_TRACE(1);
-                }
-                load(dv, tv, true);
-                ++lt_v;
-                if (++tv == dv.end) open_v();
-            };
-            publish();
-            open_v();
-            for (int i = 0; i < 2 && !kdone; ++i) step_k();
-            while (!vdone) {
-                step_v();
-                if (!kdone) step_k();
+                const int qb = ls & 1;
+                if (ls >= 2) mbar_wait(&misc->q_empty[qb], ((ls >> 1) - 1) & 1);
+                mbar_arrive_expect_tx(&misc->q_full[qb], 2u * (uint32_t)(p.G * p.npc) * 128u);
+                uint8_t *qdst = s_q + qb * kQBuf;
+                const int node0 = d.b * p.Nmax + d.c * p.npc;
+                tma_load_3d(qdst, &tm_q, &misc->q_full[qb], 0, d.g * p.G, node0);
+                tma_load_3d(qdst + RB * 128, &tm_q, &misc->q_full[qb], 64, d.g * p.G, node0);
+                lt += pre;
+                for (int t = d.begin + pre; t < d.end; ++t, ++lt) issue(d, t, lt, false);
+                ++ls;
             }
             grid_launch_dependents();
+        } else if (lane == 1) {
+            int ls = 0, lt = 0;
+            for (;;) {
+                mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
+                const SegDesc d = misc->seg[ls % kSegRing];
+                if (d.x < 0) {
+                    if (early && ls == 0) grid_dependency_wait();
+                    break;
+                }
+                int pre = 0;
+                if (early && ls == 0) {
+                    pre = n_early(d, NV);
+                    for (int i = 0; i < pre; ++i) issue(d, d.begin + i, i, true);
+                    grid_dependency_wait();
+                }
+                lt += pre;
+                for (int t = d.begin + pre; t < d.end; ++t, ++lt) issue(d, t, lt, true);
+                ++ls;
+            }
         }
     } else if (warp == 1) {
-        // ===================== S issuer: S = Q K^T (M = 128 rows, N = 128 keys) =====================
-        // S(lt) goes to buffer lt & 1; P(lt) is written over the same columns, so the buffer is
-        // free again once PV(lt - 2) has completed (p_empty).  K(j) is ring load j (j < 2) or
-        // 2j - 1 (the producer's order K0 K1 V0 K2 V1 K3 ...).
+        // ===================== S issuer: S(t) = Q K(t)^T into S buffer t & 1 =====================
+        // (the buffer is free once the softmax of tile t - 2 has loaded it: s_free)
         if (lane == 0) {
             const uint32_t idesc_s = make_idesc_bf16(128, 128, false, false);
-            const uint32_t ring_addr = smem_u32(s_ring), q_addr = smem_u32(s_q);
+            const uint32_t k_addr = smem_u32(s_k), q_addr = smem_u32(s_q);
             int lt = 0, ls = 0;
-            while (true) {
+            for (;;) {
                 mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
                 const SegDesc d = misc->seg[ls % kSegRing];
                 if (d.x < 0) break;
                 const int qb = ls & 1;
                 mbar_wait(&misc->q_full[qb], (ls >> 1) & 1);
                 for (int t = d.begin; t < d.end; ++t, ++lt) {
-                    const int li = lt < 2 ? lt : 2 * lt - 1;
-                    const int slot = li % NS;
-                    mbar_wait(&misc->full[slot], (li / NS) & 1);
                     const int sb = lt & 1;
-                    if (lt >= 2) mbar_wait(&misc->p_empty[sb], ((lt - 2) >> 1) & 1);
+                    if (lt >= 2) mbar_wait(&misc->s_free[sb], ((lt - 2) >> 1) & 1);
+                    const int slot = lt % NK;
+                    mbar_wait(&misc->k_full[slot], (lt / NK) & 1);
                     tc_fence_after();
                     SPI_TRACE(2);
-                    const uint32_t kbase = ring_addr + slot * kSlotBytes;
+                    const uint32_t kbase = k_addr + slot * kSlotBytes;
                     const uint32_t qbase = q_addr + qb * kQBuf;
 #pragma unroll
                     for (int kk = 0; kk < kHeadDim / 16; ++kk) {
@@ -339,77 +343,68 @@ __global__ void __launch_bounds__(352, 1)
                             umma_bf16_ss(tmem + kColS + sb * 128, adesc, bdesc, idesc_s, kk > 0 ? 1u : 0u);
                     }
                     umma_commit(&misc->s_full[sb]);
-                    umma_commit(&misc->empty[slot]);
+                    umma_commit(&misc->k_empty[slot]);
                     if (t == d.end - 1) umma_commit(&misc->q_empty[qb]);
                 }
                 ++ls;
             }
         }
     } else if (warp == 2) {
-        // ========== PV issuer: O_{lt&1} += P V (A = P in TMEM over S(lt), N = 128 dims) ==========
-        // V(j) is ring load 2j + 2, except the CTA's last tile (2j + 1: no K load follows it).
+        // ============ PV issuer: O += P(t) V(t) (A = P from TMEM, N = 128 dims), in tile order ============
         if (lane == 0) {
             const uint32_t idesc_o = make_idesc_bf16(128, 128, false, true);
-            const uint32_t ring_addr = smem_u32(s_ring);
+            const uint32_t v_addr = smem_u32(s_v);
             int lt = 0, ls = 0;
-            mbar_wait(&misc->seg_full[0], 0);
-            SegDesc d = misc->seg[0];
-            while (d.x >= 0) {
-                SegDesc dn{};
-                bool have_next = false;
+            for (;;) {
+                mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
+                const SegDesc d = misc->seg[ls % kSegRing];
+                if (d.x < 0) break;
                 for (int t = d.begin; t < d.end; ++t, ++lt) {
                     const int pb = lt & 1;
                     mbar_wait(&misc->p_full[pb], (lt >> 1) & 1);
-                    bool last = false;
-                    if (t == d.end - 1) {
-                        // the next descriptor is published right after this segment's last K load
-                        mbar_wait(&misc->seg_full[(ls + 1) % kSegRing], ((ls + 1) / kSegRing) & 1);
-                        dn = misc->seg[(ls + 1) % kSegRing];
-                        have_next = true;
-                        last = dn.x < 0;
-                    }
-                    const int li = last ? 2 * lt + 1 : 2 * lt + 2;
-                    const int slot = li % NS;
-                    mbar_wait(&misc->full[slot], (li / NS) & 1);
+                    const bool first = (t == d.begin);
+                    if (first && ls > 0) mbar_wait(&misc->o_free, (ls - 1) & 1);  // previous segment's O read
+                    const int slot = lt % NV;
+                    mbar_wait(&misc->v_full[slot], (lt / NV) & 1);
                     tc_fence_after();
                     SPI_TRACE(3);
-                    const uint32_t vbase = ring_addr + slot * kSlotBytes;
-                    const bool first = (t - d.begin) < 2;  // first tile of group pb in this segment
+                    const uint32_t vbase = v_addr + slot * kSlotBytes;
 #pragma unroll
                     for (int kk = 0; kk < kKeyTile / 16; ++kk) {
                         const uint64_t bdesc = make_smem_desc(vbase + kk * 16 * 128, kHalfBytes, 1024, kSw128);
                         if (!(SPI_FLAGS(p) & 2))
-                            umma_bf16_ts(tmem + kColO + pb * 128, tmem + kColS + pb * 128 + kk * 8, bdesc, idesc_o,
+                            umma_bf16_ts(tmem + kColO, tmem + kColP + pb * 64 + kk * 8, bdesc, idesc_o,
                                          (first && kk == 0) ? 0u : 1u);
                     }
-                    umma_commit(&misc->p_empty[pb]);
-                    umma_commit(&misc->empty[slot]);
+                    umma_commit(&misc->pv_done[pb]);
+                    umma_commit(&misc->v_empty[slot]);
                 }
                 ++ls;
-                if (!have_next) {  // (empty segments do not exist; kept for safety)
-                    mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
-                    dn = misc->seg[ls % kSegRing];
-                }
-                d = dn;
             }
         }
     } else {
-        // ============ softmax / epilogue: two groups of 4 warps, alternating KV tiles ============
-        // group g (warps 3 + 4g .. 6 + 4g) owns the tiles with lt & 1 == g: S buffer g, its own
-        // accumulator O_g and running (m, l) per row; thread = one query row (TMEM lane).  The
-        // groups run out of phase, so one group's TMEM / barrier latency hides behind the other's
-        // exponentials.  At a segment's end the two partial softmax states are merged by
-        // log-sum-exp (group g writes dims [64 g, 64 g + 64) of the row).
+        // ====== softmax / epilogue: two groups of 4 warps on alternating tiles, ONE shared O ======
+        // group g (warps 3 + 4g .. 6 + 4g) owns the tiles with lt & 1 == g; thread = one query row (TMEM
+        // lane).  Both groups accumulate into the same O, so every P(t) must use the row reference the
+        // previous tile left: the owner of tile t reads decision(t - 1) (the other group's, through
+        // shared memory + a producer/consumer named barrier per lane quarter), may raise it (stale
+        // max: only beyond 2^8, then O is rescaled after PV(t - 1)), publishes decision(t) and only then
+        // computes its exponentials -- the groups run out of phase, so one group's loads / maxima /
+        // handshake overlap the other's exponentials.  The owner of a segment's last tile writes the
+        // rows (the other group hands over its partial row sums through shared memory).
         const int sw = warp - 3;               // 0..7
         const int grp = sw >> 2;               // tile parity owned by this group
         const int qd = warp & 3;               // TMEM lane quarter
         const int r = qd * 32 + lane;          // query row of the item = TMEM lane
         const uint32_t lane_off = (uint32_t)(qd * 32) << 16;
-        const uint32_t pair_bar = 2 + qd;      // named barrier of the two warps of lane quarter qd
-        const uint32_t s_col = tmem + kColS + grp * 128 + lane_off;
-        const uint32_t o_col = tmem + kColO + grp * 128 + lane_off;
+        const uint32_t dec_bar = 6 + qd;       // decision(t) hand-over between the two warps of quarter qd
+        const uint32_t epi_bar = 10 + qd;      // segment-end row-sum hand-over
+        const uint32_t o_col = tmem + kColO + lane_off;
+        float *mref_s = misc->xm[0][0];        // [row] the row reference after the latest decision
+        float *xl_l = misc->xm[1][0];          // [row] the non-owner group's row sum at a segment end
+        float *xl_m = misc->xm[1][1];          //       ... and the reference it is relative to
         int lt = 0, ls = 0;
-        while (true) {
+        for (;;) {
             mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
             const SegDesc sd = misc->seg[ls % kSegRing];
             if (sd.x < 0) break;
@@ -422,16 +417,18 @@ __global__ void __launch_bounds__(352, 1)
             // ancestor-or-self bitset of this row's node, read on masked tiles only (rows without a
             // node use node 0's root path, which keeps them finite; they are never written)
             const uint32_t *anc = p.anc + ((size_t)b * p.Nmax + (row_valid ? node : 0)) * kBitWords;
-            float m = -INFINITY, l = 0.f;  // this group's running row max (log2 units) and sum
-            int last_own = -1;
+            float m = -INFINITY, l = 0.f;      // latest known row reference (log2 units), this group's sum
+            const int lt0 = lt;
             for (int t = sd.begin; t < sd.end; ++t, ++lt) {
                 if ((lt & 1) != grp) continue;
+                const int sb = lt & 1;
                 const int key0 = (t - sd.ib) * kKeyTile;
-                mbar_wait(&misc->s_full[grp], (lt >> 1) & 1);
+                mbar_wait(&misc->s_full[sb], (lt >> 1) & 1);
                 tc_fence_after();
                 if (r == 0) SPI_TRACE(4 + grp);
-                // visibility of the tile's 128 keys (4 words): committed keys visible; tree keys by
-                // the ancestor bitset; keys past the request's end: none
+                const uint32_t s_col = tmem + kColS + sb * 128 + lane_off;
+                // visibility of the tile's 128 keys (4 words): committed keys visible; tree keys by the
+                // ancestor bitset; keys past the request's end: none
                 uint32_t vis[4] = {0xFFFFFFFFu, 0xFFFFFFFFu, 0xFFFFFFFFu, 0xFFFFFFFFu};
                 const bool masked = key0 + kKeyTile > P;
                 if (masked) {
@@ -451,200 +448,243 @@ __global__ void __launch_bounds__(352, 1)
                         }
                     }
                 }
-                // pass 1: tile row max (unmasked tiles, the common case, take the select-free path)
-                float tm4[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
-                if (masked) tile_max<true>(s_col, vis, tm4);
-                else if (SPI_FLAGS(p) & 4) tm4[0] = 1.f;  // experiment: no S loads (results invalid)
-                else tile_max<false>(s_col, vis, tm4);
-                const float tm = fmaxf(fmaxf(tm4[0], tm4[1]), fmaxf(tm4[2], tm4[3])) * p.scale_log2;
-                // stale running max: move it only when this tile exceeds it by more than 2^8
+                // pass 1: this row's tile max
+                float tm;
+                {
+                    float m4[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
+#pragma unroll
+                    for (int hh = 0; hh < 2; ++hh) {
+                        uint32_t a[2][32];
+                        tmem_ld32(s_col + hh * 64, a[0]);
+                        tmem_ld32(s_col + hh * 64 + 32, a[1]);
+                        tmem_ld_wait();
+#pragma unroll
+                        for (int q = 0; q < 2; ++q) {
+                            if (masked) rows::mask32(a[q], vis[2 * hh + q]);
+#pragma unroll
+                            for (int i = 0; i < 32; ++i) m4[i & 3] = fmaxf(m4[i & 3], __uint_as_float(a[q][i]));
+                        }
+                    }
+                    tm = fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3])) * p.scale_log2;
+                }
+                // decision(t - 1): the reference P(t - 1) used (ignored at a segment's first tile: new rows)
+                if (lt > 0) {
+                    named_bar_sync(dec_bar, 64);
+                    const float mp = mref_s[r];
+                    if (lt > lt0 && mp != m) {   // the other group raised it: rebase this group's sum
+                        l = (m == -INFINITY) ? 0.f : l * ex2(m - mp);
+                        m = mp;
+                    }
+                }
+                if (r == 0) SPI_TRACE(8 + grp);
+                // decision(t): stale running max, moved only when this tile exceeds it by more than 2^8
                 float alpha = 1.f;
                 if (tm > m + kRescaleThreshold) {
                     alpha = (m == -INFINITY) ? 0.f : ex2(m - tm);
                     m = tm;
                     l *= alpha;
                 }
-                if (__any_sync(0xffffffffu, alpha != 1.f) && t - sd.begin >= 2) {
-                    // rescale O_g rows: PV of this group's previous tile must be complete
-                    mbar_wait(&misc->p_empty[grp], ((lt - 2) >> 1) & 1);
+                const bool moved = __any_sync(0xffffffffu, alpha != 1.f) && lt > lt0;
+                if (moved) {
+                    // O holds PV(<= t - 1) against the old reference: rescale once PV(t - 1) completed
+                    mbar_wait(&misc->pv_done[(lt - 1) & 1], ((lt - 1) >> 1) & 1);
                     tc_fence_after();
-#pragma unroll
+#pragma unroll 1
                     for (int q2 = 0; q2 < 4; ++q2) {
                         uint32_t v[32];
                         tmem_ld32(o_col + q2 * 32, v);
                         tmem_ld_wait();
                         uint32_t w16[16];
 #pragma unroll
-                        for (int h = 0; h < 2; ++h) {
+                        for (int hh = 0; hh < 2; ++hh) {
 #pragma unroll
-                            for (int i = 0; i < 16; ++i) w16[i] = __float_as_uint(__uint_as_float(v[h * 16 + i]) * alpha);
-                            tmem_st16(o_col + q2 * 32 + h * 16, w16);
+                            for (int i = 0; i < 16; ++i) w16[i] = __float_as_uint(__uint_as_float(v[hh * 16 + i]) * alpha);
+                            tmem_st16(o_col + q2 * 32 + hh * 16, w16);
                         }
                     }
                     tmem_st_wait();
                 }
-                const float mref = (m == -INFINITY) ? 0.f : m;
-                // pass 2: P = 2^(s * scale - m) as bf16 pairs over the first 64 columns of S(lt)
-                // (keys 32 q .. 32 q + 31 -> columns 16 q .. 16 q + 15: always already read)
-                float l4[4] = {0.f, 0.f, 0.f, 0.f};
-                if (masked) tile_exp<true>(s_col, vis, p.scale_log2, mref, l4);
-                else if (SPI_FLAGS(p) & 8) l4[0] = 1.f;  // experiment: no softmax work (results invalid)
-                else tile_exp<false>(s_col, vis, p.scale_log2, mref, l4);
-                l += (l4[0] + l4[1]) + (l4[2] + l4[3]);
+                mref_s[r] = m;
+                named_bar_arrive(dec_bar, 64);   // decision(t) -> the owner of tile t + 1
+                // pass 2: P(t) = 2^(s * scale - m) as bf16 pairs into P buffer t & 1 (free once PV(t - 2)
+                // completed), row sum of the rounded values
+                if (lt >= 2) mbar_wait(&misc->pv_done[sb], ((lt - 2) >> 1) & 1);
+                tc_fence_after();
+                {
+                    const float mref = (m == -INFINITY) ? 0.f : m;
+                    const uint64_t sc2 = f2_bits(p.scale_log2, p.scale_log2), nm2 = f2_bits(-mref, -mref);
+                    const uint32_t p_col = tmem + kColP + sb * 64 + lane_off;
+                    float ls2 = 0.f;
+#pragma unroll
+                    for (int hh = 0; hh < 2; ++hh) {
+                        uint32_t a[2][32];
+                        tmem_ld32(s_col + hh * 64, a[0]);
+                        tmem_ld32(s_col + hh * 64 + 32, a[1]);
+                        tmem_ld_wait();
+                        if (hh == 1) {
+                            tc_fence_before();
+                            __syncwarp();
+                            if (lane == 0) mbar_arrive(&misc->s_free[sb]);   // S(t + 2) may overwrite it
+                        }
+#pragma unroll
+                        for (int q = 0; q < 2; ++q) {
+                            if (masked) rows::mask32(a[q], vis[2 * hh + q]);
+                            uint32_t w16[16];
+                            float dummy = 0.f;
+                            ls2 += rows::exp32<false>(a[q], sc2, nm2, w16, dummy);
+                            tmem_st16(p_col + hh * 32 + q * 16, w16);
+                        }
+                    }
+                    l += (SPI_FLAGS(p) & 8) ? 1.f : ls2;
+                }
                 tmem_st_wait();
                 tc_fence_before();
                 __syncwarp();
-                if (lane == 0) mbar_arrive(&misc->p_full[grp]);
+                if (lane == 0) mbar_arrive(&misc->p_full[sb]);
                 if (r == 0) SPI_TRACE(6 + grp);
-                last_own = lt;
             }
 
-            // ============ epilogue of this segment: merge the two groups, store ============
-            if (last_own >= 0) mbar_wait(&misc->p_empty[grp], (last_own >> 1) & 1);  // own last PV done
-            // (m, l) exchange through one float2 per row: group 1 publishes, group 0 reads it and
-            // publishes its own after a second barrier
-            if (grp == 1) misc->xch[r] = make_float2(m, l);
-            tc_fence_before();
-            named_bar_sync(pair_bar, 64);
-            tc_fence_after();
-            const float2 other = misc->xch[r];
-            named_bar_sync(pair_bar, 64);
-            if (grp == 0) misc->xch[r] = make_float2(m, l);
-            named_bar_sync(pair_bar, 64);
-            const float2 mine = make_float2(m, l);
-            const float2 g0 = (grp == 0) ? mine : misc->xch[r];
-            const float2 g1 = (grp == 1) ? mine : other;
-            if (r == 0 && grp == 0) SPI_TRACE(8);
-            const float mA = g0.x, mB = g1.x;
-            const float M = fmaxf(mA, mB);
-            const float wA = (mA == -INFINITY) ? 0.f : ex2(mA - M);
-            const float wB = (mB == -INFINITY) ? 0.f : ex2(mB - M);
-            const float lrow = wA * g0.y + wB * g1.y;
-            const bool useA = mA != -INFINITY, useB = mB != -INFINITY;
-            const uint32_t oA = tmem + kColO + grp * 64 + lane_off;        // dims [64 grp, 64 grp + 64)
-            const uint32_t oB = tmem + kColO + 128 + grp * 64 + lane_off;
-            const bool full = (sd.begin == sd.ib) && (sd.end == sd.ie);
-            // merged, unnormalised O row half (16 dims at a time)
-            auto merged = [&](int q4, float (&o)[16]) {
-                uint32_t va[16], vb[16];
-                tmem_ld16(oA + q4 * 16, va);
-                tmem_ld16(oB + q4 * 16, vb);
-                tmem_ld_wait();
-#pragma unroll
-                for (int i = 0; i < 16; ++i)
-                    o[i] = (useA ? wA * __uint_as_float(va[i]) : 0.f) + (useB ? wB * __uint_as_float(vb[i]) : 0.f);
-            };
-            if (full) {
-                const float inv = 1.0f / lrow;
-                __nv_bfloat16 *orow = p.out + (((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim + grp * 64;
+            // ============ epilogue of this segment (the owner of its last tile writes the rows) ============
+            const int llast = lt - 1;
+            const int owner = llast & 1;
+            // (two full barriers: the non-owner may not overwrite the hand-over slots of the next segment
+            // before the owner has read them)
+            if (grp != owner) {
+                xl_l[r] = l;
+                xl_m[r] = m;
+                named_bar_sync(epi_bar, 64);
+                named_bar_sync(epi_bar, 64);
+            } else {
+                named_bar_sync(epi_bar, 64);
+                const float lo_ = xl_l[r], mo = xl_m[r];
+                named_bar_sync(epi_bar, 64);
+                const float lrow = l + ((mo == -INFINITY || lo_ == 0.f) ? 0.f : lo_ * ex2(mo - m));
+                mbar_wait(&misc->pv_done[llast & 1], (llast >> 1) & 1);   // O complete (in-order PVs)
+                tc_fence_after();
+                if (r == 0) SPI_TRACE(10);
+                const bool full = (sd.begin == sd.ib) && (sd.end == sd.ie);
+                if (full) {
+                    const float inv = 1.0f / lrow;
+                    __nv_bfloat16 *orow = p.out + (((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim;
 #pragma unroll 1
-                for (int q4 = 0; q4 < 4; ++q4) {
-                    float o[16];
-                    merged(q4, o);
-                    if (row_valid) {
+                    for (int q2 = 0; q2 < 4; ++q2) {
+                        uint32_t o[32];
+                        tmem_ld32(o_col + q2 * 32, o);
+                        tmem_ld_wait();
+                        if (row_valid) {
 #pragma unroll
-                        for (int i = 0; i < 16; i += 8) {
-                            uint4 o4;
-                            o4.x = pack_bf16x2(o[i] * inv, o[i + 1] * inv);
-                            o4.y = pack_bf16x2(o[i + 2] * inv, o[i + 3] * inv);
-                            o4.z = pack_bf16x2(o[i + 4] * inv, o[i + 5] * inv);
-                            o4.w = pack_bf16x2(o[i + 6] * inv, o[i + 7] * inv);
-                            *reinterpret_cast<uint4 *>(orow + q4 * 16 + i) = o4;
+                            for (int i = 0; i < 32; i += 8) {
+                                uint4 w;
+                                w.x = pack_bf16x2(__uint_as_float(o[i]) * inv, __uint_as_float(o[i + 1]) * inv);
+                                w.y = pack_bf16x2(__uint_as_float(o[i + 2]) * inv, __uint_as_float(o[i + 3]) * inv);
+                                w.z = pack_bf16x2(__uint_as_float(o[i + 4]) * inv, __uint_as_float(o[i + 5]) * inv);
+                                w.w = pack_bf16x2(__uint_as_float(o[i + 6]) * inv, __uint_as_float(o[i + 7]) * inv);
+                                *reinterpret_cast<uint4 *>(orow + q2 * 32 + i) = w;
+                            }
                         }
                     }
-                }
-            } else {
-                const int slot = (sd.begin == t0) ? 0 : 1;
-                float *po = p.part_o + (((size_t)blockIdx.x * 2 + slot) * RB + r) * kHeadDim + grp * 64;
+                    tc_fence_before();
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(&misc->o_free);   // the next segment's first PV may overwrite O
+                } else {
+                    // a piece of a split item: unnormalised O row, (m, l) of the row, then the last piece
+                    // merges every piece by log-sum-exp
+                    const int slot = (sd.begin == t0) ? 0 : 1;
+                    float *po = p.part_o + (((size_t)blockIdx.x * 2 + slot) * RB + r) * kHeadDim;
 #pragma unroll 1
-                for (int q4 = 0; q4 < 4; ++q4) {
-                    float o[16];
-                    merged(q4, o);
+                    for (int q2 = 0; q2 < 4; ++q2) {
+                        uint32_t o[32];
+                        tmem_ld32(o_col + q2 * 32, o);
+                        tmem_ld_wait();
 #pragma unroll
-                    for (int i = 0; i < 16; i += 4)
-                        *reinterpret_cast<float4 *>(po + q4 * 16 + i) = make_float4(o[i], o[i + 1], o[i + 2], o[i + 3]);
-                }
-                float *pml = p.part_ml + ((size_t)blockIdx.x * 2 + slot) * 2 * RB;
-                if (grp == 0) {
-                    pml[r] = M;
+                        for (int i = 0; i < 32; i += 4)
+                            *reinterpret_cast<float4 *>(po + q2 * 32 + i) =
+                                make_float4(__uint_as_float(o[i]), __uint_as_float(o[i + 1]), __uint_as_float(o[i + 2]),
+                                            __uint_as_float(o[i + 3]));
+                    }
+                    tc_fence_before();
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(&misc->o_free);
+                    float *pml = p.part_ml + ((size_t)blockIdx.x * 2 + slot) * 2 * RB;
+                    pml[r] = m;
                     pml[RB + r] = lrow;
-                }
-                __threadfence();
-                named_bar_sync(1, 256);
-                if (r == 0 && grp == 0) {
-                    const int c_first = cta_of_tile(sd.ib, T, NC);
-                    const int c_last = cta_of_tile(sd.ie - 1, T, NC);
-                    int npieces = 0;
-                    for (int cc = c_first; cc <= c_last; ++cc)
-                        npieces += cta_start(cc + 1, T, NC) > cta_start(cc, T, NC);
-                    const unsigned old = atomicAdd(&p.item_cnt[sd.x], 1u);
-                    misc->bcast = (old == (unsigned)(npieces - 1)) ? 1 : 0;
-                    if (misc->bcast) p.item_cnt[sd.x] = 0u;  // ready for the next launch
-                }
-                named_bar_sync(1, 256);
-                if (misc->bcast) {
-                    // last piece: merge every piece's (m, l, O row half) by log-sum-exp
                     __threadfence();
-                    const int c_first = cta_of_tile(sd.ib, T, NC);
-                    const int c_last = cta_of_tile(sd.ie - 1, T, NC);
-                    float Mx = -INFINITY;
-                    for (int cc = c_first; cc <= c_last; ++cc) {
-                        const int s0 = cta_start(cc, T, NC);
-                        if (cta_start(cc + 1, T, NC) <= s0) continue;
-                        const size_t po2 = ((size_t)cc * p.lanes + cl) * 2 + ((s0 >= sd.ib) ? 0 : 1);
-                        Mx = fmaxf(Mx, ldcg_f32(p.part_ml + po2 * 2 * RB + r));
+                    named_bar_sync(14, 128);   // the owner group's 4 warps
+                    if (r == 0) {
+                        const int c_first = cta_of_tile(sd.ib, T, NC);
+                        const int c_last = cta_of_tile(sd.ie - 1, T, NC);
+                        int npieces = 0;
+                        for (int cc = c_first; cc <= c_last; ++cc)
+                            npieces += cta_start(cc + 1, T, NC) > cta_start(cc, T, NC);
+                        const unsigned old = atomicAdd(&p.item_cnt[sd.x], 1u);
+                        misc->bcast = (old == (unsigned)(npieces - 1)) ? 1 : 0;
+                        if (misc->bcast) p.item_cnt[sd.x] = 0u;  // ready for the next launch
                     }
-                    float Ls = 0.f;
-                    for (int cc = c_first; cc <= c_last; ++cc) {
-                        const int s0 = cta_start(cc, T, NC);
-                        if (cta_start(cc + 1, T, NC) <= s0) continue;
-                        const size_t po2 = ((size_t)cc * p.lanes + cl) * 2 + ((s0 >= sd.ib) ? 0 : 1);
-                        const float mp = ldcg_f32(p.part_ml + po2 * 2 * RB + r);
-                        if (mp != -INFINITY) Ls += ex2(mp - Mx) * ldcg_f32(p.part_ml + po2 * 2 * RB + RB + r);
-                    }
-                    const float inv = 1.0f / Ls;
-                    __nv_bfloat16 *orow = p.out + (((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim + grp * 64;
-                    for (int q2 = 0; q2 < 2; ++q2) {
-                        float acc[32];
-#pragma unroll
-                        for (int i = 0; i < 32; ++i) acc[i] = 0.f;
+                    named_bar_sync(14, 128);
+                    if (misc->bcast) {
+                        // last piece: merge every piece's (m, l, O row) by log-sum-exp
+                        __threadfence();
+                        const int c_first = cta_of_tile(sd.ib, T, NC);
+                        const int c_last = cta_of_tile(sd.ie - 1, T, NC);
+                        float Mx = -INFINITY;
+                        for (int cc = c_first; cc <= c_last; ++cc) {
+                            const int s0 = cta_start(cc, T, NC);
+                            if (cta_start(cc + 1, T, NC) <= s0) continue;
+                            const size_t po2 = ((size_t)cc * p.lanes + cl) * 2 + ((s0 >= sd.ib) ? 0 : 1);
+                            Mx = fmaxf(Mx, ldcg_f32(p.part_ml + po2 * 2 * RB + r));
+                        }
+                        float Ls = 0.f;
                         for (int cc = c_first; cc <= c_last; ++cc) {
                             const int s0 = cta_start(cc, T, NC);
                             if (cta_start(cc + 1, T, NC) <= s0) continue;
                             const size_t po2 = ((size_t)cc * p.lanes + cl) * 2 + ((s0 >= sd.ib) ? 0 : 1);
                             const float mp = ldcg_f32(p.part_ml + po2 * 2 * RB + r);
-                            if (mp == -INFINITY) continue;
-                            const float w = ex2(mp - Mx) * inv;
-                            const float4 *src = reinterpret_cast<const float4 *>(
-                                p.part_o + (po2 * RB + r) * kHeadDim + grp * 64 + q2 * 32);
-#pragma unroll
-                            for (int i = 0; i < 8; ++i) {
-                                const float4 o4 = __ldcg(src + i);
-                                acc[4 * i] += w * o4.x;
-                                acc[4 * i + 1] += w * o4.y;
-                                acc[4 * i + 2] += w * o4.z;
-                                acc[4 * i + 3] += w * o4.w;
-                            }
+                            if (mp != -INFINITY) Ls += ex2(mp - Mx) * ldcg_f32(p.part_ml + po2 * 2 * RB + RB + r);
                         }
-                        if (row_valid) {
+                        const float inv = 1.0f / Ls;
+                        __nv_bfloat16 *orow = p.out + (((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim;
+                        for (int q2 = 0; q2 < 4; ++q2) {
+                            float acc[32];
 #pragma unroll
-                            for (int i = 0; i < 32; i += 8) {
-                                uint4 o4;
-                                o4.x = pack_bf16x2(acc[i], acc[i + 1]);
-                                o4.y = pack_bf16x2(acc[i + 2], acc[i + 3]);
-                                o4.z = pack_bf16x2(acc[i + 4], acc[i + 5]);
-                                o4.w = pack_bf16x2(acc[i + 6], acc[i + 7]);
-                                *reinterpret_cast<uint4 *>(orow + q2 * 32 + i) = o4;
+                            for (int i = 0; i < 32; ++i) acc[i] = 0.f;
+                            for (int cc = c_first; cc <= c_last; ++cc) {
+                                const int s0 = cta_start(cc, T, NC);
+                                if (cta_start(cc + 1, T, NC) <= s0) continue;
+                                const size_t po2 = ((size_t)cc * p.lanes + cl) * 2 + ((s0 >= sd.ib) ? 0 : 1);
+                                const float mp = ldcg_f32(p.part_ml + po2 * 2 * RB + r);
+                                if (mp == -INFINITY) continue;
+                                const float w = ex2(mp - Mx) * inv;
+                                const float4 *src = reinterpret_cast<const float4 *>(
+                                    p.part_o + (po2 * RB + r) * kHeadDim + q2 * 32);
+#pragma unroll
+                                for (int i = 0; i < 8; ++i) {
+                                    const float4 o4 = __ldcg(src + i);
+                                    acc[4 * i] += w * o4.x;
+                                    acc[4 * i + 1] += w * o4.y;
+                                    acc[4 * i + 2] += w * o4.z;
+                                    acc[4 * i + 3] += w * o4.w;
+                                }
+                            }
+                            if (row_valid) {
+#pragma unroll
+                                for (int i = 0; i < 32; i += 8) {
+                                    uint4 o4;
+                                    o4.x = pack_bf16x2(acc[i], acc[i + 1]);
+                                    o4.y = pack_bf16x2(acc[i + 2], acc[i + 3]);
+                                    o4.z = pack_bf16x2(acc[i + 4], acc[i + 5]);
+                                    o4.w = pack_bf16x2(acc[i + 6], acc[i + 7]);
+                                    *reinterpret_cast<uint4 *>(orow + q2 * 32 + i) = o4;
+                                }
                             }
                         }
                     }
                 }
+                if (r == 0) SPI_TRACE(11);
             }
-            tc_fence_before();
-            named_bar_sync(pair_bar, 64);  // both O accumulators and (m, l) read before reuse
-            if (r == 0 && grp == 0) SPI_TRACE(9);
             ++ls;
         }
+        // the last tile's decision has no next owner: consume it so every barrier phase completes
+        if (lt > 0 && ((lt - 1) & 1) != grp) named_bar_sync(dec_bar, 64);
     }
 
     tc_fence_before();
@@ -656,8 +696,8 @@ __global__ void __launch_bounds__(352, 1)
     if (threadIdx.x == 0) SPI_TRACE_K(1);
 }
 
-static size_t rows_smem_bytes(int num_slots) {
-    return (size_t)num_slots * kSlotBytes + 2 * rows::kQBuf + sizeof(rows::Misc);
+static size_t rows_smem_bytes(int nk, int nv) {
+    return (size_t)(nk + nv) * kSlotBytes + 2 * rows::kQBuf + sizeof(rows::Misc);
 }
 
 cudaError_t launch_tree_attention_rows(const AttnParams &prm0, const void *q, const void *k, const void *v,
@@ -671,11 +711,15 @@ cudaError_t launch_tree_attention_rows(const AttnParams &prm0, const void *q, co
         !encode_2d(&tk16, k, rows, 16) || !encode_2d(&tv16, v, rows, 16) || !encode_2d(&tk4, k, rows, 4) ||
         !encode_2d(&tv4, v, rows, 4) || !encode_2d(&tk1, k, rows, 1) || !encode_2d(&tv1, v, rows, 1))
         return cudaErrorInvalidValue;
-    int ns = rows::kMaxRing;
-    while (ns > 2 && rows_smem_bytes(ns) > max_smem) --ns;
-    prm.nk_slots = ns;  // unified K/V ring
-    prm.nv_slots = 0;
-    const size_t smem = rows_smem_bytes(ns);
+    // K ring 3 slots (K is released right after S), V ring 2 (held until PV); fewer if smem is short
+    int nk = 3, nv = 2;
+    while (rows_smem_bytes(nk, nv) > max_smem && nk + nv > 2) {
+        if (nk > nv) --nk; else --nv;
+    }
+    if (rows_smem_bytes(nk, nv) > max_smem) return cudaErrorInvalidConfiguration;
+    prm.nk_slots = nk;
+    prm.nv_slots = nv;
+    const size_t smem = rows_smem_bytes(nk, nv);
     {
         const cudaError_t e = ensure_max_smem_attr((const void *)tree_attn_rows_kernel, 3, max_smem);
         if (e != cudaSuccess) return e;

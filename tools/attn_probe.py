@@ -97,7 +97,7 @@ def main():
                 base = x[0, 0]
                 print(f"CTA {c} raw events (cycles rel. to first K issue): 0 K-iss 1 V-iss 2 S-mma 3 PV-mma 4/5 sm-beg g0/g1 6/7 P-rdy g0/g1 8 epi 9 epi-end")
                 for i in range(40):
-                    print(f"{i:3d} " + " ".join(f"{(v - base) if v else -1:8d}" for v in x[i, :10]))
+                    print(f"{i:3d} " + " ".join(f"{(v - base) if v else -1:8d}" for v in x[i, :12]))
             return
         for c in range(2):
             x = t[c]
