@@ -35,8 +35,6 @@ struct WsLayout {
     size_t part_ml;     // float[max_ctas][2][2][NT]
     size_t argmax;      // int32[B][Nmax]
     size_t verify_cnt;  // uint32[2][B]          last-CTA counters: greedy, MSS
-    size_t mss_stats;   // float2[B][Nmax]       softmax (max, sum) of every node's logits / T
-    size_t mss_leaf;    // int32[B][Nmax]        round-0 exponential-race sample of every leaf
     size_t mss_p;       // float[B][2][V]        MSS residual distributions (double buffer)
     size_t total;
     int nt;             // query rows per chunk (UMMA N): 16, 32 or 64
@@ -103,8 +101,6 @@ inline WsLayout ws_layout(const specinfer_shape_t &s, int num_sms, bool allow_sp
     w.part_ml = take(size_t(w.max_ctas) * 2 * 2 * w.nt * 4);
     w.argmax = take(size_t(B) * N * 4);
     w.verify_cnt = take(size_t(B) * 2 * 4);
-    w.mss_stats = take(size_t(B) * N * 8);
-    w.mss_leaf = take(size_t(B) * N * 4);
     w.mss_p = take(size_t(B) * 2 * (size_t)(s.vocab > 0 ? s.vocab : 1) * 4);
     w.total = o;
     return w;

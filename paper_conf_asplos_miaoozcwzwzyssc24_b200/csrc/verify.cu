@@ -9,14 +9,16 @@
 // per-node key is the exponential-race key of x ~ softmax(l / T) instead of the logit, and the
 // walk follows the child whose token equals that sample.
 //
-// VerifyStochastic = MSS (Alg. 2 lines 24-44, L403-425; Fig. 5): also one launch.  Phase 1, one
-// CTA per (node, request): the softmax statistics (max, sum of exp) of logits[u]/T for every
-// node, in parallel.  Phase 2, the last CTA of the request: the sequential walk of Alg. 2.  An
-// accept test then costs O(1) (p[x] from the statistics); only a rejection (residual
-// p <- norm(max(0, p - q)), double-buffered so that an all-zero residual keeps p, reading R11)
-// and the final exponential-race sample stream a V-wide row.  The RNG contract (Philox4x32-10,
-// counters from the global request id, node, round, offset; readings R9, R15) makes the result
-// independent of batching and GPU count.
+// VerifyStochastic = MSS (Alg. 2 lines 24-44, L403-425; Fig. 5): also one launch, one 8-CTA
+// thread-block cluster per request walking Alg. 2 sequentially.  At every visited node the
+// cluster computes the softmax statistics of logits[u]/T (a V-wide pass split over the 8 CTAs and
+// reduced through distributed shared memory); an accept test is then O(1); a rejection streams one
+// V-wide residual pass p <- norm(max(0, p - q)) (double-buffered so that an all-zero residual
+// keeps p, reading R11) split the same way, and the exponential race of the final sample is fused
+// into the last pass.  The RNG contract (Philox4x32-10, counters from the global request id, node,
+// round, offset; readings R9, R15) makes the result independent of batching and GPU count.
+// NEXT-4a: with a gather descriptor, the finishing warp of every request also stores its packed
+// row into every rank's receive table (gather.cuh).
 #include "common.cuh"
 #include "gather.cuh"
 

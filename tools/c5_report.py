@@ -7,14 +7,18 @@ import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 R = sys.argv[1] if len(sys.argv) > 1 else "r01"
-src = os.path.join(ROOT, "gpurun_out", "c5_sweep.jsonl")
+src = os.path.join(ROOT, "gpurun_out", f"c5_sweep_{R}.jsonl")
+if not os.path.exists(src):
+    src = os.path.join(ROOT, "gpurun_out", "c5_sweep.jsonl")
 rows = [json.loads(l) for l in open(src)]
 pk = rows[0]["peaks"]
 out = [f"# C5 sweep, round {R[1:]} (`tools/c5_sweep.py`, one B200)", "",
        "BASELINE.json configs[4]: tree size x batch x prefix, LLaMA-7B attention shape (32 heads x 128, MHA), one layer per point,",
-       "random trees of exactly n nodes (depth <= 8, fanout <= 8, seeded), greedy verification over V = 32000. CUDA-event time per",
-       "launch on the launching stream (host launch overhead included: small points are bounded by it), median of 10, L2 flushed",
-       "(256 MB write) before every timed launch. Algorithmic bytes per (request, kv-head) = (P + n)*512 + G*n*512; FLOPs per",
+       "random trees of exactly n nodes (depth <= 8, fanout <= 8, seeded), greedy verification over V = 32000. Attention: device",
+       "time per launch from a CUDA graph of consecutive launches (SPECINFER_ATTN_EARLY_PREFIX after the first, as bench.py runs",
+       "the layers) rotating over enough layers' caches that each replay streams > 512 MB (no L2 flush needed; `graph_layers`),",
+       "median of 3 replays; verification: CUDA events per launch after a 256 MB L2 flush. Algorithmic bytes per (request,",
+       "kv-head) = (P + n)*512 + G*n*512; FLOPs per",
        "(request, q-head) = 4*128*(n*P + sum(depth+1)); bound = the roof the arithmetic intensity hits first",
        f"(ridge = {pk['bf16_tflops'] * 1e3 / pk['hbm_gbs']:.0f} flop/B). Peaks: {pk['hbm_gbs']} GB/s HBM, {pk['bf16_tflops']} TFLOP/s bf16 "
        f"({pk['source']}{', B200_PROFILING.md; MEASURED_PEAKS.json was absent' if pk['source'] == 'fallback' else ''}).",
@@ -28,9 +32,11 @@ for r in rows:
 big = [r for r in rows if r['bound'] == 'hbm' and r['n'] <= 64 and r['batch'] * r['prefix'] >= 8 * 8192]
 out += ["", f"Memory-bound points with n <= 64 and B*P >= 65536 (>= 1.07 GB of KV per launch): HBM fraction "
         f"{min(r['hbm_frac'] for r in big):.3f}-{max(r['hbm_frac'] for r in big):.3f}.",
-        "Small points (B = 1, or B*P <= 4096) are latency-bound: one launch covers a few MB and the host launch, the",
-        "prologue and the first TMA round trip dominate. n = 128 / 256 run the rows kernel, bound by its softmax -> PV -> S",
-        "chain (`profiles/rows_kernel_r01.md`)."]
+        "Fractions slightly above 1 are possible: the denominator is a read+write copy, these launches only read (the TMA",
+        "read probe reaches ~6.1-7.0 TB/s on large buffers, `bench.py` roofline). Small points (B = 1, B*P <= 4096) are",
+        "latency-bound: a launch covers a few MB and the kernel-boundary costs dominate (dispatch, prologue, first loads,",
+        "split merge: `profiles/small_batch_r02.md`). n = 128 / 256 run the rows kernel, bound by its per-tile softmax",
+        "instruction stream (`profiles/rows_kernel_r02.md`)."]
 open(os.path.join(ROOT, "profiles", f"c5_sweep_{R}.md"), "w").write("\n".join(out) + "\n")
 shutil.copy(src, os.path.join(ROOT, "profiles", f"c5_sweep_{R}.jsonl"))
 print("\n".join(out[-5:]))

@@ -5,9 +5,11 @@ each point reported against the HBM and the tensor roofline.
     python tools/c5_sweep.py [--out gpurun_out/c5_sweep.jsonl] [--iters 10] [--quick]
 
 Per point: random trees of exactly n nodes (depth <= 8, fanout <= 8, DFS preorder, seeded), prefix P
-for every request.  Timing: CUDA events on the launching stream around each launch, median of
-`iters`; L2 (126 MB) is flushed before every timed launch by writing a 256 MB buffer, so small points
-are measured from HBM like large ones.  Algorithmic bytes per (request, kv-head) = (P + n)*128*2*2
+for every request.  Attention timing: a CUDA graph of consecutive launches (as bench.py runs the layers:
+SPECINFER_ATTN_EARLY_PREFIX after the first) rotating over enough layers' caches that the streamed bytes
+exceed 512 MB (4x the L2), per-launch = graph time / launches (tools/graph_timing.py).  Verification:
+CUDA events around each launch with a 256 MB L2 flush before it.  Roofline denominators: the driver's
+MEASURED_PEAKS.json (hbm_gbs; bf16 sustained for tensor-bound points), else the guide's fallback.  Algorithmic bytes per (request, kv-head) = (P + n)*128*2*2
 (K, V read once) + G*n*128*2*2 (q in, out); FLOPs per (request, q-head) = 4*128*(n*P + sum(depth+1)).
 """
 import argparse
@@ -23,13 +25,14 @@ import torch
 
 import paper_conf_asplos_miaoozcwzwzyssc24_b200 as spi
 import workloads as W
+from tools.graph_timing import graph_us_per_launch, layers_for
 
 
 def peaks():
     try:
         d = json.load(open(os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))),
                                         "MEASURED_PEAKS.json")))
-        return float(d["hbm_gbs"]), float(d["bf16_tflops"]), "measured"
+        return float(d["hbm_gbs"]), float(d.get("bf16_tflops_sustained", d["bf16_tflops"])), "measured"
     except Exception:
         return 6650.0, 1590.0, "fallback"
 
@@ -69,15 +72,14 @@ def main():
     for (n, B, P) in pts:
         tb = W.random_tree_batch(B, n, P, seed=1000 + n, device=dev)
         smax = P + n
-        ai = W.make_attention_inputs(tb, 1, H, H, smax, seed=5, device=dev)
+        nl = layers_for(B * H * smax * 512)
+        ai = W.make_attention_inputs(tb, nl, H, H, smax, seed=5, device=dev)
         shape = spi.make_shape(B, tb.max_nodes, H, H, smax, vocab=a.vocab, max_depth=tb.max_depth)
         st = spi.TreeState.create(shape, tb.parent, tb.depth, tb.prefix_len, tb.n_nodes)
         st.prepare()
         out = torch.empty_like(ai.q[0])
-        run_attn = lambda: st.attention(ai.q[0], ai.k_cache[0], ai.v_cache[0], out)
-        for _ in range(3):
-            run_attn()
-        us = timed(run_attn, flush, a.iters)
+        us = graph_us_per_launch(lambda i, first: st.attention(ai.q[i % nl], ai.k_cache[i % nl], ai.v_cache[i % nl],
+                                                               out, prefetch=not first), nl)
         # greedy verification of the same trees (logits fp32 [B][n][V])
         vi = W.make_verify_inputs(tb, a.vocab, seed=5, mode="greedy", device=dev)
         an = torch.empty((B, tb.max_depth + 1), dtype=torch.int32, device=dev)
@@ -104,7 +106,7 @@ def main():
                "AI": round(ai_, 1), "bound": bound,
                "roofline_frac": round(gbs / hbm if bound == "hbm" else tfs / tf, 4),
                "verify_greedy_us": round(us_v, 2), "verify_GBps": round(vbytes / us_v / 1e3, 1),
-               "tree_tok_per_s_per_layer": round(int(nn.sum()) / (us * 1e-6), 1),
+               "tree_tok_per_s_per_layer": round(int(nn.sum()) / (us * 1e-6), 1), "graph_layers": nl,
                "peaks": {"hbm_gbs": hbm, "bf16_tflops": tf, "source": src}}
         print(json.dumps(rec), flush=True)
         fo.write(json.dumps(rec) + "\n")

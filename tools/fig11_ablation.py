@@ -7,8 +7,9 @@ token tree (the paper's <1,1,k,1,1,1,1,1> of width k, L1078-1079):
   seq-batch   one launch per layer over all root-to-leaf sequences, each with its own cache
               (specinfer_sequence_pack; the committed prefix is read once per leaf)
   seq-launch  one launch per sequence per layer (Fig. 4's Kernel 1/2/3)
-Times are CUDA-event device times per layer (median of `--iters` launches after warm-up,
-alternating between two cache copies so L2 reuse does not flatter any arm), x 32 layers.
+Times are device times per layer from CUDA-graph replays of consecutive launches rotating over enough
+layers' caches that every arm streams > 1 GB per replay (tools/graph_timing.py; host launch overhead
+excluded, as in bench.py), x 32 layers.
 
     python tools/fig11_ablation.py [--prefix 2048] [--batches 1,2,4,8,16] [--widths 1,2,3,4,5]
 Writes one JSON line per point to stdout (and to --out).
@@ -25,6 +26,7 @@ import torch
 
 import paper_conf_asplos_miaoozcwzwzyssc24_b200 as spi
 import workloads as W
+from tools.graph_timing import graph_us_per_launch, layers_for
 
 
 def timed(fn, iters, warm=3):
@@ -60,19 +62,22 @@ def main():
         for B in [int(x) for x in a.batches.split(",")]:
             tb = W.make_tree_batch([(par, dep)] * B, [a.prefix] * B, device=dev, max_depth=len(expansion))
             smax = a.prefix + tb.max_nodes
-            ai = W.make_attention_inputs(tb, 2, H, H, smax, seed=11, device=dev)
+            nl = layers_for(B * H * smax * 512, target=1 << 30, cap=8)
+            ai = W.make_attention_inputs(tb, nl, H, H, smax, seed=11, device=dev)
             shape = spi.make_shape(B, tb.max_nodes, H, H, smax, max_depth=len(expansion))
             st = spi.TreeState.create(shape, tb.parent, tb.depth, tb.prefix_len, tb.n_nodes)
             st.prepare()
             out = torch.empty_like(ai.q[0])
-            t_tree = timed(lambda i: st.attention(ai.q[i & 1], ai.k_cache[i & 1], ai.v_cache[i & 1], out), a.iters)
+            t_tree = graph_us_per_launch(lambda i, first: st.attention(ai.q[i % nl], ai.k_cache[i % nl],
+                                                                       ai.v_cache[i % nl], out, prefetch=not first), nl)
             sbs = []
-            for l in range(2):
+            for l in range(nl):
                 sb = spi.SequenceBaseline(shape, tb.parent, tb.depth, tb.prefix_len, tb.n_nodes)
                 sb.build(ai.q[l], ai.k_cache[l], ai.v_cache[l])
                 sbs.append(sb)
-            t_seq = timed(lambda i: sbs[i & 1].attention(), a.iters)
-            t_seql = timed(lambda i: sbs[i & 1].attention(per_sequence=True), max(3, a.iters // 2), warm=1)
+            t_seq = graph_us_per_launch(lambda i, first: sbs[i % nl].attention(), nl)
+            t_seql = graph_us_per_launch(lambda i, first: sbs[i % nl].attention(per_sequence=True), nl,
+                                         reps=max(nl, 4))
             n = int(tb.n_nodes.sum())
             nseq = sbs[0].num_seqs
             kv_tree = B * H * (a.prefix + tb.max_nodes) * 512
