@@ -105,7 +105,7 @@ __global__ void __launch_bounds__(1024) schedule_kernel(
     const int32_t *__restrict__ req_ok, int B, int Hkv, int chunks, int npc, int lanes,
     int32_t *__restrict__ item_start, uint32_t *__restrict__ item_cnt, int4 *__restrict__ item_info,
     int4 *__restrict__ cta_info, int num_ctas, int splitk, uint32_t *__restrict__ verify_cnt,
-    int32_t *__restrict__ status) {
+    int32_t *__restrict__ status, int no_split_slack) {
     const int n_items = B * Hkv * chunks;
     const int n_units = n_items / lanes;
     const int per = (n_units + blockDim.x - 1) / blockDim.x;
@@ -184,10 +184,9 @@ __global__ void __launch_bounds__(1024) schedule_kernel(
     // parallelism it buys (C1: 2 tiles per unit; B = 1..4 at P = 2048: 17).  Otherwise even stream-K slices.
     const long long T = s_total;
     const int NCv = num_ctas / lanes;
-#ifndef SPECINFER_NOSPLIT_SLACK
-#define SPECINFER_NOSPLIT_SLACK 8
-#endif
-    constexpr int kNoSplitSlack = SPECINFER_NOSPLIT_SLACK;
+    // (no_split_slack: 8 tiles for the swapped kernel; 24 for the rows kernel, whose split merge
+    // reads 64 KB partials per piece -- a few L2 round trips -- so tiny stream-K pieces do not pay)
+    const int kNoSplitSlack = no_split_slack;
     // whole units per CTA group (contiguous ranges of floor / ceil(n_units / NCv) units) when the
     // busiest group's upper bound exceeds an even share by at most kNoSplitSlack tiles
     const int upc = (n_units + NCv - 1) / NCv;
@@ -258,7 +257,8 @@ cudaError_t launch_tree_prepare(const specinfer_shape_t &s, const WsLayout &w,
         prefix_len, n_nodes, reinterpret_cast<int32_t *>(ws + w.req_ok), s.batch,
         s.num_kv_heads, w.chunks, w.npc, w.lanes, reinterpret_cast<int32_t *>(ws + w.item_start),
         reinterpret_cast<uint32_t *>(ws + w.item_cnt), reinterpret_cast<int4 *>(ws + w.item_info),
-        reinterpret_cast<int4 *>(ws + w.cta_info), num_ctas, w.splitk, reinterpret_cast<uint32_t *>(ws + w.verify_cnt), status);
+        reinterpret_cast<int4 *>(ws + w.cta_info), num_ctas, w.splitk, reinterpret_cast<uint32_t *>(ws + w.verify_cnt), status,
+        w.nt == kRowsBlock ? 24 : 8);
     return cudaGetLastError();
 }
 

@@ -39,6 +39,7 @@ struct Misc {
     uint64_t o_free;                         // the epilogue has read O (next segment may overwrite it)
     uint64_t seg_full[kSegRing];
     SegDesc seg[kSegRing];
+    uint64_t stage_bar;                      // bulk staging of split pieces (CTA's last segment)
     uint32_t tmem_base;
     int32_t bcast;
     float xm[2][2][RB];                      // [0][0]: row references; [1][0] / [1][1]: segment-end hand-over
@@ -170,6 +171,7 @@ __global__ void __launch_bounds__(352, 1)
             mbar_init(&misc->pv_done[i], 1);
         }
         mbar_init(&misc->o_free, 4);
+        mbar_init(&misc->stage_bar, 1);
         for (int i = 0; i < kSegRing; ++i) mbar_init(&misc->seg_full[i], 1);
         fence_barrier_init();
     }
@@ -608,6 +610,7 @@ __global__ void __launch_bounds__(352, 1)
                     float *pml = p.part_ml + ((size_t)blockIdx.x * 2 + slot) * 2 * RB;
                     pml[r] = m;
                     pml[RB + r] = lrow;
+                    if (r == 0) SPI_TRACE(12);
                     __threadfence();
                     named_bar_sync(14, 128);   // the owner group's 4 warps
                     if (r == 0) {
@@ -621,59 +624,151 @@ __global__ void __launch_bounds__(352, 1)
                         if (misc->bcast) p.item_cnt[sd.x] = 0u;  // ready for the next launch
                     }
                     named_bar_sync(14, 128);
+                    if (r == 0) SPI_TRACE(13);
                     if (misc->bcast) {
                         // last piece: merge every piece's (m, l, O row) by log-sum-exp
                         __threadfence();
                         const int c_first = cta_of_tile(sd.ib, T, NC);
                         const int c_last = cta_of_tile(sd.ie - 1, T, NC);
-                        float Mx = -INFINITY;
-                        for (int cc = c_first; cc <= c_last; ++cc) {
+                        auto piece = [&](int cc) -> long long {   // partial slot of CTA cc's piece, -1 if empty
                             const int s0 = cta_start(cc, T, NC);
-                            if (cta_start(cc + 1, T, NC) <= s0) continue;
-                            const size_t po2 = ((size_t)cc * p.lanes + cl) * 2 + ((s0 >= sd.ib) ? 0 : 1);
-                            Mx = fmaxf(Mx, ldcg_f32(p.part_ml + po2 * 2 * RB + r));
-                        }
-                        float Ls = 0.f;
-                        for (int cc = c_first; cc <= c_last; ++cc) {
-                            const int s0 = cta_start(cc, T, NC);
-                            if (cta_start(cc + 1, T, NC) <= s0) continue;
-                            const size_t po2 = ((size_t)cc * p.lanes + cl) * 2 + ((s0 >= sd.ib) ? 0 : 1);
-                            const float mp = ldcg_f32(p.part_ml + po2 * 2 * RB + r);
-                            if (mp != -INFINITY) Ls += ex2(mp - Mx) * ldcg_f32(p.part_ml + po2 * 2 * RB + RB + r);
-                        }
-                        const float inv = 1.0f / Ls;
-                        __nv_bfloat16 *orow = p.out + (((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim;
-                        for (int q2 = 0; q2 < 4; ++q2) {
-                            float acc[32];
-#pragma unroll
-                            for (int i = 0; i < 32; ++i) acc[i] = 0.f;
-                            for (int cc = c_first; cc <= c_last; ++cc) {
-                                const int s0 = cta_start(cc, T, NC);
-                                if (cta_start(cc + 1, T, NC) <= s0) continue;
-                                const size_t po2 = ((size_t)cc * p.lanes + cl) * 2 + ((s0 >= sd.ib) ? 0 : 1);
-                                const float mp = ldcg_f32(p.part_ml + po2 * 2 * RB + r);
-                                if (mp == -INFINITY) continue;
-                                const float w = ex2(mp - Mx) * inv;
-                                const float4 *src = reinterpret_cast<const float4 *>(
-                                    p.part_o + (po2 * RB + r) * kHeadDim + q2 * 32);
-#pragma unroll
-                                for (int i = 0; i < 8; ++i) {
-                                    const float4 o4 = __ldcg(src + i);
-                                    acc[4 * i] += w * o4.x;
-                                    acc[4 * i + 1] += w * o4.y;
-                                    acc[4 * i + 2] += w * o4.z;
-                                    acc[4 * i + 3] += w * o4.w;
+                            if (cta_start(cc + 1, T, NC) <= s0) return -1;
+                            return ((long long)cc * p.lanes + cl) * 2 + ((s0 >= sd.ib) ? 0 : 1);
+                        };
+                        // (compact, rolled loops: this code runs cold in the instruction cache, once per item,
+                        // and its length -- not its loads -- set the cost: ~350 ns per missed 128-B line)
+                        if (sd.end == t1) {
+                            // the CTA's last segment: K / V rings and Q buffers are idle -> stage the pieces with
+                            // bulk copies (all in flight at once) instead of one L2 round trip per (piece, chunk):
+                            // (m, l) of every piece, then up to `cap` 64 KB O blocks per round; each warp merges
+                            // its 32 rows with lane = 4 dims (conflict-free, coalesced 256 B output rows)
+                            uint8_t *area = smem;
+                            const size_t area_bytes = (size_t)(NK + NV) * kSlotBytes + 2 * kQBuf;
+                            constexpr uint32_t kOB = RB * kHeadDim * 4, kMLB = 2 * RB * 4;
+                            int npc = 0;
+                            for (int cc = c_first; cc <= c_last; ++cc) npc += piece(cc) >= 0;
+                            float *sml = reinterpret_cast<float *>(area + area_bytes) - (size_t)npc * 3 * RB;  // [npc][m, l, w][RB]
+                            const int cap = (int)(((size_t)((uint8_t *)sml - area)) / kOB);
+                            uint32_t ph = 0;
+                            if (r == 0) {
+                                fence_proxy_async_global();
+                                mbar_arrive_expect_tx(&misc->stage_bar, (uint32_t)npc * kMLB);
+                                int k = 0;
+                                for (int cc = c_first; cc <= c_last; ++cc) {
+                                    const long long po2 = piece(cc);
+                                    if (po2 < 0) continue;
+                                    bulk_load_g2s(sml + (size_t)k * 3 * RB, p.part_ml + po2 * 2 * RB, kMLB, &misc->stage_bar);
+                                    ++k;
                                 }
                             }
-                            if (row_valid) {
+                            mbar_wait(&misc->stage_bar, ph);
+                            ph ^= 1u;
+                            float Mx = -INFINITY, Ls = 0.f;
+                            for (int k = 0; k < npc; ++k) Mx = fmaxf(Mx, sml[(size_t)k * 3 * RB + r]);
+                            for (int k = 0; k < npc; ++k) {
+                                const float mk = sml[(size_t)k * 3 * RB + r];
+                                const float w = (mk == -INFINITY) ? 0.f : ex2(mk - Mx);
+                                Ls += w * sml[(size_t)k * 3 * RB + RB + r];
+                                sml[(size_t)k * 3 * RB + 2 * RB + r] = w;
+                            }
+                            const float inv = 1.0f / Ls;
+                            for (int k = 0; k < npc; ++k) sml[(size_t)k * 3 * RB + 2 * RB + r] *= inv;
+                            named_bar_sync(14, 128);   // weights visible to the whole group
+                            float4 acc[32];   // [row of the warp] lane's 4 dims
 #pragma unroll
-                                for (int i = 0; i < 32; i += 8) {
+                            for (int i = 0; i < 32; ++i) acc[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+                            const int wrow0 = qd * 32;   // this warp's rows
+                            for (int k0 = 0; k0 < npc; k0 += cap) {
+                                const int kn = min(cap, npc - k0);
+                                if (r == 0) {
+                                    mbar_arrive_expect_tx(&misc->stage_bar, (uint32_t)kn * kOB);
+                                    int k = 0;
+                                    for (int cc = c_first; cc <= c_last; ++cc) {
+                                        const long long po2 = piece(cc);
+                                        if (po2 < 0) continue;
+                                        if (k >= k0 && k < k0 + kn)
+                                            bulk_load_g2s(area + (size_t)(k - k0) * kOB, p.part_o + po2 * RB * kHeadDim, kOB,
+                                                          &misc->stage_bar);
+                                        ++k;
+                                    }
+                                }
+                                mbar_wait(&misc->stage_bar, ph);
+                                ph ^= 1u;
+#pragma unroll 1
+                                for (int k = 0; k < kn; ++k) {
+                                    const float *blk = reinterpret_cast<const float *>(area + (size_t)k * kOB);
+                                    const float *wk = sml + (size_t)(k0 + k) * 3 * RB + 2 * RB + wrow0;
+#pragma unroll
+                                    for (int i = 0; i < 32; ++i) {
+                                        const float4 x = *reinterpret_cast<const float4 *>(blk + (size_t)(wrow0 + i) * kHeadDim + 4 * lane);
+                                        const float w = wk[i];
+                                        acc[i].x += w * x.x;
+                                        acc[i].y += w * x.y;
+                                        acc[i].z += w * x.z;
+                                        acc[i].w += w * x.w;
+                                    }
+                                }
+                                named_bar_sync(14, 128);   // the staging area is reused by the next round
+                            }
+                            // rows of this warp: row wrow0 + i -> its node / head (padding rows skipped)
+#pragma unroll
+                            for (int i = 0; i < 32; ++i) {
+                                const int rr = wrow0 + i;
+                                const int nd = c * p.npc + rr / G, hh = rr % G;
+                                if (rr < rc && nd < n) {
+                                    uint2 o2;
+                                    o2.x = pack_bf16x2(acc[i].x, acc[i].y);
+                                    o2.y = pack_bf16x2(acc[i].z, acc[i].w);
+                                    *reinterpret_cast<uint2 *>(p.out + (((size_t)b * p.Nmax + nd) * p.Hq + g * G + hh) * kHeadDim +
+                                                               4 * lane) = o2;
+                                }
+                            }
+                        } else {
+                            float Mx = -INFINITY, Ls = 0.f;
+    #pragma unroll 1
+                            for (int cc = c_first; cc <= c_last; ++cc) {
+                                const long long po2 = piece(cc);
+                                if (po2 < 0) continue;
+                                const float mp = ldcg_f32(p.part_ml + po2 * 2 * RB + r);
+                                const float lp = ldcg_f32(p.part_ml + po2 * 2 * RB + RB + r);
+                                if (mp == -INFINITY) continue;
+                                const float nM = fmaxf(Mx, mp);
+                                Ls = (Mx == -INFINITY ? 0.f : Ls * ex2(Mx - nM)) + ex2(mp - nM) * lp;
+                                Mx = nM;
+                            }
+                            const float inv = 1.0f / Ls;
+                            if (r == 0) SPI_TRACE(14);
+                            __nv_bfloat16 *orow = p.out + (((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim;
+    #pragma unroll 1
+                            for (int q2 = 0; q2 < 8; ++q2) {   // 16 dims at a time
+                                float4 a0 = make_float4(0.f, 0.f, 0.f, 0.f), a1 = a0, a2 = a0, a3 = a0;
+    #pragma unroll 1
+                                for (int cc = c_first; cc <= c_last; ++cc) {
+                                    const long long po2 = piece(cc);
+                                    if (po2 < 0) continue;
+                                    const float mp = ldcg_f32(p.part_ml + po2 * 2 * RB + r);
+                                    const float4 *src = reinterpret_cast<const float4 *>(
+                                        p.part_o + (po2 * RB + r) * kHeadDim + q2 * 16);
+                                    const float4 x0 = __ldcg(src), x1 = __ldcg(src + 1), x2 = __ldcg(src + 2),
+                                                 x3 = __ldcg(src + 3);
+                                    const float w = (mp == -INFINITY) ? 0.f : ex2(mp - Mx) * inv;
+                                    a0.x += w * x0.x; a0.y += w * x0.y; a0.z += w * x0.z; a0.w += w * x0.w;
+                                    a1.x += w * x1.x; a1.y += w * x1.y; a1.z += w * x1.z; a1.w += w * x1.w;
+                                    a2.x += w * x2.x; a2.y += w * x2.y; a2.z += w * x2.z; a2.w += w * x2.w;
+                                    a3.x += w * x3.x; a3.y += w * x3.y; a3.z += w * x3.z; a3.w += w * x3.w;
+                                }
+                                if (row_valid) {
                                     uint4 o4;
-                                    o4.x = pack_bf16x2(acc[i], acc[i + 1]);
-                                    o4.y = pack_bf16x2(acc[i + 2], acc[i + 3]);
-                                    o4.z = pack_bf16x2(acc[i + 4], acc[i + 5]);
-                                    o4.w = pack_bf16x2(acc[i + 6], acc[i + 7]);
-                                    *reinterpret_cast<uint4 *>(orow + q2 * 32 + i) = o4;
+                                    o4.x = pack_bf16x2(a0.x, a0.y);
+                                    o4.y = pack_bf16x2(a0.z, a0.w);
+                                    o4.z = pack_bf16x2(a1.x, a1.y);
+                                    o4.w = pack_bf16x2(a1.z, a1.w);
+                                    *reinterpret_cast<uint4 *>(orow + q2 * 16) = o4;
+                                    o4.x = pack_bf16x2(a2.x, a2.y);
+                                    o4.y = pack_bf16x2(a2.z, a2.w);
+                                    o4.z = pack_bf16x2(a3.x, a3.y);
+                                    o4.w = pack_bf16x2(a3.z, a3.w);
+                                    *reinterpret_cast<uint4 *>(orow + q2 * 16 + 8) = o4;
                                 }
                             }
                         }

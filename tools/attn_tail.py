@@ -13,6 +13,7 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="C2")
 ap.add_argument("--batch", type=int, default=1)
 ap.add_argument("--prefix", type=int, default=None)
+ap.add_argument("--expansion", default=None, help="override the tree: comma list <k1,..,km>")
 ap.add_argument("--flags", type=int, default=0, help="debug flags (64: no split-KV clusters)")
 a = ap.parse_args()
 os.environ["SPECINFER_DEBUG_FLAGS"] = str(a.flags)
@@ -20,11 +21,11 @@ spi.specinfer_debug_set_trace(None)
 cfg = W.CONFIGS[a.config]
 dev = torch.device("cuda:0")
 P = a.prefix or cfg.prefix
-p, d = cfg.tree
-tb = W.make_tree_batch([(p, d)] * a.batch, [P] * a.batch, device=dev, max_depth=cfg.max_depth)
+p, d = cfg.tree if not a.expansion else W.expansion_tree([int(x) for x in a.expansion.split(",")])
+tb = W.make_tree_batch([(p, d)] * a.batch, [P] * a.batch, device=dev, max_depth=max(cfg.max_depth, int(d.max())))
 smax = P + tb.max_nodes
 ai = W.make_attention_inputs(tb, 1, cfg.num_q_heads, cfg.num_kv_heads, smax, seed=1, device=dev)
-shape = spi.make_shape(a.batch, tb.max_nodes, cfg.num_q_heads, cfg.num_kv_heads, smax, max_depth=cfg.max_depth)
+shape = spi.make_shape(a.batch, tb.max_nodes, cfg.num_q_heads, cfg.num_kv_heads, smax, max_depth=tb.max_depth)
 st = spi.TreeState.create(shape, tb.parent, tb.depth, tb.prefix_len, tb.n_nodes)
 st.prepare()
 out = torch.empty_like(ai.q[0])
