@@ -62,9 +62,10 @@ def parse():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-early", action="store_true", help="plain attention launches (no EARLY_PREFIX)")
     ap.add_argument("--verify", default=None, help="comma list overriding the config's verify modes")
-    ap.add_argument("--gather", default="p2p", choices=["p2p", "nccl"],
-                    help="tokens-only exchange: fused into the verifier with peer stores (NEXT-4a, default) or an "
-                         "NCCL all-gather between the verify and commit graphs (the baseline)")
+    ap.add_argument("--gather", default="auto", choices=["auto", "p2p", "nccl"],
+                    help="tokens-only exchange: fused into the verifier with peer stores (NEXT-4a) or an NCCL "
+                         "all-gather between the verify and commit graphs (the baseline); auto = p2p when there "
+                         "is something to exchange (N > 1 or kv-head sharding), else none")
     ap.add_argument("--shard", default="auto", choices=["auto", "request", "kv"],
                     help="layout: request sharding, or kv-head sharding (GQA; auto for G > 1 at N > 1)")
     return ap.parse_args()
@@ -240,7 +241,10 @@ def run_ours(args, ws, rank, local):
     from paper_conf_asplos_miaoozcwzwzyssc24_b200 import dist as D
     p2p, gather_note = None, "NCCL all_gather_into_tensor between the verify and commit graphs" if ws > 1 else \
         "local copy (N = 1)"
-    if args.gather == "p2p":
+    need_gather = ws > 1 or kv_shard or args.gather != "auto"
+    if not need_gather:
+        gather_note = "none (N = 1, request-sharded: the verifier's own output is the whole table)"
+    if args.gather in ("auto", "p2p") and need_gather:
         try:
             p2p = D.P2PGather(Bg, ws, rank, Lp, device, exchange=D.all_gather_object_exchange if ws > 1 else None)
             gather_note = ("fused into the committed verifier: peer stores of every request's row + epoch flags "
@@ -268,7 +272,7 @@ def run_ours(args, ws, rank, local):
             step.gather()    # device-side wait for every rank's rows (graph-capturable)
 
     def gather_between():
-        if p2p is None:
+        if p2p is None and need_gather:
             step.gather()    # NCCL / local copy: eager, between the verify and commit graphs
 
     def seg_commit():
@@ -328,6 +332,9 @@ def run_ours(args, ws, rank, local):
     step_ms = [ev[k][0].elapsed_time(ev[k + 1][0]) for k in range(K - 1)] + \
               [ev[K - 1][0].elapsed_time(e_all[1])]
     attn_ms = sum(ev[k][1].elapsed_time(ev[k][2]) for k in range(K))
+    prep_ms = sum(ev[k][0].elapsed_time(ev[k][1]) for k in range(K)) / K
+    post_ms = (sum(ev[k][2].elapsed_time(ev[k + 1][0]) for k in range(K - 1)) +
+               ev[K - 1][2].elapsed_time(e_all[1])) / K
     attn_ms_max = max_over_ranks(attn_ms, ws, device)
     ms_per_step = total_ms / K
     tokens_step_global = int(wl.tree_tokens_per_step())
@@ -521,7 +528,9 @@ def run_ours(args, ws, rank, local):
         "extra": {"tree_tokens_per_step": tokens_step_global,
                   "mean_n_accepted": acc, "committed_verifier": step.commit_mode,
                   "accepted_tokens_per_s_rank0": round(float(na_c.sum().item()) * K / (total_ms / 1e3), 1),
-                  "attention_ms_per_step": round(attn_ms_max / K, 4)},
+                  "attention_ms_per_step": round(attn_ms_max / K, 4),
+                  "prepare_ms_per_step": round(prep_ms, 4),
+                  "verify_gather_commit_ms_per_step": round(post_ms, 4)},
     }
     if rank == 0:
         print(json.dumps(line), flush=True)

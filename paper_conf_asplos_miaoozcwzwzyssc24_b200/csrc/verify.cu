@@ -1,9 +1,10 @@
 // verify.cu — K4 verify_greedy and K5 verify_mss, sm_100a.
 //
 // VerifyGreedy (Alg. 2 lines 16-22, L395-401; §4.3): one CTA per (node, request)
-// computes O(u) = argmax_x logits[u][x] (128-bit loads, 4 in flight per thread, warp-shuffle
+// computes O(u) = argmax_x logits[u][x] (128-bit loads, 8 in flight per thread, warp-shuffle
 // argmax with the lowest index on ties, reading R7); the last CTA of a request (counter in the
-// workspace) walks the tree from the root.  One launch.
+// workspace) stages parents, tokens and O(u) in shared memory and walks the tree from the root
+// there.  One launch.
 //
 // Naive sampling (NEXT-3, L747-753, the baseline of Theorem 4.3) reuses the K4 kernel: the
 // per-node key is the exponential-race key of x ~ softmax(l / T) instead of the logit, and the
@@ -207,6 +208,7 @@ __global__ void __launch_bounds__(kGreedyThreads) verify_greedy_kernel(
     const int n = n_nodes[b];
     __shared__ ArgMax sh[32];
     __shared__ int s_last;
+    __shared__ int32_t s_par[kMaxNodes], s_tok[kMaxNodes], s_o[kMaxNodes];
     if (!req_ok[b]) {
         if (u == 0) {
             for (int j = threadIdx.x; j < path_len; j += blockDim.x) {
@@ -258,21 +260,29 @@ __global__ void __launch_bounds__(kGreedyThreads) verify_greedy_kernel(
     __syncthreads();
     if (!s_last) return;
     // ---- last CTA of this request: the greedy walk (one warp) ----
+    // parents, tokens and every node's O(u) are staged in shared memory with one round of
+    // parallel loads (one L2 round trip), so the walk itself is dependent shared-memory reads only
     if (threadIdx.x >= 32) return;
     __threadfence();
     const int lane = threadIdx.x;
     const int32_t *par = parent + (size_t)b * Nmax;
     const int32_t *tok = tree_tokens + (size_t)b * Nmax;
+    for (int j = lane; j < n; j += 32) {
+        s_par[j] = par[j];
+        s_tok[j] = tok[j];
+        s_o[j] = __ldcg(argmax_ws + (size_t)b * Nmax + j);
+    }
+    __syncwarp();
     int32_t *an = acc_nodes + (size_t)b * path_len;
     int32_t *at = acc_tokens + (size_t)b * path_len;
     int cur = 0, cnt = 0;
     if (lane == 0) an[0] = 0;
     for (;;) {
-        const int o = __ldcg(argmax_ws + (size_t)b * Nmax + cur);
+        const int o = s_o[cur];
         int next = -1;
         for (int base = cur + 1; base < n && next < 0; base += 32) {
             const int cidx = base + lane;
-            const bool hit = cidx < n && par[cidx] == cur && tok[cidx] == o;
+            const bool hit = cidx < n && s_par[cidx] == cur && s_tok[cidx] == o;
             const unsigned m = __ballot_sync(0xffffffffu, hit);
             if (m) next = base + __ffs(m) - 1;
         }
@@ -281,7 +291,7 @@ __global__ void __launch_bounds__(kGreedyThreads) verify_greedy_kernel(
             break;
         }
         if (lane == 0) {
-            at[cnt] = tok[next];
+            at[cnt] = s_tok[next];
             an[cnt + 1] = next;
         }
         ++cnt;
