@@ -7,11 +7,14 @@
 //    accumulator, P (bf16 pairs) in its own columns, so the S buffer of tile t is free as soon as
 //    the softmax has loaded it and S(t + 2) never waits for PV(t) (round 1 aliased P over S and the
 //    chain S -> softmax -> PV -> S(t + 2) bounded the kernel);
-//  * 8 softmax warps, two per TMEM lane quarter: thread (row r, half h) owns keys [64 h, 64 h + 64)
-//    of every tile and dims [64 h, 64 h + 64) of O; the two halves of a row exchange their partial
-//    tile maxima through shared memory (one 64-thread barrier per tile), so both hold the same
-//    stale running max; O is rescaled in TMEM (after PV(t - 1)) only when a tile raises a row's
-//    max by more than 2^8;
+//  * 8 softmax warps in two groups of 4 (one warp per TMEM lane quarter each, thread = query row);
+//    group g owns the tiles with t & 1 == g and both accumulate into the one O, so every P(t) uses
+//    the row reference the previous tile left: the owner of tile t reads decision(t - 1) from the
+//    other group (shared memory + one named barrier per direction and lane quarter), may raise it
+//    (stale max: only beyond 2^8, then O is rescaled in TMEM after PV(t - 1)), publishes decision(t)
+//    and only then computes its exponentials -- the groups run out of phase;
+//  * segment end: the owner of the last tile combines both groups' row sums, then both groups write
+//    half of the output row each (a whole item) or the owner writes the fp32 partial (a split piece);
 //  * K and V in separate TMA rings fed by two producer lanes; S issuer and PV issuer threads;
 //  * lane mode (schedule_kernel): the row blocks of one (request, kv-head) run on `lanes` CTAs in
 //    lock-step over the same tile range, so each KV tile is read from HBM once;
@@ -42,7 +45,8 @@ struct Misc {
     uint64_t stage_bar;                      // bulk staging of split pieces (CTA's last segment)
     uint32_t tmem_base;
     int32_t bcast;
-    float xm[2][2][RB];                      // [0][0]: row references; [1][0] / [1][1]: segment-end hand-over
+    float xm[2][2][RB];                      // [0][0]: row references; [0][1]: the row's final sum;
+                                             // [1][0] / [1][1]: segment-end hand-over
 };
 
 __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
@@ -54,6 +58,28 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
           "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
           "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
         : "r"(taddr));
+}
+
+// The normalised bf16 output of one query row, dims [64 h, 64 h + 64) (TMEM columns of O), with
+// 16-byte stores; both TMEM loads are issued before the first wait.
+__device__ __forceinline__ void store_o_half(uint32_t o_col, float inv, bool row_valid, __nv_bfloat16 *orow, int h) {
+    uint32_t o[2][32];
+    tmem_ld32(o_col + h * 64, o[0]);
+    tmem_ld32(o_col + h * 64 + 32, o[1]);
+    tmem_ld_wait();
+    if (!row_valid) return;
+#pragma unroll
+    for (int q = 0; q < 2; ++q) {
+#pragma unroll
+        for (int i = 0; i < 32; i += 8) {
+            uint4 w;
+            w.x = pack_bf16x2(__uint_as_float(o[q][i]) * inv, __uint_as_float(o[q][i + 1]) * inv);
+            w.y = pack_bf16x2(__uint_as_float(o[q][i + 2]) * inv, __uint_as_float(o[q][i + 3]) * inv);
+            w.z = pack_bf16x2(__uint_as_float(o[q][i + 4]) * inv, __uint_as_float(o[q][i + 5]) * inv);
+            w.w = pack_bf16x2(__uint_as_float(o[q][i + 6]) * inv, __uint_as_float(o[q][i + 7]) * inv);
+            *reinterpret_cast<uint4 *>(orow + h * 64 + q * 32 + i) = w;
+        }
+    }
 }
 
 // D[tmem] (+)= A[tmem] * B[smem desc], kind::f16 (A = P, bf16 packed two per column)
@@ -170,7 +196,7 @@ __global__ void __launch_bounds__(352, 1)
             mbar_init(&misc->p_full[i], 4);
             mbar_init(&misc->pv_done[i], 1);
         }
-        mbar_init(&misc->o_free, 4);
+        mbar_init(&misc->o_free, 8);   // every softmax warp (both groups share the epilogue)
         mbar_init(&misc->stage_bar, 1);
         for (int i = 0; i < kSegRing; ++i) mbar_init(&misc->seg_full[i], 1);
         fence_barrier_init();
@@ -399,12 +425,18 @@ __global__ void __launch_bounds__(352, 1)
         const int qd = warp & 3;               // TMEM lane quarter
         const int r = qd * 32 + lane;          // query row of the item = TMEM lane
         const uint32_t lane_off = (uint32_t)(qd * 32) << 16;
-        const uint32_t dec_bar = 6 + qd;       // decision(t) hand-over between the two warps of quarter qd
+        // decision(t) hand-over between the two warps of quarter qd: one named barrier PER DIRECTION.
+        // (With a single barrier, the publisher's arrive(t) and its own sync at tile t + 2 could complete
+        // the barrier together whenever the other warp reached its sync for t + 1 late -- the publisher
+        // would then read a stale reference.  Per direction, arrivals and syncs strictly alternate.)
+        const uint32_t dec_out = grp == 0 ? 6 + qd : 1 + qd;   // the decisions this group publishes
+        const uint32_t dec_in = grp == 0 ? 1 + qd : 6 + qd;    // the other group's decisions
         const uint32_t epi_bar = 10 + qd;      // segment-end row-sum hand-over
         const uint32_t o_col = tmem + kColO + lane_off;
         float *mref_s = misc->xm[0][0];        // [row] the row reference after the latest decision
         float *xl_l = misc->xm[1][0];          // [row] the non-owner group's row sum at a segment end
         float *xl_m = misc->xm[1][1];          //       ... and the reference it is relative to
+        float *xl_f = misc->xm[0][1];          // [row] the final row sum (owner -> the other group)
         int lt = 0, ls = 0;
         for (;;) {
             mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
@@ -471,7 +503,7 @@ __global__ void __launch_bounds__(352, 1)
                 }
                 // decision(t - 1): the reference P(t - 1) used (ignored at a segment's first tile: new rows)
                 if (lt > 0) {
-                    named_bar_sync(dec_bar, 64);
+                    named_bar_sync(dec_in, 64);
                     const float mp = mref_s[r];
                     if (lt > lt0 && mp != m) {   // the other group raised it: rebase this group's sum
                         l = (m == -INFINITY) ? 0.f : l * ex2(m - mp);
@@ -488,7 +520,11 @@ __global__ void __launch_bounds__(352, 1)
                 }
                 const bool moved = __any_sync(0xffffffffu, alpha != 1.f) && lt > lt0;
                 if (moved) {
-                    // O holds PV(<= t - 1) against the old reference: rescale once PV(t - 1) completed
+                    // O holds PV(<= t - 1) against the old reference: rescale once PV(t - 1) completed.
+                    // This group last observed pv_done of ITS parity (PV(t - 4)); the other barrier may
+                    // still be a phase behind PV(t - 1)'s, which a parity wait cannot tell apart from
+                    // "complete": first PV(t - 2) (own barrier, one phase ahead), which implies PV(t - 3).
+                    if (lt >= 2) mbar_wait(&misc->pv_done[lt & 1], ((lt - 2) >> 1) & 1);
                     mbar_wait(&misc->pv_done[(lt - 1) & 1], ((lt - 1) >> 1) & 1);
                     tc_fence_after();
 #pragma unroll 1
@@ -507,7 +543,7 @@ __global__ void __launch_bounds__(352, 1)
                     tmem_st_wait();
                 }
                 mref_s[r] = m;
-                named_bar_arrive(dec_bar, 64);   // decision(t) -> the owner of tile t + 1
+                named_bar_arrive(dec_out, 64);   // decision(t) -> the owner of tile t + 1
                 // pass 2: P(t) = 2^(s * scale - m) as bf16 pairs into P buffer t & 1 (free once PV(t - 2)
                 // completed), row sum of the rounded values
                 if (lt >= 2) mbar_wait(&misc->pv_done[sb], ((lt - 2) >> 1) & 1);
@@ -546,45 +582,47 @@ __global__ void __launch_bounds__(352, 1)
                 if (r == 0) SPI_TRACE(6 + grp);
             }
 
-            // ============ epilogue of this segment (the owner of its last tile writes the rows) ============
+            // ============ epilogue of this segment ============
+            // The owner of the segment's last tile combines both groups' row sums; for a whole item both
+            // groups then write half of the row's 128 dims each (the output store of one group alone
+            // stalled the other group's next tile for the whole epilogue), a split piece is written by
+            // the owner.
             const int llast = lt - 1;
             const int owner = llast & 1;
+            const bool full = (sd.begin == sd.ib) && (sd.end == sd.ie);
             // (two full barriers: the non-owner may not overwrite the hand-over slots of the next segment
-            // before the owner has read them)
+            // before the owner has read them, and it reads the final sum only after the owner wrote it)
             if (grp != owner) {
                 xl_l[r] = l;
                 xl_m[r] = m;
                 named_bar_sync(epi_bar, 64);
                 named_bar_sync(epi_bar, 64);
+                if (full) {
+                    const float inv = 1.0f / xl_f[r];
+                    // O complete: this group last observed pv_done of ITS parity, so first wait for PV(llast - 1)
+                    // (its own tile: at most one phase ahead), which implies PV(llast - 2); only then is the
+                    // parity wait for PV(llast) on the other barrier unambiguous
+                    if (llast >= 1) mbar_wait(&misc->pv_done[(llast - 1) & 1], ((llast - 1) >> 1) & 1);
+                    mbar_wait(&misc->pv_done[llast & 1], (llast >> 1) & 1);
+                    tc_fence_after();
+                    store_o_half(o_col, inv, row_valid,
+                                 p.out + (((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim, 1);
+                }
+                tc_fence_before();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&misc->o_free);
             } else {
                 named_bar_sync(epi_bar, 64);
                 const float lo_ = xl_l[r], mo = xl_m[r];
-                named_bar_sync(epi_bar, 64);
                 const float lrow = l + ((mo == -INFINITY || lo_ == 0.f) ? 0.f : lo_ * ex2(mo - m));
+                xl_f[r] = lrow;
+                named_bar_sync(epi_bar, 64);
                 mbar_wait(&misc->pv_done[llast & 1], (llast >> 1) & 1);   // O complete (in-order PVs)
                 tc_fence_after();
                 if (r == 0) SPI_TRACE(10);
-                const bool full = (sd.begin == sd.ib) && (sd.end == sd.ie);
                 if (full) {
-                    const float inv = 1.0f / lrow;
-                    __nv_bfloat16 *orow = p.out + (((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim;
-#pragma unroll 1
-                    for (int q2 = 0; q2 < 4; ++q2) {
-                        uint32_t o[32];
-                        tmem_ld32(o_col + q2 * 32, o);
-                        tmem_ld_wait();
-                        if (row_valid) {
-#pragma unroll
-                            for (int i = 0; i < 32; i += 8) {
-                                uint4 w;
-                                w.x = pack_bf16x2(__uint_as_float(o[i]) * inv, __uint_as_float(o[i + 1]) * inv);
-                                w.y = pack_bf16x2(__uint_as_float(o[i + 2]) * inv, __uint_as_float(o[i + 3]) * inv);
-                                w.z = pack_bf16x2(__uint_as_float(o[i + 4]) * inv, __uint_as_float(o[i + 5]) * inv);
-                                w.w = pack_bf16x2(__uint_as_float(o[i + 6]) * inv, __uint_as_float(o[i + 7]) * inv);
-                                *reinterpret_cast<uint4 *>(orow + q2 * 32 + i) = w;
-                            }
-                        }
-                    }
+                    store_o_half(o_col, 1.0f / lrow, row_valid,
+                                 p.out + (((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim, 0);
                     tc_fence_before();
                     __syncwarp();
                     if (lane == 0) mbar_arrive(&misc->o_free);   // the next segment's first PV may overwrite O
@@ -779,7 +817,7 @@ __global__ void __launch_bounds__(352, 1)
             ++ls;
         }
         // the last tile's decision has no next owner: consume it so every barrier phase completes
-        if (lt > 0 && ((lt - 1) & 1) != grp) named_bar_sync(dec_bar, 64);
+        if (lt > 0 && ((lt - 1) & 1) != grp) named_bar_sync(dec_in, 64);
     }
 
     tc_fence_before();

@@ -329,6 +329,53 @@ def _torch_reference_check(out, ai, tb, Hq, Hkv):
         assert e.max().item() <= MAX_ABS and e.mean().item() <= MEAN_ABS
 
 
+@pytest.mark.parametrize("name,batch", [("C4", 16), ("C3", 32), ("C2", 16)])
+def test_attention_rescales_across_segments(name, batch):
+    """Production shapes (every CTA runs many segments) with keys ramped along the sequence, so the
+    rows' running reference moves on most tiles (stale-max rescales of O) while the softmax groups
+    hand decisions and segment ends to each other.  Eight launches must be bit-identical (the two
+    latent races this guards against -- a shared decision barrier that the publisher could complete
+    itself, and an ambiguous parity wait before a rescale -- made the rows kernel non-deterministic
+    here), and every row must match an fp32 torch reference, sampled rows the oracle."""
+    cfg = W.CONFIGS[name]
+    tb = W.config_tree_batch(cfg, device=DEV, ragged=True, batch=batch)
+    smax = cfg.prefix + tb.max_nodes + 3
+    ai = W.make_attention_inputs(tb, 1, cfg.num_q_heads, cfg.num_kv_heads, smax, seed=cfg.seed + 5, device=DEV)
+    ramp = torch.linspace(0.2, 3.0, smax, device=DEV).view(1, 1, smax, 1)
+    ai.k_cache[0].copy_((ai.k_cache[0].float() * ramp).to(torch.bfloat16))
+    out, st = _gpu_attention(tb, ai, cfg.num_q_heads, cfg.num_kv_heads)
+    for _ in range(7):
+        again = torch.full_like(out, float("nan"))
+        st.attention(ai.q[0], ai.k_cache[0], ai.v_cache[0], again)
+        torch.cuda.synchronize()
+        assert torch.equal(torch.nan_to_num(again, nan=7.0), torch.nan_to_num(out, nan=7.0))
+    # fp32 torch reference, every row; the bar is relative to max(1, |ref|) as in the spike test
+    # (peaked rows: |out| approaches |v|, where one bf16 rounding of the output is ~|v| 2^-8)
+    B, N = tb.parent.shape
+    G = cfg.num_q_heads // cfg.num_kv_heads
+    par, n, pl = tb.parent.cpu().numpy(), tb.n_nodes.cpu().numpy(), tb.prefix_len.cpu().numpy()
+    for b in range(B):
+        P, nb = int(pl[b]), int(n[b])
+        mask = torch.ones((nb, P + nb), dtype=torch.bool, device=DEV)
+        anc = torch.zeros((nb, nb), dtype=torch.bool)
+        for i in range(nb):
+            u = i
+            while u >= 0:
+                anc[i, u] = True
+                u = par[b, u]
+        mask[:, P:] = anc.to(DEV)
+        k = ai.k_cache[0, b, :, :P + nb].float().repeat_interleave(G, 0)
+        v = ai.v_cache[0, b, :, :P + nb].float().repeat_interleave(G, 0)
+        ref = torch.nn.functional.scaled_dot_product_attention(ai.q[0, b, :nb].float().permute(1, 0, 2), k, v,
+                                                               attn_mask=mask)
+        e = (out[b, :nb].float().permute(1, 0, 2) - ref).abs()
+        assert (e <= MAX_ABS * ref.abs().clamp(min=1.0)).all() and e.mean().item() <= MEAN_ABS, (b, e.max().item())
+    ref_o = _oracle_attention(ai, tb, bs=[0])
+    g = out[0, :n[0]].float().cpu().numpy()
+    e = np.abs(g - ref_o[0, :n[0]])
+    assert np.all(e <= MAX_ABS * np.maximum(1.0, np.abs(ref_o[0, :n[0]]))) and e.mean() <= MEAN_ABS
+
+
 @pytest.mark.parametrize("n,B,P", [(8, 64, 512), (32, 8, 2048), (128, 4, 8192), (256, 2, 2048), (64, 1, 512)])
 def test_config_c5_points(n, B, P):
     """C5 sweep points (random trees, depth <= 8), one layer, sampled requests vs the oracle."""

@@ -15,6 +15,7 @@ ap.add_argument("--batch", type=int, default=1)
 ap.add_argument("--prefix", type=int, default=None)
 ap.add_argument("--expansion", default=None, help="override the tree: comma list <k1,..,km>")
 ap.add_argument("--flags", type=int, default=0, help="debug flags (64: no split-KV clusters)")
+ap.add_argument("--all", action="store_true", help="print every traced tile of CTAs 0-1")
 a = ap.parse_args()
 os.environ["SPECINFER_DEBUG_FLAGS"] = str(a.flags)
 spi.specinfer_debug_set_trace(None)
@@ -60,5 +61,7 @@ for c in range(8):
     print(f"CTA {c} exit {ex[c]:.2f} us, raw per-tile events (cycles rel. to its first K issue; -1 none): "
           "K-iss V-iss S-mma PV-mma 4..11")
     show = list(range(min(nv + 1, 8))) + [i for i in range(max(8, nv - 3), min(nv + 2, 64))]
+    if a.all and c < 2:
+        show = list(range(min(nv + 1, 64)))
     for i in show:
         print(f"  {i:3d} " + " ".join(f"{(v - base) if v else -1:7d}" for v in x[i, :16]))
