@@ -517,7 +517,7 @@ int32_t specinfer_debug_hooks_enabled(void) {
 
 int32_t specinfer_launches_per_call(const char *name) {
     if (!name) return -1;
-    if (!strcmp(name, "tree_prepare")) return 2;     // validate+bitsets, schedule (+1 memset)
+    if (!strcmp(name, "tree_prepare")) return 2;     // validate+bitsets, schedule+status
     if (!strcmp(name, "tree_attention")) return 1;   // split combine fused (last piece merges)
     if (!strcmp(name, "tree_attention_ex")) return 1;
     if (!strcmp(name, "verify_greedy")) return 1;    // argmax + walk fused (last CTA walks)

@@ -10,37 +10,33 @@
 
 namespace specinfer {
 
-__global__ void __launch_bounds__(256) tree_validate_bitsets_kernel(
-    const int32_t *__restrict__ parent, const int32_t *__restrict__ depth,
+constexpr int kPrepThreads = 512;
+
+// Per request (one CTA): validate the tree and build its bitsets / row masks.  Parents and depths
+// are staged in shared memory first (one round of loads), desc = the transpose of anc is built
+// 32 x 32 bits at a time with warp ballots.
+__device__ void validate_bitsets(
+    int b, const int32_t *__restrict__ parent, const int32_t *__restrict__ depth,
     const int32_t *__restrict__ prefix_len, const int32_t *__restrict__ n_nodes, int Nmax,
     int max_depth, int Smax, int G, int npc, int chunks, int32_t *__restrict__ status, int32_t *__restrict__ req_ok,
     uint32_t *__restrict__ anc, uint32_t *__restrict__ desc, unsigned long long *__restrict__ rowmask) {
-    const int b = blockIdx.x;
-    __shared__ int32_t s_par[kMaxNodes];
+    __shared__ int32_t s_par[kMaxNodes], s_dep[kMaxNodes];
     __shared__ uint32_t s_anc[kMaxNodes][kBitWords];
     __shared__ int s_bad;
     const int n = n_nodes[b];
     const int P = prefix_len[b];
-    if (threadIdx.x == 0) {
-        int bad = (n < 1 || n > Nmax || P < 0 || (long long)P + n > Smax) ? 1 : 0;
-        s_bad = bad;
+    if (threadIdx.x == 0) s_bad = (n < 1 || n > Nmax || P < 0 || (long long)P + n > Smax) ? 1 : 0;
+    for (int i = threadIdx.x; i < Nmax; i += blockDim.x) {
+        s_par[i] = parent[(size_t)b * Nmax + i];
+        s_dep[i] = depth[(size_t)b * Nmax + i];
     }
     __syncthreads();
     const bool n_ok = !s_bad;
-    for (int i = threadIdx.x; i < Nmax; i += blockDim.x) {
-        const int p = parent[(size_t)b * Nmax + i];
-        s_par[i] = p;
-        if (n_ok && i < n) {
-            const int d = depth[(size_t)b * Nmax + i];
-            bool bad;
-            if (i == 0) {
-                bad = (p != -1) || (d != 0);
-            } else {
-                bad = (p < 0) || (p >= i) || (d > max_depth) ||
-                      (d != depth[(size_t)b * Nmax + p] + 1);
-            }
-            if (bad) atomicOr(&s_bad, 1);
-        }
+    for (int i = threadIdx.x; n_ok && i < n; i += blockDim.x) {
+        const int p = s_par[i], d = s_dep[i];
+        const bool bad = (i == 0) ? (p != -1 || d != 0)
+                                  : (p < 0 || p >= i || d > max_depth || d != s_dep[p] + 1);
+        if (bad) atomicOr(&s_bad, 1);
     }
     __syncthreads();
     const bool ok = !s_bad;
@@ -52,7 +48,9 @@ __global__ void __launch_bounds__(256) tree_validate_bitsets_kernel(
         if (ok && i < n) {
             int u = i;
             while (u >= 0) {
-                w[u >> 5] |= 1u << (u & 31);
+#pragma unroll
+                for (int k = 0; k < kBitWords; ++k)
+                    if ((u >> 5) == k) w[k] |= 1u << (u & 31);
                 u = s_par[u];
             }
         }
@@ -63,17 +61,24 @@ __global__ void __launch_bounds__(256) tree_validate_bitsets_kernel(
         }
     }
     __syncthreads();
-    // descendant-or-self bitsets: desc[j] bit i  <=>  anc[i] bit j
-    for (int j = threadIdx.x; j < Nmax; j += blockDim.x) {
-        uint32_t w[kBitWords];
-#pragma unroll
-        for (int k = 0; k < kBitWords; ++k) w[k] = 0;
-        if (ok && j < n) {
-            for (int i = j; i < n; ++i)
-                if ((s_anc[i][j >> 5] >> (j & 31)) & 1u) w[i >> 5] |= 1u << (i & 31);
+    // descendant-or-self bitsets: desc[j] bit i  <=>  anc[i] bit j; warp task (iw, jw) transposes
+    // the 32 x 32 block of rows i in [32 iw, 32 iw + 32) and columns j in [32 jw, 32 jw + 32)
+    {
+        const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+        const int njw = (Nmax + 31) >> 5;
+        for (int task = wid; task < njw * kBitWords; task += nw) {
+            const int jw = task / kBitWords, iw = task % kBitWords;
+            const int i = 32 * iw + lane;
+            const uint32_t a = (i < Nmax) ? s_anc[i][jw] : 0u;   // rows past n / invalid trees are 0
+            uint32_t mine = 0u;
+#pragma unroll 8
+            for (int k = 0; k < 32; ++k) {
+                const uint32_t col = __ballot_sync(0xffffffffu, (a >> k) & 1u);
+                if (lane == k) mine = col;
+            }
+            const int j = 32 * jw + lane;
+            if (j < Nmax) desc[((size_t)b * Nmax + j) * kBitWords + iw] = mine;
         }
-#pragma unroll
-        for (int k = 0; k < kBitWords; ++k) desc[((size_t)b * Nmax + j) * kBitWords + k] = w[k];
     }
     // row masks of the tree part for the attention kernel: bit r of rowmask[b][c][j] is set iff
     // query row r of chunk c (node c*npc + r/G) exists and has tree node j on its root path
@@ -89,10 +94,7 @@ __global__ void __launch_bounds__(256) tree_validate_bitsets_kernel(
         }
         rowmask[((size_t)b * chunks + c) * Nmax + j] = m;
     }
-    if (threadIdx.x == 0) {
-        req_ok[b] = ok ? 1 : 0;
-        if (!ok) atomicOr(status, kStatusBadTree);
-    }
+    if (threadIdx.x == 0) req_ok[b] = ok ? 1 : 0;   // (the schedule kernel sets the status words)
 }
 
 // Single block: tiles per schedule unit, exclusive scan, total; zero the split/verify counters.
@@ -100,9 +102,9 @@ __global__ void __launch_bounds__(256) tree_validate_bitsets_kernel(
 // the rows-as-M kernel).  In lane mode CTA c runs chunk c % lanes of every unit in its tile range
 // [t0, t1) of the unit stream, so the `lanes` CTAs of a group read the same KV tile at about the
 // same time: one HBM read, the other chunks hit L2.
-__global__ void __launch_bounds__(1024) schedule_kernel(
+__device__ void schedule(
     const int32_t *__restrict__ prefix_len, const int32_t *__restrict__ n_nodes,
-    const int32_t *__restrict__ req_ok, int B, int Hkv, int chunks, int npc, int lanes,
+    const int32_t *req_ok, int B, int Hkv, int chunks, int npc, int lanes,
     int32_t *__restrict__ item_start, uint32_t *__restrict__ item_cnt, int4 *__restrict__ item_info,
     int4 *__restrict__ cta_info, int num_ctas, int splitk, uint32_t *__restrict__ verify_cnt,
     int32_t *__restrict__ status, int no_split_slack) {
@@ -111,16 +113,40 @@ __global__ void __launch_bounds__(1024) schedule_kernel(
     const int per = (n_units + blockDim.x - 1) / blockDim.x;
     const int lo = threadIdx.x * per;
     const int hi = min(n_units, lo + per);
+    // per-request (n, P, ok) and the unit tile prefix live in shared memory when they fit, so the
+    // schedule is one round of global loads and then shared-memory work (this block runs on the
+    // critical path of every step; each dependent L2 round trip is ~0.5 us)
+    constexpr int kSmB = 1024, kSmU = 4096;
+    __shared__ int s_n[kSmB], s_P[kSmB], s_ok[kSmB];
+    __shared__ int s_start[kSmU + 1];
+    const bool smB = B <= kSmB, smU = n_units <= kSmU;
+    if (smB)
+        for (int b = threadIdx.x; b < B; b += blockDim.x) {
+            s_n[b] = n_nodes[b];
+            s_P[b] = prefix_len[b];
+            s_ok[b] = __ldcg(req_ok + b);   // written by the other CTAs of the launch
+        }
+    __syncthreads();
+    // status words of this tree: [0] = bad-tree bit if any request failed validation (replaces every
+    // earlier sticky bit), [1] = total tiles (below), [2..63] = 0
+    int bad_local = 0;
+    for (int b = threadIdx.x; b < B; b += blockDim.x) bad_local |= (smB ? s_ok[b] : __ldcg(req_ok + b)) == 0;
+    const int any_bad = __syncthreads_or(bad_local);
+    if (threadIdx.x == 0) status[0] = any_bad ? kStatusBadTree : 0;
+    for (int i = 2 + threadIdx.x; i < 64; i += blockDim.x) status[i] = 0;
+    auto N_of = [&](int b) { return smB ? s_n[b] : n_nodes[b]; };
+    auto P_of = [&](int b) { return smB ? s_P[b] : prefix_len[b]; };
+    auto ok_of = [&](int b) { return smB ? s_ok[b] : __ldcg(req_ok + b); };
     // tiles of unit u: a unit's chunks share its KV stream; an empty chunk (c * npc >= n) of a
     // lane-mode unit keeps the unit's tile range and is skipped by its CTAs (n field 0)
     auto tiles_of = [&](int u) -> int {
         const int x = u * lanes;
         const int c = x % chunks;
         const int b = x / (chunks * Hkv);
-        if (!req_ok[b]) return 0;
-        const int n = n_nodes[b];
+        if (!ok_of(b)) return 0;
+        const int n = N_of(b);
         if (c * npc >= n) return 0;
-        return (prefix_len[b] + n + kKeyTile - 1) / kKeyTile;
+        return (P_of(b) + n + kKeyTile - 1) / kKeyTile;
     };
     int local = 0, local_max = 0;
     for (int u = lo; u < hi; ++u) {
@@ -157,12 +183,13 @@ __global__ void __launch_bounds__(1024) schedule_kernel(
     for (int u = lo; u < hi; ++u) {
         const int tl = tiles_of(u);
         item_start[u] = run;
+        if (smU) s_start[u] = run;
         for (int x = u * lanes; x < (u + 1) * lanes; ++x) {
             const int b = x / (chunks * Hkv);
             const int c = x % chunks;
-            const int n = n_nodes[b];
+            const int n = N_of(b);
             const bool empty = lanes > 1 && c * npc >= n;
-            item_info[x] = make_int4(run, run + tl, prefix_len[b], empty ? 0 : n);
+            item_info[x] = make_int4(run, run + tl, P_of(b), empty ? 0 : n);
             item_cnt[x] = 0u;
         }
         run += tl;
@@ -170,6 +197,7 @@ __global__ void __launch_bounds__(1024) schedule_kernel(
     __shared__ int s_total;
     if (threadIdx.x == blockDim.x - 1) {
         item_start[n_units] = run;
+        if (smU) s_start[n_units] = run;
         item_info[n_items] = make_int4(run, run, 0, 0);
         status[1] = run;
         s_total = run;
@@ -192,6 +220,14 @@ __global__ void __launch_bounds__(1024) schedule_kernel(
     const int upc = (n_units + NCv - 1) / NCv;
     const bool one_per_cta = n_units > 0 &&
         (long long)upc * s_max_tiles * NCv <= T + (long long)kNoSplitSlack * NCv;
+    auto start_of = [&](int u) { return smU ? s_start[u] : item_start[u]; };
+    auto info_of = [&](int x) -> int4 {   // == item_info[x], rebuilt from shared memory
+        if (!smU || !smB) return item_info[x];
+        const int u = x / lanes, b = x / (chunks * Hkv), c = x % chunks;
+        const int n = s_n[b];
+        const bool empty = lanes > 1 && c * npc >= n;
+        return make_int4(s_start[u], s_start[u + 1], s_P[b], empty ? 0 : n);
+    };
     for (int c = threadIdx.x; c < num_ctas; c += blockDim.x) {
         const int vc = c / lanes, cl = c % lanes;
         if (splitk > 1) {  // split-KV mode (lanes == 1): CTA c = part c % splitk of item c / splitk
@@ -201,7 +237,7 @@ __global__ void __launch_bounds__(1024) schedule_kernel(
                 // short items stay whole on rank 0 (written directly, no merge): the cluster merge
                 // costs about as much as streaming kMinSplitTiles tiles on one CTA
                 constexpr int kMinSplitTiles = 12;
-                const int s0 = item_start[u], len = item_start[u + 1] - s0;
+                const int s0 = start_of(u), len = start_of(u + 1) - s0;
                 if (len < kMinSplitTiles) {
                     t0 = r == 0 ? s0 : s0 + len;
                     t1 = s0 + len;
@@ -212,18 +248,18 @@ __global__ void __launch_bounds__(1024) schedule_kernel(
             }
             const int x0 = u < n_units ? u : n_items;
             cta_info[2 * c] = make_int4(t0, t1, x0, (int)T);
-            cta_info[2 * c + 1] = x0 < n_items ? item_info[x0] : make_int4(0, 0, 0, 0);
+            cta_info[2 * c + 1] = x0 < n_items ? info_of(x0) : make_int4(0, 0, 0, 0);
             continue;
         }
         if (one_per_cta) {
             // (at most one unit per group: units on groups 0 .. n_units-1, measured 7.4 -> 6.8 us at C1)
             const int u_lo = n_units <= NCv ? min(vc, n_units) : (int)((long long)vc * n_units / NCv);
             const int u_hi = n_units <= NCv ? min(vc + 1, n_units) : (int)((long long)(vc + 1) * n_units / NCv);
-            const int t0 = item_start[u_lo];
-            const int t1 = item_start[u_hi];
+            const int t0 = start_of(u_lo);
+            const int t1 = start_of(u_hi);
             const int x0 = u_lo < u_hi ? u_lo * lanes + cl : n_items;
             cta_info[2 * c] = make_int4(t0, t1, x0, (int)T);
-            cta_info[2 * c + 1] = x0 < n_items ? item_info[x0] : make_int4(0, 0, 0, 0);
+            cta_info[2 * c + 1] = x0 < n_items ? info_of(x0) : make_int4(0, 0, 0, 0);
             continue;
         }
         const int t0 = (int)((long long)vc * T / NCv);
@@ -231,12 +267,32 @@ __global__ void __launch_bounds__(1024) schedule_kernel(
         int lo2 = 0, hi2 = n_units;  // last unit with start <= t0
         while (hi2 - lo2 > 1) {
             const int mid = (lo2 + hi2) >> 1;
-            if (item_start[mid] <= t0) lo2 = mid; else hi2 = mid;
+            if (start_of(mid) <= t0) lo2 = mid; else hi2 = mid;
         }
         const int x0 = lo2 * lanes + cl;
         cta_info[2 * c] = make_int4(t0, t1, x0, (int)T);
-        cta_info[2 * c + 1] = x0 < n_items ? item_info[x0] : make_int4(0, 0, 0, 0);
+        cta_info[2 * c + 1] = x0 < n_items ? info_of(x0) : make_int4(0, 0, 0, 0);
     }
+}
+
+// Two launches per tree, no memset: one CTA per request validates it and builds its bitsets; then
+// one CTA builds the schedule and the status words from req_ok (the kernel boundary orders them).
+__global__ void __launch_bounds__(kPrepThreads) tree_validate_kernel(
+    const int32_t *__restrict__ parent, const int32_t *__restrict__ depth,
+    const int32_t *__restrict__ prefix_len, const int32_t *__restrict__ n_nodes, int Nmax, int max_depth,
+    int Smax, int G, int npc, int chunks, int32_t *__restrict__ status, int32_t *__restrict__ req_ok,
+    uint32_t *__restrict__ anc, uint32_t *__restrict__ desc, unsigned long long *__restrict__ rowmask) {
+    validate_bitsets(blockIdx.x, parent, depth, prefix_len, n_nodes, Nmax, max_depth, Smax, G, npc, chunks, status,
+                     req_ok, anc, desc, rowmask);
+}
+
+__global__ void __launch_bounds__(kPrepThreads) schedule_kernel(
+    const int32_t *__restrict__ prefix_len, const int32_t *__restrict__ n_nodes, const int32_t *req_ok, int B,
+    int Hkv, int chunks, int npc, int lanes, int32_t *__restrict__ item_start, uint32_t *__restrict__ item_cnt,
+    int4 *__restrict__ item_info, int4 *__restrict__ cta_info, int num_ctas, int splitk,
+    uint32_t *__restrict__ verify_cnt, int32_t *__restrict__ status, int no_split_slack) {
+    schedule(prefix_len, n_nodes, req_ok, B, Hkv, chunks, npc, lanes, item_start, item_cnt, item_info, cta_info,
+             num_ctas, splitk, verify_cnt, status, no_split_slack);
 }
 
 cudaError_t launch_tree_prepare(const specinfer_shape_t &s, const WsLayout &w,
@@ -244,21 +300,19 @@ cudaError_t launch_tree_prepare(const specinfer_shape_t &s, const WsLayout &w,
                                 const int32_t *prefix_len, const int32_t *n_nodes, char *ws,
                                 int num_ctas, cudaStream_t stream) {
     int32_t *status = reinterpret_cast<int32_t *>(ws + w.status);
-    cudaError_t e = cudaMemsetAsync(status, 0, 64 * 4, stream);
-    if (e != cudaSuccess) return e;
-    tree_validate_bitsets_kernel<<<s.batch, 256, 0, stream>>>(
+    int32_t *req_ok = reinterpret_cast<int32_t *>(ws + w.req_ok);
+    tree_validate_kernel<<<s.batch, kPrepThreads, 0, stream>>>(
         parent, depth, prefix_len, n_nodes, s.max_nodes, s.max_depth, s.max_seq,
-        s.num_q_heads / s.num_kv_heads, w.npc, w.chunks, status, reinterpret_cast<int32_t *>(ws + w.req_ok),
+        s.num_q_heads / s.num_kv_heads, w.npc, w.chunks, status, req_ok,
         reinterpret_cast<uint32_t *>(ws + w.anc), reinterpret_cast<uint32_t *>(ws + w.desc),
         reinterpret_cast<unsigned long long *>(ws + w.rowmask));
-    e = cudaGetLastError();
+    cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
-    schedule_kernel<<<1, 1024, 0, stream>>>(
-        prefix_len, n_nodes, reinterpret_cast<int32_t *>(ws + w.req_ok), s.batch,
-        s.num_kv_heads, w.chunks, w.npc, w.lanes, reinterpret_cast<int32_t *>(ws + w.item_start),
-        reinterpret_cast<uint32_t *>(ws + w.item_cnt), reinterpret_cast<int4 *>(ws + w.item_info),
-        reinterpret_cast<int4 *>(ws + w.cta_info), num_ctas, w.splitk, reinterpret_cast<uint32_t *>(ws + w.verify_cnt), status,
-        w.nt == kRowsBlock ? 24 : 8);
+    schedule_kernel<<<1, kPrepThreads, 0, stream>>>(
+        prefix_len, n_nodes, req_ok, s.batch, s.num_kv_heads, w.chunks, w.npc, w.lanes,
+        reinterpret_cast<int32_t *>(ws + w.item_start), reinterpret_cast<uint32_t *>(ws + w.item_cnt),
+        reinterpret_cast<int4 *>(ws + w.item_info), reinterpret_cast<int4 *>(ws + w.cta_info), num_ctas, w.splitk,
+        reinterpret_cast<uint32_t *>(ws + w.verify_cnt), status, w.nt == kRowsBlock ? 24 : 8);
     return cudaGetLastError();
 }
 

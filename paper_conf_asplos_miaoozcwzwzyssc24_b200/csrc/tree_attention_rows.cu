@@ -590,13 +590,22 @@ __global__ void __launch_bounds__(352, 1)
             const int llast = lt - 1;
             const int owner = llast & 1;
             const bool full = (sd.begin == sd.ib) && (sd.end == sd.ie);
-            // (two full barriers: the non-owner may not overwrite the hand-over slots of the next segment
-            // before the owner has read them, and it reads the final sum only after the owner wrote it)
+            // (two full barriers, executed by both groups at the same two instructions: the non-owner may
+            // not overwrite the hand-over slots of the next segment before the owner has read them, and
+            // it reads the final sum only after the owner wrote it)
             if (grp != owner) {
                 xl_l[r] = l;
                 xl_m[r] = m;
-                named_bar_sync(epi_bar, 64);
-                named_bar_sync(epi_bar, 64);
+            }
+            named_bar_sync(epi_bar, 64);
+            float lrow = 0.f;
+            if (grp == owner) {
+                const float lo_ = xl_l[r], mo = xl_m[r];
+                lrow = l + ((mo == -INFINITY || lo_ == 0.f) ? 0.f : lo_ * ex2(mo - m));
+                xl_f[r] = lrow;
+            }
+            named_bar_sync(epi_bar, 64);
+            if (grp != owner) {
                 if (full) {
                     const float inv = 1.0f / xl_f[r];
                     // O complete: this group last observed pv_done of ITS parity, so first wait for PV(llast - 1)
@@ -612,11 +621,6 @@ __global__ void __launch_bounds__(352, 1)
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&misc->o_free);
             } else {
-                named_bar_sync(epi_bar, 64);
-                const float lo_ = xl_l[r], mo = xl_m[r];
-                const float lrow = l + ((mo == -INFINITY || lo_ == 0.f) ? 0.f : lo_ * ex2(mo - m));
-                xl_f[r] = lrow;
-                named_bar_sync(epi_bar, 64);
                 mbar_wait(&misc->pv_done[llast & 1], (llast >> 1) & 1);   // O complete (in-order PVs)
                 tc_fence_after();
                 if (r == 0) SPI_TRACE(10);

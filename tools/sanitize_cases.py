@@ -126,7 +126,10 @@ CASES = {"c1": case_c1, "tiny": case_tiny, "splitkv": case_splitkv, "streamk": c
 if __name__ == "__main__":
     ap = argparse.ArgumentParser()
     ap.add_argument("--only", default=None, choices=sorted(CASES))
+    ap.add_argument("--lib", default=None, help="A/B: load another build of libspecinfer.so")
     a = ap.parse_args()
+    if a.lib:
+        spi.load_library(a.lib)
     for name, fn in CASES.items():
         if a.only is None or a.only == name:
             fn()
