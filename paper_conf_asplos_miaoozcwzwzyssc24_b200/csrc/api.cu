@@ -102,7 +102,15 @@ bool device_info(DeviceInfo *out) {
 // the split-KV cluster mode off: experiment flag 64)
 WsLayout layout(const specinfer_shape_t &s, int num_sms) {
 #ifdef SPECINFER_DEBUG_HOOKS
-    return ws_layout(s, num_sms, !(g_attn_debug_flags & 64));
+    WsLayout w = ws_layout(s, num_sms, !(g_attn_debug_flags & 64));
+    if (const char *gs = getenv("SPECINFER_DEBUG_GRID")) {   // experiment: persistent grid of N CTAs
+        const int g = atoi(gs);
+        if (g > 0 && g <= w.max_ctas && w.lanes == 1) {
+            w.splitk = 1;
+            w.grid = g;
+        }
+    }
+    return w;
 #else
     return ws_layout(s, num_sms);
 #endif

@@ -60,26 +60,34 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
         : "r"(taddr));
 }
 
-// The normalised bf16 output of one query row, dims [64 h, 64 h + 64) (TMEM columns of O), with
-// 16-byte stores; both TMEM loads are issued before the first wait.
-__device__ __forceinline__ void store_o_half(uint32_t o_col, float inv, bool row_valid, __nv_bfloat16 *orow, int h) {
+// The normalised bf16 output of one query row, dims [64 h, 64 h + 64) (TMEM columns of O): both
+// TMEM loads, one wait, the bf16 packing -- then the warp releases O (arrives on `o_free`: the next
+// segment's first PV may overwrite it) BEFORE its 16-byte global stores, which stay off the
+// critical path of the next segment.
+__device__ __forceinline__ void store_o_half(uint32_t o_col, float inv, bool row_valid, __nv_bfloat16 *orow, int h,
+                                             uint64_t *o_free) {
     uint32_t o[2][32];
     tmem_ld32(o_col + h * 64, o[0]);
     tmem_ld32(o_col + h * 64 + 32, o[1]);
     tmem_ld_wait();
-    if (!row_valid) return;
+    uint4 w[8];
 #pragma unroll
     for (int q = 0; q < 2; ++q) {
 #pragma unroll
         for (int i = 0; i < 32; i += 8) {
-            uint4 w;
-            w.x = pack_bf16x2(__uint_as_float(o[q][i]) * inv, __uint_as_float(o[q][i + 1]) * inv);
-            w.y = pack_bf16x2(__uint_as_float(o[q][i + 2]) * inv, __uint_as_float(o[q][i + 3]) * inv);
-            w.z = pack_bf16x2(__uint_as_float(o[q][i + 4]) * inv, __uint_as_float(o[q][i + 5]) * inv);
-            w.w = pack_bf16x2(__uint_as_float(o[q][i + 6]) * inv, __uint_as_float(o[q][i + 7]) * inv);
-            *reinterpret_cast<uint4 *>(orow + h * 64 + q * 32 + i) = w;
+            uint4 &x = w[q * 4 + i / 8];
+            x.x = pack_bf16x2(__uint_as_float(o[q][i]) * inv, __uint_as_float(o[q][i + 1]) * inv);
+            x.y = pack_bf16x2(__uint_as_float(o[q][i + 2]) * inv, __uint_as_float(o[q][i + 3]) * inv);
+            x.z = pack_bf16x2(__uint_as_float(o[q][i + 4]) * inv, __uint_as_float(o[q][i + 5]) * inv);
+            x.w = pack_bf16x2(__uint_as_float(o[q][i + 6]) * inv, __uint_as_float(o[q][i + 7]) * inv);
         }
     }
+    tc_fence_before();
+    __syncwarp();
+    if ((threadIdx.x & 31) == 0) mbar_arrive(o_free);
+    if (!row_valid) return;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) *reinterpret_cast<uint4 *>(orow + h * 64 + k * 8) = w[k];
 }
 
 // D[tmem] (+)= A[tmem] * B[smem desc], kind::f16 (A = P, bf16 packed two per column)
@@ -615,21 +623,21 @@ __global__ void __launch_bounds__(352, 1)
                     mbar_wait(&misc->pv_done[llast & 1], (llast >> 1) & 1);
                     tc_fence_after();
                     store_o_half(o_col, inv, row_valid,
-                                 p.out + (((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim, 1);
+                                 p.out + (((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim, 1,
+                                 &misc->o_free);
+                } else {
+                    tc_fence_before();
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(&misc->o_free);
                 }
-                tc_fence_before();
-                __syncwarp();
-                if (lane == 0) mbar_arrive(&misc->o_free);
             } else {
                 mbar_wait(&misc->pv_done[llast & 1], (llast >> 1) & 1);   // O complete (in-order PVs)
                 tc_fence_after();
                 if (r == 0) SPI_TRACE(10);
                 if (full) {
                     store_o_half(o_col, 1.0f / lrow, row_valid,
-                                 p.out + (((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim, 0);
-                    tc_fence_before();
-                    __syncwarp();
-                    if (lane == 0) mbar_arrive(&misc->o_free);   // the next segment's first PV may overwrite O
+                                 p.out + (((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim, 0,
+                                 &misc->o_free);
                 } else {
                     // a piece of a split item: unnormalised O row, (m, l) of the row, then the last piece
                     // merges every piece by log-sum-exp

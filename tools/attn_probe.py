@@ -29,6 +29,8 @@ def main():
     ap.add_argument("--expansion", default=None, help="override the tree: comma list <k1,..,km>")
     ap.add_argument("--lib", default=None, help="load this libspecinfer build instead (A/B experiments)")
     ap.add_argument("--flags", type=int, default=0, help="debug flags: 1 skip TMA, 2 skip MMA (timing only)")
+    ap.add_argument("--early", action="store_true", help="SPECINFER_ATTN_EARLY_PREFIX on every launch but the "
+                                                         "graph's first (as bench.py runs the layers)")
     a = ap.parse_args()
     if a.lib:
         spi.load_library(a.lib)
@@ -61,7 +63,7 @@ def main():
         with torch.cuda.graph(g, stream=s):
             for i in range(a.iters):
                 l = i % a.layers
-                st.attention(ai.q[l], ai.k_cache[l], ai.v_cache[l], out[l])
+                st.attention(ai.q[l], ai.k_cache[l], ai.v_cache[l], out[l], prefetch=a.early and i > 0)
     torch.cuda.synchronize()
     g.replay()
     torch.cuda.synchronize()
