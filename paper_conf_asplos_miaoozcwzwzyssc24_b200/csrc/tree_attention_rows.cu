@@ -86,8 +86,20 @@ __device__ __forceinline__ void store_o_half(uint32_t o_col, float inv, bool row
     __syncwarp();
     if ((threadIdx.x & 31) == 0) mbar_arrive(o_free);
     if (!row_valid) return;
+    __nv_bfloat16 *dst = orow + h * 64;
+    if ((reinterpret_cast<uintptr_t>(dst) & 31u) == 0) {
+        // 32-byte stores (one full L2 sector per thread and instruction): each warp instruction writes
+        // 32 different rows, so the store cost is per instruction -- half as many as 16-byte stores
 #pragma unroll
-    for (int k = 0; k < 8; ++k) *reinterpret_cast<uint4 *>(orow + h * 64 + k * 8) = w[k];
+        for (int k = 0; k < 4; ++k)
+            asm volatile("st.global.v8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"l"(dst + k * 16),
+                         "r"(w[2 * k].x), "r"(w[2 * k].y), "r"(w[2 * k].z), "r"(w[2 * k].w), "r"(w[2 * k + 1].x),
+                         "r"(w[2 * k + 1].y), "r"(w[2 * k + 1].z), "r"(w[2 * k + 1].w)
+                         : "memory");
+    } else {
+#pragma unroll
+        for (int k = 0; k < 8; ++k) *reinterpret_cast<uint4 *>(dst + k * 8) = w[k];
+    }
 }
 
 // D[tmem] (+)= A[tmem] * B[smem desc], kind::f16 (A = P, bf16 packed two per column)
@@ -649,10 +661,11 @@ __global__ void __launch_bounds__(352, 1)
                         tmem_ld32(o_col + q2 * 32, o);
                         tmem_ld_wait();
 #pragma unroll
-                        for (int i = 0; i < 32; i += 4)
-                            *reinterpret_cast<float4 *>(po + q2 * 32 + i) =
-                                make_float4(__uint_as_float(o[i]), __uint_as_float(o[i + 1]), __uint_as_float(o[i + 2]),
-                                            __uint_as_float(o[i + 3]));
+                        for (int i = 0; i < 32; i += 8)   // 32-byte stores (part_o rows are 512-byte aligned)
+                            asm volatile("st.global.v8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"l"(po + q2 * 32 + i),
+                                         "r"(o[i]), "r"(o[i + 1]), "r"(o[i + 2]), "r"(o[i + 3]), "r"(o[i + 4]),
+                                         "r"(o[i + 5]), "r"(o[i + 6]), "r"(o[i + 7])
+                                         : "memory");
                     }
                     tc_fence_before();
                     __syncwarp();
