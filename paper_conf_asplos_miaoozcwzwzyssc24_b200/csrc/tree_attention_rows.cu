@@ -471,6 +471,9 @@ __global__ void __launch_bounds__(352, 1)
             // ancestor-or-self bitset of this row's node, read on masked tiles only (rows without a
             // node use node 0's root path, which keeps them finite; they are never written)
             const uint32_t *anc = p.anc + ((size_t)b * p.Nmax + (row_valid ? node : 0)) * kBitWords;
+            // the masked (tree) tiles come last in a segment: pull the row's bitset into L1 now, so their
+            // __ldg's hit L1 instead of paying an L2 round trip on the softmax critical path
+            asm volatile("prefetch.global.L1 [%0];" ::"l"(anc));
             float m = -INFINITY, l = 0.f;      // latest known row reference (log2 units), this group's sum
             const int lt0 = lt;
             for (int t = sd.begin; t < sd.end; ++t, ++lt) {
