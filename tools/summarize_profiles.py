@@ -117,6 +117,8 @@ for k in ("verify_mss", "verify_greedy", "kv_commit", "tree_validate", "gather_w
     if not os.path.exists(p):
         continue
     rows = list(csv.reader(open(p)))
+    if not rows or "Metric Name" not in rows[0]:
+        continue   # (no launch of that kernel in the profiled run)
     h = rows[0]
     mi, vi, ui = h.index("Metric Name"), h.index("Metric Value"), h.index("Metric Unit")
     vals = {r[mi]: (r[vi], r[ui]) for r in rows[1:]}
