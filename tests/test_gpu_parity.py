@@ -211,6 +211,70 @@ def test_attention_invalid_tree_status():
     _check_rows(out, ref, tb, bs=[0])
 
 
+@pytest.mark.parametrize("name,batch", [("C2", 3), ("C3", 2), ("C1", 1)])
+def test_prepare_initialises_a_garbage_workspace(name, batch):
+    """tree_prepare needs no zeroed workspace (no memset since round 2): with every byte of the workspace
+    set to 0xFF first, prepare -> attention -> greedy verify -> MSS verify -> KV commit give bit-identical
+    results to a zero-filled workspace, twice in a row (counters re-armed by the calls themselves); a bad
+    tree's status bit is cleared by the next prepare of a good tree."""
+    cfg = W.CONFIGS[name]
+    tb = W.config_tree_batch(cfg, device=DEV, ragged=True, batch=batch)
+    smax = cfg.prefix + tb.max_nodes + 3
+    ai = W.make_attention_inputs(tb, 1, cfg.num_q_heads, cfg.num_kv_heads, smax, seed=11, device=DEV)
+    V = 4000
+    vg = W.make_verify_inputs(tb, V, seed=12, mode="greedy", device=DEV)
+    vm = W.make_verify_inputs(tb, V, seed=13, mode="mss", device=DEV)
+    shape = spi.make_shape(batch, tb.max_nodes, cfg.num_q_heads, cfg.num_kv_heads, smax, vocab=V,
+                           max_depth=tb.max_depth)
+    B, Lp = batch, tb.max_depth + 1
+
+    def run(fill):
+        ws = spi.alloc_workspace(shape, DEV)
+        ws.fill_(fill)
+        st = spi.TreeState.create(shape, tb.parent, tb.depth, tb.prefix_len, tb.n_nodes, workspace=ws)
+        res = []
+        for _ in range(2):
+            k, v, pl = ai.k_cache.clone(), ai.v_cache.clone(), tb.prefix_len.clone()
+            st.prefix_len = pl
+            st.prepare()
+            out = torch.full(ai.q.shape[1:], float("nan"), dtype=torch.bfloat16, device=DEV)
+            st.attention(ai.q[0], k[0], v[0], out)
+            outs = [out]
+            for mode, vi in (("greedy", vg), ("mss", vm)):
+                an = torch.empty((B, Lp), dtype=torch.int32, device=DEV)
+                at, na = torch.empty_like(an), torch.empty((B,), dtype=torch.int32, device=DEV)
+                if mode == "greedy":
+                    spi.specinfer_verify_greedy(shape, vi.logits, vi.tree_tokens, tb.parent, tb.n_nodes, an, at, na,
+                                                ws)
+                else:
+                    spi.specinfer_verify_mss(shape, vi.logits, vi.tree_tokens, tb.parent, tb.n_nodes, vi.draft_probs,
+                                             1.0, 5, 0, None, an, at, na, ws)
+                outs += [an, at, na]
+            spi.specinfer_kv_commit(shape, k, v, pl, outs[1], outs[3])
+            outs += [k, v, pl]
+            torch.cuda.synchronize()
+            assert spi.specinfer_read_device_status(ws) == 0
+            res.append([torch.nan_to_num(x.float(), nan=7.0).cpu() if x.is_floating_point() else x.cpu() for x in outs])
+        return ws, st, res
+
+    _, _, r0 = run(0)
+    ws, st, r1 = run(255)
+    for a_, b_ in ((r0[0], r1[0]), (r0[1], r1[1]), (r0[0], r0[1])):
+        for x, y in zip(a_, b_):
+            assert torch.equal(x, y)
+    # status: a bad tree sets the bit, the next good prepare clears it
+    bad = tb.parent.clone()
+    bad[0, min(2, int(tb.n_nodes[0]) - 1)] = 99
+    st.parent = bad
+    st.prepare()
+    torch.cuda.synchronize()
+    assert spi.specinfer_read_device_status(ws) & 1
+    st.parent = tb.parent
+    st.prepare()
+    torch.cuda.synchronize()
+    assert spi.specinfer_read_device_status(ws) == 0
+
+
 def test_host_validation_errors():
     tb = W.make_tree_batch([W.chain_tree(4)], [3], device=DEV)
     ai = W.make_attention_inputs(tb, 1, 2, 2, 16, seed=5, device=DEV)
