@@ -55,7 +55,6 @@ struct SmemMisc {
     uint64_t seg_full[kSegRing];
     SegDesc seg[kSegRing];
     uint32_t tmem_base;
-    int32_t flags[2][8];
     int32_t bcast;
     alignas(16) float m_thr[64];   // running row max + threshold (-inf: no key seen yet)
     alignas(16) float m_ref[64];   // running row max used as exp2 reference (0 if none yet)
@@ -417,14 +416,9 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
                     const float4 m4 = *reinterpret_cast<const float4 *>(&misc->m_thr[r0 + r]);
                     need |= (xv[r] > m4.x) | (xv[r + 1] > m4.y) | (xv[r + 2] > m4.z) | (xv[r + 3] > m4.w);
                 }
-                const unsigned ballot = __ballot_sync(0xffffffffu, need);
-                if (lane == 0) misc->flags[sb][half * 4 + qd] = ballot != 0u;
                 bulk_wait_read_all();  // output staging (P^T buffer) read by the bulk stores
-                named_bar_sync(1, kSoft);
-                int any_flag = 0;
-#pragma unroll
-                for (int f = 0; f < 4 * kSplit; ++f) any_flag |= misc->flags[sb][f];
-                const bool rescale = any_flag != 0;
+                // one barrier instruction both synchronises the softmax warps and ORs their verdicts
+                const bool rescale = named_bar_red_or(1, kSoft, need);
                 if (rescale) {
                     // exact tile max per row: transpose-reduce within the warp, combine 4 warps
 #pragma unroll

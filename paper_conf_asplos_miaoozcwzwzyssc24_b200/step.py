@@ -64,6 +64,8 @@ def make_layout(batch_global: int, world: int, rank: int, num_q_heads: int, num_
 class DeviceOps:
     """The library calls the step is made of (argument marshalling in __init__.py)."""
 
+    concurrent_verifiers = True   # independent verifiers may run on a side stream (own workspace regions)
+
     def __init__(self):
         import paper_conf_asplos_miaoozcwzwzyssc24_b200 as spi   # the binding (no CPU path)
         self.spi = spi
@@ -118,6 +120,7 @@ class VerifyStep:
         self.plan = D.GatherPlan(layout.batch_global, layout.world, path_len, device)
         self.p2p = p2p
         self.an_all = torch.zeros((layout.batch_global, path_len), **i32)
+        self.device, self._side = device, None
         self.na_all = torch.zeros((layout.batch_global,), **i32)
         self._layer = 0
 
@@ -138,9 +141,12 @@ class VerifyStep:
 
     # ---- a4 | a5 ----
     def verify(self, inputs: dict, seed: int, offset: int = 0, temperature: float = 1.0):
-        """inputs[mode] = (logits, tree_tokens, draft_probs or None) for this rank's requests."""
+        """inputs[mode] = (logits, tree_tokens, draft_probs or None) for this rank's requests.  With more than
+        one verifier, the ones whose result is not committed run on a side stream, concurrently with the
+        committed one (they use separate workspace counters / buffers); the caller's stream joins them."""
         parent, _, _, n_nodes = self.verify_tree
-        for m in self.modes:
+
+        def one(m):
             an, at, na = self.res[m]
             logits, tokens, draft = inputs[m]
             kw = {"gather": self.p2p.desc} if (self.p2p is not None and m == self.commit_mode) else {}
@@ -149,6 +155,21 @@ class VerifyStep:
             else:
                 self.ops.verify_mss(self.shape_verify, self.st_v, logits, tokens, parent, n_nodes, draft,
                                     temperature, seed, offset, self.rids, an, at, na, **kw)
+
+        others = [m for m in self.modes if m != self.commit_mode]
+        if others and getattr(self.ops, "concurrent_verifiers", False):
+            main = torch.cuda.current_stream(self.device)
+            if self._side is None:
+                self._side = torch.cuda.Stream(self.device)
+            self._side.wait_stream(main)
+            with torch.cuda.stream(self._side):
+                for m in others:
+                    one(m)
+            one(self.commit_mode)
+            main.wait_stream(self._side)
+        else:
+            for m in self.modes:
+                one(m)
 
     # ---- a7 ----
     def gather(self):
