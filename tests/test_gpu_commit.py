@@ -157,3 +157,80 @@ def test_kv_shard_layout_n1_commit():
     spi.specinfer_kv_commit(shape, k1, v1, P1, an_all, na_all)
     torch.cuda.synchronize()
     _check_commit(k, v, k1, v1, tb.prefix_len, P1, an, na, N)
+
+
+def test_verify_step_concurrent_verifiers_eager_and_graph():
+    """step.VerifyStep with both verifiers (C2's "greedy + MSS"): the MSS verifier runs on a side stream
+    concurrently with the committed greedy verifier.  Eager and inside a captured CUDA graph (as bench.py
+    replays it), every verifier's outputs equal the plain sequential C-ABI calls, and the committed cache
+    equals a commit of the greedy paths."""
+    from paper_conf_asplos_miaoozcwzwzyssc24_b200 import step as S
+    B, N, Hq, Hkv, P, V, L = 5, 21, 4, 4, 300, 3000, 2
+    p_, d_ = W.expansion_tree((1, 1, 3, 1, 1, 1, 1, 1))
+    tb = W.make_tree_batch([(p_, d_)] * B, list(W.ragged_prefix(P, B)), device=DEV, max_depth=8)
+    Lp = tb.max_depth + 1
+    smax = P + N + 3
+    ai = W.make_attention_inputs(tb, L, Hq, Hkv, smax, seed=21, device=DEV)
+    vi = {m: W.make_verify_inputs(tb, V, seed=22, mode=m, device=DEV) for m in ("greedy", "mss")}
+    layout = S.make_layout(B, 1, 0, Hq, Hkv, False)
+    shape = spi.make_shape(B, N, Hq, Hkv, smax, num_layers=L, vocab=V, max_depth=tb.max_depth)
+    tree = (tb.parent, tb.depth, tb.prefix_len, tb.n_nodes)
+    inputs = {m: (vi[m].logits, vi[m].tree_tokens, vi[m].draft_probs if m == "mss" else None) for m in vi}
+    rids = torch.arange(B, dtype=torch.int32, device=DEV)
+
+    # reference: the plain calls, one after the other
+    st = spi.TreeState.create(shape, *tree)
+    st.prepare()
+    ref = {}
+    for m in ("greedy", "mss"):
+        an = torch.empty((B, Lp), dtype=torch.int32, device=DEV)
+        at, na = torch.empty_like(an), torch.empty((B,), dtype=torch.int32, device=DEV)
+        if m == "greedy":
+            spi.specinfer_verify_greedy(shape, vi[m].logits, vi[m].tree_tokens, tb.parent, tb.n_nodes, an, at, na,
+                                        st.workspace)
+        else:
+            spi.specinfer_verify_mss(shape, vi[m].logits, vi[m].tree_tokens, tb.parent, tb.n_nodes, vi[m].draft_probs,
+                                     1.0, 7, 0, rids, an, at, na, st.workspace)
+        ref[m] = (na.clone(), at.clone(), an.clone())
+    k_ref, v_ref, p_ref = ai.k_cache.clone(), ai.v_cache.clone(), tb.prefix_len.clone()
+    spi.specinfer_kv_commit(shape, k_ref, v_ref, p_ref, ref["greedy"][2], ref["greedy"][0])
+    torch.cuda.synchronize()
+
+    p0 = tb.prefix_len.clone()
+    step = S.VerifyStep(S.DeviceOps(), layout, shape, shape, tree, tree, ("greedy", "mss"), Lp, DEV)
+    out = torch.empty_like(ai.q)
+    k, v = ai.k_cache.clone(), ai.v_cache.clone()
+
+    def one_step():
+        tb.prefix_len.copy_(p0)
+        step.prepare()
+        for l in range(L):
+            step.attention(ai.q[l], k[l], v[l], out[l], layer=l)
+        step.verify(inputs, seed=7, offset=0)
+        step.commit(k, v)
+
+    def check():
+        torch.cuda.synchronize()
+        for m in ("greedy", "mss"):
+            na, at, an = step.accepted(m)
+            for x, y in zip((na, at, an), ref[m]):
+                assert torch.equal(x, y), m
+        assert torch.equal(k, k_ref) and torch.equal(v, v_ref) and torch.equal(tb.prefix_len, p_ref)
+
+    s = torch.cuda.Stream()
+    s.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(s):
+        one_step()
+    check()
+    g = torch.cuda.CUDAGraph()
+    k.copy_(ai.k_cache), v.copy_(ai.v_cache)
+    with torch.cuda.graph(g, stream=s):
+        one_step()
+    for _ in range(2):
+        k.copy_(ai.k_cache), v.copy_(ai.v_cache)
+        for m in ("greedy", "mss"):
+            for t_ in step.res[m]:
+                t_.fill_(-5)
+        torch.cuda.synchronize()
+        g.replay()
+        check()
