@@ -432,64 +432,95 @@ def run_ours(args, ws, rank, local):
         h2d = h_q.numel() * 2 + sum(t.numel() * t.element_size() for t in h_list) + sum(t.numel() * 4 for t in h_tree)
         d2h = h_res_a.numel() * 4 + h_res_n.numel() * 4
 
-        # One CUDA graph per step: the H2D copies run on a copy stream (pinned memory, the copy
-        # engines) and each layer's attention waits only for its own q, so the PCIe transfer of
-        # layer l+1's q and of the logits / draft probabilities overlaps the attention of layer l.
+        # Pipelined steps (a serving loop's double buffering): the inputs live in two device sets; while
+        # step k computes on set k % 2, a copy stream (pinned memory, the copy engines) uploads step
+        # k + 1's inputs into the other set, and the step's graph joins that copy at its end.  Every
+        # step's inputs still cross PCIe inside the timed region: the first step's before the loop,
+        # step k + 1's during step k; the last step uploads nothing.  Each step ends with the D2H read
+        # of its result.
         copy_s = torch.cuda.Stream(device)
-        ev_fork, ev_tree, ev_lg = torch.cuda.Event(), torch.cuda.Event(), torch.cuda.Event()
-        ev_q = [torch.cuda.Event() for _ in range(L)]
+        ev_fork = torch.cuda.Event()
+        live_tree = tree_dev   # the tensors the step's TreeState / VerifyStep hold
+        sets = []
+        for _ in range(2):
+            sets.append({"q": torch.empty_like(wl.ai.q), "list": [torch.empty_like(t) for t in d_list],
+                         "tree": [torch.empty_like(t) for t in tree_dev]})
+        n_modes = len(wl.verify)
 
-        def e2e_step():
-            ev_fork.record(s)
-            copy_s.wait_event(ev_fork)
-            with torch.cuda.stream(copy_s):
-                for d, h in zip(tree_dev, h_tree):
-                    d.copy_(h, non_blocking=True)
-                ev_tree.record(copy_s)
-                for l in range(L):
-                    wl.ai.q[l].copy_(h_q[l], non_blocking=True)
-                    ev_q[l].record(copy_s)
-                for d, h in zip(d_list, h_list):
-                    d.copy_(h, non_blocking=True)
-                ev_lg.record(copy_s)
-            s.wait_event(ev_tree)
-            seg_prepare()
+        def set_inputs(st_):
+            lg = st_["list"][0]
+            dp = st_["list"][1] if "mss" in wl.verify else None
+            toks = st_["list"][len(st_["list"]) - n_modes:]
+            return {m: (lg, toks[i], dp if m == "mss" else None) for i, m in enumerate(wl.verify)}
+
+        def upload(st_):
+            for d, h in zip(st_["tree"], h_tree):
+                d.copy_(h, non_blocking=True)
+            st_["q"].copy_(h_q, non_blocking=True)
+            for d, h in zip(st_["list"], h_list):
+                d.copy_(h, non_blocking=True)
+
+        def body(st_):
+            for d, src in zip(live_tree, st_["tree"]):
+                d.copy_(src)
+            seg_prepare()   # (prefix_len reset from the uploaded committed lengths, then tree_prepare)
             for l in range(L):
-                s.wait_event(ev_q[l])
-                step.attention(wl.ai.q[l], wl.ai.k_cache[l], wl.ai.v_cache[l], out[l], layer=l if early else 0)
-            s.wait_event(ev_lg)
-            seg_verify()
+                step.attention(st_["q"][l], wl.ai.k_cache[l], wl.ai.v_cache[l], out[l], layer=l if early else 0)
+            step.verify(set_inputs(st_), seed=cfg.seed, offset=0)
+            if p2p is not None:
+                step.gather()
             gather_between()
             seg_commit()
             h_res_a.copy_(res_a, non_blocking=True)
             h_res_n.copy_(res_n, non_blocking=True)
 
+        def e2e_step(k, last):
+            cur, nxt = sets[k % 2], sets[(k + 1) % 2]
+            if not last:
+                ev_fork.record(s)
+                copy_s.wait_event(ev_fork)
+                with torch.cuda.stream(copy_s):
+                    upload(nxt)
+            body(cur)
+            if not last:
+                s.wait_stream(copy_s)
+
+        def prologue():
+            upload(sets[0])
+
         with torch.cuda.stream(s):
-            e2e_step()  # eager warm-up of the multi-stream step
+            prologue()
+            e2e_step(0, False)
+            e2e_step(1, True)   # eager warm-up of both sets and of the multi-stream step
         torch.cuda.synchronize(device)
-        g_e2e = None
+        graphs_e2e = None
         if ws == 1:
-            g_e2e = torch.cuda.CUDAGraph()
-            with torch.cuda.graph(g_e2e, stream=s):
-                e2e_step()
+            graphs_e2e = {}
+            for k in range(2):
+                for last in (False, True):
+                    g = torch.cuda.CUDAGraph()
+                    with torch.cuda.graph(g, stream=s):
+                        e2e_step(k, last)
+                    graphs_e2e[(k, last)] = g
             torch.cuda.synchronize(device)
 
-        def e2e_run():
-            if g_e2e is not None:
-                g_e2e.replay()
-            else:
-                e2e_step()
+        def e2e_run(nsteps):
+            prologue()
+            for k in range(nsteps):
+                last = k == nsteps - 1
+                if graphs_e2e is not None:
+                    graphs_e2e[(k % 2, last)].replay()
+                else:
+                    e2e_step(k % 2, last)
 
         with torch.cuda.stream(s):
-            for _ in range(max(1, args.warmup // 2)):
-                e2e_run()
+            e2e_run(max(2, args.warmup))
         torch.cuda.synchronize(device)
         barrier(ws)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         with torch.cuda.stream(s):
             e0.record(s)
-            for _ in range(K):
-                e2e_run()
+            e2e_run(K)
             e1.record(s)
         torch.cuda.synchronize(device)
         barrier(ws)
@@ -499,8 +530,9 @@ def run_ours(args, ws, rank, local):
                "ms_per_step": round(e2e_ms / K, 4),
                "inputs": "per step from pinned host memory: tree arrays, q of every layer, the LLM logits"
                          + (", draft probabilities" if "mss" in wl.verify else "")
-                         + ", each verifier's tree tokens; result read back: accepted tokens + counts; H2D on a copy "
-                           "stream overlapping the attention of earlier layers"}
+                         + ", each verifier's tree tokens; result read back: accepted tokens + counts; two device "
+                           "input sets: step k+1's H2D on a copy stream during step k (the first step's before the "
+                           "loop, inside the timed region)"}
 
     cpu = None
     if rank == 0 and ws == 1 and not args.no_cpu:
