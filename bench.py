@@ -280,6 +280,17 @@ def run_ours(args, ws, rank, local):
     def seg_commit():
         step.commit(wl.ai.k_cache, wl.ai.v_cache)
 
+    # verify and commit in one graph unless an eager (NCCL) gather sits between them: the commit needs
+    # only the committed verifier, so it overlaps the other verifier running on the side stream
+    eager_gather = p2p is None and need_gather
+
+    def seg_verify_commit():
+        step.verify(inputs, seed=cfg.seed, offset=0, join=False)
+        if p2p is not None:
+            step.gather()
+        step.commit(wl.ai.k_cache, wl.ai.v_cache)
+        step.join()
+
     launches_per_step = (spi.specinfer_launches_per_call("tree_prepare") * (2 if kv_shard else 1) +
                          L * spi.specinfer_launches_per_call("tree_attention") +
                          ("greedy" in wl.verify) * spi.specinfer_launches_per_call("verify_greedy") +
@@ -295,7 +306,9 @@ def run_ours(args, ws, rank, local):
             seg_prepare(); seg_attention(); seg_verify(); gather_between(); seg_commit()
     torch.cuda.synchronize(device)
     graphs = []
-    for fn in (seg_prepare, seg_attention, seg_verify, seg_commit):
+    segs = (seg_prepare, seg_attention, seg_verify, seg_commit) if eager_gather else \
+        (seg_prepare, seg_attention, seg_verify_commit)
+    for fn in segs:
         g = torch.cuda.CUDAGraph()
         with torch.cuda.graph(g, stream=s):
             fn()
@@ -304,7 +317,9 @@ def run_ours(args, ws, rank, local):
 
     with torch.cuda.stream(s):
         for _ in range(args.warmup):
-            graphs[0].replay(); graphs[1].replay(); graphs[2].replay(); gather_between(); graphs[3].replay()
+            graphs[0].replay(); graphs[1].replay(); graphs[2].replay()
+            if eager_gather:
+                gather_between(); graphs[3].replay()
     torch.cuda.synchronize(device)
     K = args.steps
     ev = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(K)]
@@ -324,8 +339,9 @@ def run_ours(args, ws, rank, local):
             graphs[1].replay()
             ev[k][2].record(s)
             graphs[2].replay()
-            gather_between()
-            graphs[3].replay()
+            if eager_gather:
+                gather_between()
+                graphs[3].replay()
         e_all[1].record(s)
     torch.cuda.synchronize(device)
     barrier(ws)
@@ -466,11 +482,12 @@ def run_ours(args, ws, rank, local):
             seg_prepare()   # (prefix_len reset from the uploaded committed lengths, then tree_prepare)
             for l in range(L):
                 step.attention(st_["q"][l], wl.ai.k_cache[l], wl.ai.v_cache[l], out[l], layer=l if early else 0)
-            step.verify(set_inputs(st_), seed=cfg.seed, offset=0)
+            step.verify(set_inputs(st_), seed=cfg.seed, offset=0, join=False)
             if p2p is not None:
                 step.gather()
             gather_between()
             seg_commit()
+            step.join()
             h_res_a.copy_(res_a, non_blocking=True)
             h_res_n.copy_(res_n, non_blocking=True)
 
@@ -555,7 +572,8 @@ def run_ours(args, ws, rank, local):
                                    else f"request-sharded x{ws}") if ws > 1 else "single GPU",
                    "l2": "no flush: every step streams this GPU's KV cache "
                          f"({2 * L * layout.attn_cnt * wl.Hkv * wl.smax * 256 / 1e9:.1f} GB) >> 126 MB L2",
-                   "graph": "4 CUDA graphs per step (prepare | L x attention | verify | commit)",
+                   "graph": ("4 CUDA graphs per step (prepare | L x attention | verify | commit)" if eager_gather else
+                             "3 CUDA graphs per step (prepare | L x attention | verify + gather + commit)"),
                    "gather": gather_note,
                    "host_binding": (f"pinned buffers allocated under the GPU-local CPU set ({bound_cpus} "
                                     "CPUs, sysfs local_cpulist)" if affinity_before else "unbound"),

@@ -120,7 +120,7 @@ class VerifyStep:
         self.plan = D.GatherPlan(layout.batch_global, layout.world, path_len, device)
         self.p2p = p2p
         self.an_all = torch.zeros((layout.batch_global, path_len), **i32)
-        self.device, self._side = device, None
+        self.device, self._side, self._pending = device, None, False
         self.na_all = torch.zeros((layout.batch_global,), **i32)
         self._layer = 0
 
@@ -140,10 +140,12 @@ class VerifyStep:
         self._layer += 1
 
     # ---- a4 | a5 ----
-    def verify(self, inputs: dict, seed: int, offset: int = 0, temperature: float = 1.0):
+    def verify(self, inputs: dict, seed: int, offset: int = 0, temperature: float = 1.0, join: bool = True):
         """inputs[mode] = (logits, tree_tokens, draft_probs or None) for this rank's requests.  With more than
         one verifier, the ones whose result is not committed run on a side stream, concurrently with the
-        committed one (they use separate workspace counters / buffers); the caller's stream joins them."""
+        committed one (they use separate workspace counters / buffers); the caller's stream joins them now,
+        or, with join=False, at join() -- so that gather / commit (which need only the committed verifier)
+        overlap them too."""
         parent, _, _, n_nodes = self.verify_tree
 
         def one(m):
@@ -166,10 +168,18 @@ class VerifyStep:
                 for m in others:
                     one(m)
             one(self.commit_mode)
-            main.wait_stream(self._side)
+            self._pending = True
+            if join:
+                self.join()
         else:
             for m in self.modes:
                 one(m)
+
+    def join(self):
+        """The caller's stream waits for the verifiers still running on the side stream."""
+        if self._pending:
+            torch.cuda.current_stream(self.device).wait_stream(self._side)
+            self._pending = False
 
     # ---- a7 ----
     def gather(self):

@@ -159,7 +159,8 @@ def test_kv_shard_layout_n1_commit():
     _check_commit(k, v, k1, v1, tb.prefix_len, P1, an, na, N)
 
 
-def test_verify_step_concurrent_verifiers_eager_and_graph():
+@pytest.mark.parametrize("join_early", [True, False])
+def test_verify_step_concurrent_verifiers_eager_and_graph(join_early):
     """step.VerifyStep with both verifiers (C2's "greedy + MSS"): the MSS verifier runs on a side stream
     concurrently with the committed greedy verifier.  Eager and inside a captured CUDA graph (as bench.py
     replays it), every verifier's outputs equal the plain sequential C-ABI calls, and the committed cache
@@ -206,8 +207,9 @@ def test_verify_step_concurrent_verifiers_eager_and_graph():
         step.prepare()
         for l in range(L):
             step.attention(ai.q[l], k[l], v[l], out[l], layer=l)
-        step.verify(inputs, seed=7, offset=0)
-        step.commit(k, v)
+        step.verify(inputs, seed=7, offset=0, join=join_early)
+        step.commit(k, v)     # (join_early False: the commit overlaps the side-stream MSS, as bench.py runs it)
+        step.join()
 
     def check():
         torch.cuda.synchronize()
