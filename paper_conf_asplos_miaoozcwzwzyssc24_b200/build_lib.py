@@ -34,10 +34,11 @@ def _stale(lib=LIB) -> bool:
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def build(force: bool = False, verbose: bool = False, extra=(), debug_hooks: bool = False) -> str:
+def build(force: bool = False, verbose: bool = False, extra=(), debug_hooks: bool = False, out=None) -> str:
     """Compiles every csrc/*.cu for sm_100a and links libspecinfer.so; with debug_hooks, the
-    development variant libspecinfer_debug.so (pipeline traces, experiment switches)."""
-    target = DEBUG_LIB if debug_hooks else LIB
+    development variant libspecinfer_debug.so (pipeline traces, experiment switches); with `out`,
+    an A/B variant at that path (development tools: `extra` holds its -D switches)."""
+    target = out or (DEBUG_LIB if debug_hooks else LIB)
     if debug_hooks:
         extra = tuple(extra) + ("-DSPECINFER_DEBUG_HOOKS",)
     if not force and not _stale(target):
@@ -71,5 +72,8 @@ def build(force: bool = False, verbose: bool = False, extra=(), debug_hooks: boo
 
 
 if __name__ == "__main__":
-    print(build(force="--force" in sys.argv, verbose="--verbose" in sys.argv,
-                debug_hooks="--debug-hooks" in sys.argv))
+    # python -m ...build_lib [--force] [--verbose] [--debug-hooks] [--out PATH -DNAME ...]
+    out = sys.argv[sys.argv.index("--out") + 1] if "--out" in sys.argv else None
+    print(build(force="--force" in sys.argv or out is not None, verbose="--verbose" in sys.argv,
+                debug_hooks="--debug-hooks" in sys.argv, out=out,
+                extra=tuple(a for a in sys.argv[1:] if a.startswith("-D"))))

@@ -88,16 +88,33 @@ __device__ __forceinline__ int kv_tile_row(const AttnParams &p, int b, int g, in
     return (page * p.Hkv + g) * kKeyTile;
 }
 
+// 64-bit unsigned division by shift-subtract, inline: the emulated `/` on 64-bit integers is a called
+// subroutine, and a call site in a kernel that reallocates registers per warpgroup (setmaxnreg) makes
+// ptxas compile the whole kernel under the smallest register budget.  Cold path only.
+__device__ __forceinline__ unsigned long long udiv64_inline(unsigned long long n, unsigned long long d) {
+    unsigned long long q = 0, r = 0;
+#pragma unroll 1
+    for (int i = 63; i >= 0; --i) {
+        r = (r << 1) | ((n >> i) & 1ull);
+        if (r >= d) {
+            r -= d;
+            q |= 1ull << i;
+        }
+    }
+    return q;
+}
+
 __device__ __forceinline__ int cta_start(long long c, long long T, long long NC) {
-    // 32-bit division when c * T fits (every practical schedule); 64-bit division is emulated
+    // 32-bit division when c * T fits (every practical schedule)
     if (c * T <= 0xFFFFFFFFll) return (int)((uint32_t)(c * T) / (uint32_t)NC);
-    return (int)((c * T) / NC);
+    return (int)udiv64_inline((unsigned long long)(c * T), (unsigned long long)NC);
 }
 
 __device__ __forceinline__ int cta_of_tile(int t, int T, int NC) {
     // the largest c with cta_start(c) <= t: floor(c T / NC) <= t <=> c T < (t + 1) NC
     const long long num = (long long)(t + 1) * NC - 1;
-    int c = num <= 0xFFFFFFFFll ? (int)((uint32_t)num / (uint32_t)T) : (int)(num / T);
+    int c = num <= 0xFFFFFFFFll ? (int)((uint32_t)num / (uint32_t)T)
+                                : (int)udiv64_inline((unsigned long long)num, (unsigned long long)T);
     return c < NC ? c : NC - 1;
 }
 

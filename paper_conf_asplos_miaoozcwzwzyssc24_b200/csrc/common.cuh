@@ -152,11 +152,10 @@ __device__ __forceinline__ bool mbar_try_wait(uint64_t *bar, uint32_t parity) {
 #ifndef SPECINFER_WATCHDOG_CYCLES
 #define SPECINFER_WATCHDOG_CYCLES 40000000000ll
 #endif
-static __device__ __noinline__ void mbar_hang_report(uint64_t *bar, uint32_t parity) {
-    printf("specinfer: mbarrier wait timeout block %d thread %d bar smem 0x%x parity %u\n", blockIdx.x,
-           threadIdx.x, smem_u32(bar), parity);
-    __trap();
-}
+// A wait that never completes is a protocol bug: trap (the launch fails with an error instead of hanging
+// the GPU).  Inline on purpose -- no printf: a called subroutine in a kernel that reallocates registers
+// per warpgroup (setmaxnreg) makes ptxas compile the whole kernel under the smallest register budget.
+__device__ __forceinline__ void mbar_hang_report(uint64_t *, uint32_t) { __trap(); }
 __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
     if (mbar_try_wait(bar, parity)) return;
     const long long t0 = clock64();
@@ -351,6 +350,16 @@ __host__ __device__ constexpr uint32_t make_idesc_bf16(int M, int N, bool a_mn_m
 }
 
 // ---- misc ---------------------------------------------------------------------------------
+// warpgroup register reallocation (all 128 threads of an aligned warpgroup execute it)
+template <int N>
+__device__ __forceinline__ void setmaxnreg_inc() {
+    asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(N));
+}
+template <int N>
+__device__ __forceinline__ void setmaxnreg_dec() {
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(N));
+}
+
 __device__ __forceinline__ float ex2(float x) {
     float y;
     asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));

@@ -31,6 +31,12 @@ constexpr int RB = kRowsBlock;              // 128 query rows per item
 constexpr int kQBuf = 2 * RB * 128;          // one Q buffer: 2 halves x 128 rows x 128 B
 constexpr int kTmemCols = 512;
 constexpr int kColS = 0, kColO = 256, kColP = 384;
+// warp roles: 0-7 softmax / epilogue (two groups of 4, warp & 3 = TMEM lane quarter), 8 TMA producers,
+// 9 S issuer (+ TMEM allocation), 10 PV issuer, 11 idle.  The control warpgroup (8-11) gives registers
+// to the softmax warpgroups (setmaxnreg): 168 per thread at launch -> 56 / 224
+constexpr int kThreads = 384;
+constexpr int kWarpProd = 8, kWarpS = 9, kWarpPV = 10;
+constexpr int kRegsCtl = 56, kRegsSoftmax = 224;
 constexpr int kMaxK = 4, kMaxV = 4;          // ring slots (the launch picks 3 K + 2 V)
 
 struct Misc {
@@ -176,7 +182,7 @@ __device__ __forceinline__ void mask32(uint32_t (&v)[32], uint32_t vis) {
 
 }  // namespace rows
 
-__global__ void __launch_bounds__(352, 1)
+__global__ void __maxnreg__(168)
     tree_attn_rows_kernel(const __grid_constant__ CUtensorMap tm_q, const __grid_constant__ CUtensorMap tm_k,
                           const __grid_constant__ CUtensorMap tm_v, const __grid_constant__ CUtensorMap tm_k16,
                           const __grid_constant__ CUtensorMap tm_v16, const __grid_constant__ CUtensorMap tm_k4,
@@ -221,21 +227,21 @@ __global__ void __launch_bounds__(352, 1)
         for (int i = 0; i < kSegRing; ++i) mbar_init(&misc->seg_full[i], 1);
         fence_barrier_init();
     }
-    if (warp == 0 && lane == 0) {
+    if (warp == kWarpProd && lane == 0) {
         tma_prefetch_desc(&tm_q);
         tma_prefetch_desc(&tm_k);
         tma_prefetch_desc(&tm_v);
     }
-    if (warp >= 3) {
+    if (warp < 8) {
         // Q rows beyond an item's G*npc rows are never written by TMA: keep them zero
-        for (int i = threadIdx.x - 96; i < 2 * kQBuf / 16; i += 256)
+        for (int i = threadIdx.x; i < 2 * kQBuf / 16; i += 256)
             reinterpret_cast<uint4 *>(s_q)[i] = make_uint4(0, 0, 0, 0);
         // rows past a request's last key are never loaded: slots must hold finite data (0 * NaN)
-        for (int i = threadIdx.x - 96; i < (NK + NV) * kSlotBytes / 16; i += 256)
+        for (int i = threadIdx.x; i < (NK + NV) * kSlotBytes / 16; i += 256)
             reinterpret_cast<uint4 *>(s_k)[i] = make_uint4(0, 0, 0, 0);
         fence_proxy_async_smem();
     }
-    if (warp == 1) tmem_alloc<kTmemCols>(&misc->tmem_base);
+    if (warp == kWarpS) tmem_alloc<kTmemCols>(&misc->tmem_base);
     tc_fence_before();
     __syncthreads();
     tc_fence_after();
@@ -243,614 +249,616 @@ __global__ void __launch_bounds__(352, 1)
 
     // Programmatic dependent launch (see tree_attention.cu): the producer warp may stage
     // committed-prefix tiles of its first segment before the dependency resolves (early_prefix)
-    const bool early = p.early_prefix != 0 && warp == 0;
+    const bool early = p.early_prefix != 0 && warp == kWarpProd;
     if (!early) grid_dependency_wait();
     const int4 ci = __ldg(p.cta_info + 2 * blockIdx.x);
     const int4 first_info = __ldg(p.cta_info + 2 * blockIdx.x + 1);
     const int t0 = ci.x, t1 = ci.y, x_first = ci.z, T = ci.w;
     const int ntiles = t1 - t0;
 
-    if (ntiles <= 0) {
-        if (early) grid_dependency_wait();
-    } else if (warp == 0) {
-        // ============================ TMA producers ============================
-        // lane 0: segment descriptors, Q and the K ring; lane 1: the V ring (follows the descriptors)
-        const uint64_t pol = p.lanes > 1 ? l2_evict_normal_policy() : l2_evict_first_policy();
-        auto issue = [&](const SegDesc &d, int t, int lt, bool is_v) {
-            const int key0 = (t - d.ib) * kKeyTile;
-            const int nv = min(kKeyTile, d.P + d.n - key0);
-            const int row0 = kv_tile_row(p, d.b, d.g, key0);
-            const int NS = is_v ? NV : NK;
-            const int slot = lt % NS, f = lt / NS;
-            if (f >= 1) mbar_wait(is_v ? &misc->v_empty[slot] : &misc->k_empty[slot], (f - 1) & 1);
-            if (!is_v) {
-                SPI_TRACE(0);
-                if (lt == 0) SPI_TRACE_K(2);
-            } else {
-                SPI_TRACE(1);
-            }
-            uint8_t *dst = (is_v ? s_v : s_k) + (size_t)slot * kSlotBytes;
-            uint64_t *bar = is_v ? &misc->v_full[slot] : &misc->k_full[slot];
-            const CUtensorMap *m = is_v ? &tm_v : &tm_k;
-            if (SPI_FLAGS(p) & 1) {  // experiment: no K/V traffic (results invalid)
-                mbar_arrive(bar);
-            } else if (nv == kKeyTile) {
-                mbar_arrive_expect_tx(bar, kSlotBytes);
-                tma_load_2d(dst, m, bar, 0, row0, pol);
-                tma_load_2d(dst + kHalfBytes, m, bar, 64, row0, pol);
-            } else if (is_v) {
-                tma_load_rows(dst, bar, nv, row0, pol, &tm_v16, &tm_v4, &tm_v1);
-            } else {
-                tma_load_rows(dst, bar, nv, row0, pol, &tm_k16, &tm_k4, &tm_k1);
-            }
-        };
-        auto n_early = [&](const SegDesc &d, int NS) {
-            int c = 0;
-            while (c < NS && d.begin + c < d.end && (d.begin + c - d.ib + 1) * kKeyTile <= d.P) ++c;
-            return c;
-        };
-        if (lane == 0) {
-            int x = x_first, ls = 0, lt = 0;
-            int4 next_info = first_info;
-            for (;;) {
-                // next non-empty segment of this CTA's range (terminal descriptor if none)
-                SegDesc d{};
-                d.x = -1;
-                for (;; x += p.lanes) {
-                    const int4 info = next_info;
-                    if (info.x >= t1) break;  // (the sentinel item_info[n_items] starts at T)
-                    next_info = __ldg(p.item_info + min(x + p.lanes, p.n_items));
-                    const int begin = max(t0, info.x), end = min(t1, info.y);
-                    if (end <= begin || info.w == 0) continue;  // no tiles here / empty chunk of the unit
-                    d.x = x;
-                    d.begin = begin;
-                    d.end = end;
-                    d.ib = info.x;
-                    d.ie = info.y;
-                    d.c = x % p.chunks;
-                    d.g = (x / p.chunks) % p.Hkv;
-                    d.b = x / (p.chunks * p.Hkv);
-                    d.P = info.z;
-                    d.n = info.w;
-                    x += p.lanes;
-                    break;
+    if (warp >= 8) {
+        // control warpgroup: its registers go to the softmax warps (all 4 warps execute this one
+        // instruction; no code path below rejoins the softmax path)
+        setmaxnreg_dec<kRegsCtl>();
+        if (ntiles <= 0) {
+            if (early) grid_dependency_wait();
+        } else if (warp == kWarpProd) {
+            // ============================ TMA producers ============================
+            // lane 0: segment descriptors, Q and the K ring; lane 1: the V ring (follows the descriptors)
+            const uint64_t pol = p.lanes > 1 ? l2_evict_normal_policy() : l2_evict_first_policy();
+            auto issue = [&](const SegDesc &d, int t, int lt, bool is_v) {
+                const int key0 = (t - d.ib) * kKeyTile;
+                const int nv = min(kKeyTile, d.P + d.n - key0);
+                const int row0 = kv_tile_row(p, d.b, d.g, key0);
+                const int NS = is_v ? NV : NK;
+                const int slot = lt % NS, f = lt / NS;
+                if (f >= 1) mbar_wait(is_v ? &misc->v_empty[slot] : &misc->k_empty[slot], (f - 1) & 1);
+                if (!is_v) {
+                    SPI_TRACE(0);
+                    if (lt == 0) SPI_TRACE_K(2);
+                } else {
+                    SPI_TRACE(1);
                 }
-                misc->seg[ls % kSegRing] = d;
-                mbar_arrive(&misc->seg_full[ls % kSegRing]);
-                if (d.x < 0) {
-                    if (early && ls == 0) grid_dependency_wait();
-                    break;
+                uint8_t *dst = (is_v ? s_v : s_k) + (size_t)slot * kSlotBytes;
+                uint64_t *bar = is_v ? &misc->v_full[slot] : &misc->k_full[slot];
+                const CUtensorMap *m = is_v ? &tm_v : &tm_k;
+                if (SPI_FLAGS(p) & 1) {  // experiment: no K/V traffic (results invalid)
+                    mbar_arrive(bar);
+                } else if (nv == kKeyTile) {
+                    mbar_arrive_expect_tx(bar, kSlotBytes);
+                    tma_load_2d(dst, m, bar, 0, row0, pol);
+                    tma_load_2d(dst + kHalfBytes, m, bar, 64, row0, pol);
+                } else if (is_v) {
+                    tma_load_rows(dst, bar, nv, row0, pol, &tm_v16, &tm_v4, &tm_v1);
+                } else {
+                    tma_load_rows(dst, bar, nv, row0, pol, &tm_k16, &tm_k4, &tm_k1);
                 }
-                int pre = 0;
-                if (early && ls == 0) {
-                    pre = n_early(d, NK);
-                    for (int i = 0; i < pre; ++i) issue(d, d.begin + i, i, false);
-                    grid_dependency_wait();
-                }
-                const int qb = ls & 1;
-                if (ls >= 2) mbar_wait(&misc->q_empty[qb], ((ls >> 1) - 1) & 1);
-                mbar_arrive_expect_tx(&misc->q_full[qb], 2u * (uint32_t)(p.G * p.npc) * 128u);
-                uint8_t *qdst = s_q + qb * kQBuf;
-                const int node0 = d.b * p.Nmax + d.c * p.npc;
-                tma_load_3d(qdst, &tm_q, &misc->q_full[qb], 0, d.g * p.G, node0);
-                tma_load_3d(qdst + RB * 128, &tm_q, &misc->q_full[qb], 64, d.g * p.G, node0);
-                lt += pre;
-                for (int t = d.begin + pre; t < d.end; ++t, ++lt) issue(d, t, lt, false);
-                ++ls;
-            }
-            grid_launch_dependents();
-        } else if (lane == 1) {
-            int ls = 0, lt = 0;
-            for (;;) {
-                mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
-                const SegDesc d = misc->seg[ls % kSegRing];
-                if (d.x < 0) {
-                    if (early && ls == 0) grid_dependency_wait();
-                    break;
-                }
-                int pre = 0;
-                if (early && ls == 0) {
-                    pre = n_early(d, NV);
-                    for (int i = 0; i < pre; ++i) issue(d, d.begin + i, i, true);
-                    grid_dependency_wait();
-                }
-                lt += pre;
-                for (int t = d.begin + pre; t < d.end; ++t, ++lt) issue(d, t, lt, true);
-                ++ls;
-            }
-        }
-    } else if (warp == 1) {
-        // ===================== S issuer: S(t) = Q K(t)^T into S buffer t & 1 =====================
-        // (the buffer is free once the softmax of tile t - 2 has loaded it: s_free)
-        if (lane == 0) {
-            const uint32_t idesc_s = make_idesc_bf16(128, 128, false, false);
-            const uint32_t k_addr = smem_u32(s_k), q_addr = smem_u32(s_q);
-            int lt = 0, ls = 0;
-            for (;;) {
-                mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
-                const SegDesc d = misc->seg[ls % kSegRing];
-                if (d.x < 0) break;
-                const int qb = ls & 1;
-                mbar_wait(&misc->q_full[qb], (ls >> 1) & 1);
-                for (int t = d.begin; t < d.end; ++t, ++lt) {
-                    const int sb = lt & 1;
-                    if (lt >= 2) mbar_wait(&misc->s_free[sb], ((lt - 2) >> 1) & 1);
-                    const int slot = lt % NK;
-                    mbar_wait(&misc->k_full[slot], (lt / NK) & 1);
-                    tc_fence_after();
-                    SPI_TRACE(2);
-                    const uint32_t kbase = k_addr + slot * kSlotBytes;
-                    const uint32_t qbase = q_addr + qb * kQBuf;
-#pragma unroll
-                    for (int kk = 0; kk < kHeadDim / 16; ++kk) {
-                        const uint32_t off = (kk >> 2) * (RB * 128) + (kk & 3) * 32;
-                        const uint64_t adesc = make_smem_desc(qbase + off, 16, 1024, kSw128);
-                        const uint64_t bdesc = make_smem_desc(kbase + (kk >> 2) * kHalfBytes + (kk & 3) * 32, 16,
-                                                              1024, kSw128);
-                        if (!(SPI_FLAGS(p) & 2))
-                            umma_bf16_ss(tmem + kColS + sb * 128, adesc, bdesc, idesc_s, kk > 0 ? 1u : 0u);
+            };
+            auto n_early = [&](const SegDesc &d, int NS) {
+                int c = 0;
+                while (c < NS && d.begin + c < d.end && (d.begin + c - d.ib + 1) * kKeyTile <= d.P) ++c;
+                return c;
+            };
+            if (lane == 0) {
+                int x = x_first, ls = 0, lt = 0;
+                int4 next_info = first_info;
+                for (;;) {
+                    // next non-empty segment of this CTA's range (terminal descriptor if none)
+                    SegDesc d{};
+                    d.x = -1;
+                    for (;; x += p.lanes) {
+                        const int4 info = next_info;
+                        if (info.x >= t1) break;  // (the sentinel item_info[n_items] starts at T)
+                        next_info = __ldg(p.item_info + min(x + p.lanes, p.n_items));
+                        const int begin = max(t0, info.x), end = min(t1, info.y);
+                        if (end <= begin || info.w == 0) continue;  // no tiles here / empty chunk of the unit
+                        d.x = x;
+                        d.begin = begin;
+                        d.end = end;
+                        d.ib = info.x;
+                        d.ie = info.y;
+                        d.c = x % p.chunks;
+                        d.g = (x / p.chunks) % p.Hkv;
+                        d.b = x / (p.chunks * p.Hkv);
+                        d.P = info.z;
+                        d.n = info.w;
+                        x += p.lanes;
+                        break;
                     }
-                    umma_commit(&misc->s_full[sb]);
-                    umma_commit(&misc->k_empty[slot]);
-                    if (t == d.end - 1) umma_commit(&misc->q_empty[qb]);
-                }
-                ++ls;
-            }
-        }
-    } else if (warp == 2) {
-        // ============ PV issuer: O += P(t) V(t) (A = P from TMEM, N = 128 dims), in tile order ============
-        if (lane == 0) {
-            const uint32_t idesc_o = make_idesc_bf16(128, 128, false, true);
-            const uint32_t v_addr = smem_u32(s_v);
-            int lt = 0, ls = 0;
-            for (;;) {
-                mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
-                const SegDesc d = misc->seg[ls % kSegRing];
-                if (d.x < 0) break;
-                for (int t = d.begin; t < d.end; ++t, ++lt) {
-                    const int pb = lt & 1;
-                    mbar_wait(&misc->p_full[pb], (lt >> 1) & 1);
-                    const bool first = (t == d.begin);
-                    if (first && ls > 0) mbar_wait(&misc->o_free, (ls - 1) & 1);  // previous segment's O read
-                    const int slot = lt % NV;
-                    mbar_wait(&misc->v_full[slot], (lt / NV) & 1);
-                    tc_fence_after();
-                    SPI_TRACE(3);
-                    const uint32_t vbase = v_addr + slot * kSlotBytes;
-#pragma unroll
-                    for (int kk = 0; kk < kKeyTile / 16; ++kk) {
-                        const uint64_t bdesc = make_smem_desc(vbase + kk * 16 * 128, kHalfBytes, 1024, kSw128);
-                        if (!(SPI_FLAGS(p) & 2))
-                            umma_bf16_ts(tmem + kColO, tmem + kColP + pb * 64 + kk * 8, bdesc, idesc_o,
-                                         (first && kk == 0) ? 0u : 1u);
+                    misc->seg[ls % kSegRing] = d;
+                    mbar_arrive(&misc->seg_full[ls % kSegRing]);
+                    if (d.x < 0) {
+                        if (early && ls == 0) grid_dependency_wait();
+                        break;
                     }
-                    umma_commit(&misc->pv_done[pb]);
-                    umma_commit(&misc->v_empty[slot]);
+                    int pre = 0;
+                    if (early && ls == 0) {
+                        pre = n_early(d, NK);
+                        for (int i = 0; i < pre; ++i) issue(d, d.begin + i, i, false);
+                        grid_dependency_wait();
+                    }
+                    const int qb = ls & 1;
+                    if (ls >= 2) mbar_wait(&misc->q_empty[qb], ((ls >> 1) - 1) & 1);
+                    mbar_arrive_expect_tx(&misc->q_full[qb], 2u * (uint32_t)(p.G * p.npc) * 128u);
+                    uint8_t *qdst = s_q + qb * kQBuf;
+                    const int node0 = d.b * p.Nmax + d.c * p.npc;
+                    tma_load_3d(qdst, &tm_q, &misc->q_full[qb], 0, d.g * p.G, node0);
+                    tma_load_3d(qdst + RB * 128, &tm_q, &misc->q_full[qb], 64, d.g * p.G, node0);
+                    lt += pre;
+                    for (int t = d.begin + pre; t < d.end; ++t, ++lt) issue(d, t, lt, false);
+                    ++ls;
                 }
-                ++ls;
+                grid_launch_dependents();
+            } else if (lane == 1) {
+                int ls = 0, lt = 0;
+                for (;;) {
+                    mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
+                    const SegDesc d = misc->seg[ls % kSegRing];
+                    if (d.x < 0) {
+                        if (early && ls == 0) grid_dependency_wait();
+                        break;
+                    }
+                    int pre = 0;
+                    if (early && ls == 0) {
+                        pre = n_early(d, NV);
+                        for (int i = 0; i < pre; ++i) issue(d, d.begin + i, i, true);
+                        grid_dependency_wait();
+                    }
+                    lt += pre;
+                    for (int t = d.begin + pre; t < d.end; ++t, ++lt) issue(d, t, lt, true);
+                    ++ls;
+                }
+            }
+        } else if (warp == kWarpS) {
+            // ===================== S issuer: S(t) = Q K(t)^T into S buffer t & 1 =====================
+            // (the buffer is free once the softmax of tile t - 2 has loaded it: s_free)
+            if (lane == 0) {
+                const uint32_t idesc_s = make_idesc_bf16(128, 128, false, false);
+                const uint32_t k_addr = smem_u32(s_k), q_addr = smem_u32(s_q);
+                int lt = 0, ls = 0;
+                for (;;) {
+                    mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
+                    const SegDesc d = misc->seg[ls % kSegRing];
+                    if (d.x < 0) break;
+                    const int qb = ls & 1;
+                    mbar_wait(&misc->q_full[qb], (ls >> 1) & 1);
+                    for (int t = d.begin; t < d.end; ++t, ++lt) {
+                        const int sb = lt & 1;
+                        if (lt >= 2) mbar_wait(&misc->s_free[sb], ((lt - 2) >> 1) & 1);
+                        const int slot = lt % NK;
+                        mbar_wait(&misc->k_full[slot], (lt / NK) & 1);
+                        tc_fence_after();
+                        SPI_TRACE(2);
+                        const uint32_t kbase = k_addr + slot * kSlotBytes;
+                        const uint32_t qbase = q_addr + qb * kQBuf;
+    #pragma unroll
+                        for (int kk = 0; kk < kHeadDim / 16; ++kk) {
+                            const uint32_t off = (kk >> 2) * (RB * 128) + (kk & 3) * 32;
+                            const uint64_t adesc = make_smem_desc(qbase + off, 16, 1024, kSw128);
+                            const uint64_t bdesc = make_smem_desc(kbase + (kk >> 2) * kHalfBytes + (kk & 3) * 32, 16,
+                                                                  1024, kSw128);
+                            if (!(SPI_FLAGS(p) & 2))
+                                umma_bf16_ss(tmem + kColS + sb * 128, adesc, bdesc, idesc_s, kk > 0 ? 1u : 0u);
+                        }
+                        umma_commit(&misc->s_full[sb]);
+                        umma_commit(&misc->k_empty[slot]);
+                        if (t == d.end - 1) umma_commit(&misc->q_empty[qb]);
+                    }
+                    ++ls;
+                }
+            }
+        } else if (warp == kWarpPV) {
+            // ============ PV issuer: O += P(t) V(t) (A = P from TMEM, N = 128 dims), in tile order ============
+            if (lane == 0) {
+                const uint32_t idesc_o = make_idesc_bf16(128, 128, false, true);
+                const uint32_t v_addr = smem_u32(s_v);
+                int lt = 0, ls = 0;
+                for (;;) {
+                    mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
+                    const SegDesc d = misc->seg[ls % kSegRing];
+                    if (d.x < 0) break;
+                    for (int t = d.begin; t < d.end; ++t, ++lt) {
+                        const int pb = lt & 1;
+                        mbar_wait(&misc->p_full[pb], (lt >> 1) & 1);
+                        const bool first = (t == d.begin);
+                        if (first && ls > 0) mbar_wait(&misc->o_free, (ls - 1) & 1);  // previous segment's O read
+                        const int slot = lt % NV;
+                        mbar_wait(&misc->v_full[slot], (lt / NV) & 1);
+                        tc_fence_after();
+                        SPI_TRACE(3);
+                        const uint32_t vbase = v_addr + slot * kSlotBytes;
+    #pragma unroll
+                        for (int kk = 0; kk < kKeyTile / 16; ++kk) {
+                            const uint64_t bdesc = make_smem_desc(vbase + kk * 16 * 128, kHalfBytes, 1024, kSw128);
+                            if (!(SPI_FLAGS(p) & 2))
+                                umma_bf16_ts(tmem + kColO, tmem + kColP + pb * 64 + kk * 8, bdesc, idesc_o,
+                                             (first && kk == 0) ? 0u : 1u);
+                        }
+                        umma_commit(&misc->pv_done[pb]);
+                        umma_commit(&misc->v_empty[slot]);
+                    }
+                    ++ls;
+                }
             }
         }
     } else {
-        // ====== softmax / epilogue: two groups of 4 warps on alternating tiles, ONE shared O ======
-        // group g (warps 3 + 4g .. 6 + 4g) owns the tiles with lt & 1 == g; thread = one query row (TMEM
-        // lane).  Both groups accumulate into the same O, so every P(t) must use the row reference the
-        // previous tile left: the owner of tile t reads decision(t - 1) (the other group's, through
-        // shared memory + a producer/consumer named barrier per lane quarter), may raise it (stale
-        // max: only beyond 2^8, then O is rescaled after PV(t - 1)), publishes decision(t) and only then
-        // computes its exponentials -- the groups run out of phase, so one group's loads / maxima /
-        // handshake overlap the other's exponentials.  The owner of a segment's last tile writes the
-        // rows (the other group hands over its partial row sums through shared memory).
-        const int sw = warp - 3;               // 0..7
-        const int grp = sw >> 2;               // tile parity owned by this group
-        const int qd = warp & 3;               // TMEM lane quarter
-        const int r = qd * 32 + lane;          // query row of the item = TMEM lane
-        const uint32_t lane_off = (uint32_t)(qd * 32) << 16;
-        // decision(t) hand-over between the two warps of quarter qd: one named barrier PER DIRECTION.
-        // (With a single barrier, the publisher's arrive(t) and its own sync at tile t + 2 could complete
-        // the barrier together whenever the other warp reached its sync for t + 1 late -- the publisher
-        // would then read a stale reference.  Per direction, arrivals and syncs strictly alternate.)
-        const uint32_t dec_out = grp == 0 ? 6 + qd : 1 + qd;   // the decisions this group publishes
-        const uint32_t dec_in = grp == 0 ? 1 + qd : 6 + qd;    // the other group's decisions
-        const uint32_t epi_bar = 10 + qd;      // segment-end row-sum hand-over
-        const uint32_t o_col = tmem + kColO + lane_off;
-        float *mref_s = misc->xm[0][0];        // [row] the row reference after the latest decision
-        float *xl_l = misc->xm[1][0];          // [row] the non-owner group's row sum at a segment end
-        float *xl_m = misc->xm[1][1];          //       ... and the reference it is relative to
-        float *xl_f = misc->xm[0][1];          // [row] the final row sum (owner -> the other group)
-        int lt = 0, ls = 0;
-        for (;;) {
-            mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
-            const SegDesc sd = misc->seg[ls % kSegRing];
-            if (sd.x < 0) break;
-            const int b = sd.b, g = sd.g, c = sd.c, P = sd.P, n = sd.n;
-            const int Kend = P + n;
-            const int G = p.G;
-            const int rc = G * p.npc;
-            const int node = c * p.npc + r / G, hl = r % G;
-            const bool row_valid = (r < rc) && (node < n);
-            // ancestor-or-self bitset of this row's node, read on masked tiles only (rows without a
-            // node use node 0's root path, which keeps them finite; they are never written)
-            const uint32_t *anc = p.anc + ((size_t)b * p.Nmax + (row_valid ? node : 0)) * kBitWords;
-            // the masked (tree) tiles come last in a segment: pull the row's bitset into L1 now, so their
-            // __ldg's hit L1 instead of paying an L2 round trip on the softmax critical path
-            asm volatile("prefetch.global.L1 [%0];" ::"l"(anc));
-            float m = -INFINITY, l = 0.f;      // latest known row reference (log2 units), this group's sum
-            const int lt0 = lt;
-            for (int t = sd.begin; t < sd.end; ++t, ++lt) {
-                if ((lt & 1) != grp) continue;
-                const int sb = lt & 1;
-                const int key0 = (t - sd.ib) * kKeyTile;
-                mbar_wait(&misc->s_full[sb], (lt >> 1) & 1);
-                tc_fence_after();
-                if (r == 0) SPI_TRACE(4 + grp);
-                const uint32_t s_col = tmem + kColS + sb * 128 + lane_off;
-                // visibility of the tile's 128 keys (4 words): committed keys visible; tree keys by the
-                // ancestor bitset; keys past the request's end: none
-                uint32_t vis[4] = {0xFFFFFFFFu, 0xFFFFFFFFu, 0xFFFFFFFFu, 0xFFFFFFFFu};
-                const bool masked = key0 + kKeyTile > P;
-                if (masked) {
-#pragma unroll
-                    for (int q = 0; q < 4; ++q) {
-                        const int j0 = key0 + 32 * q - P;  // tree index of the group's first key
-                        if (j0 + 32 > 0) {
-                            const int jb = max(j0, 0);
-                            const int wi = jb >> 5, sh = jb & 31;
-                            const uint32_t lo = __ldg(anc + wi);
-                            const uint32_t hi = wi + 1 < kBitWords ? __ldg(anc + wi + 1) : 0u;
-                            uint32_t bits = sh ? ((lo >> sh) | (hi << (32 - sh))) : lo;
-                            if (j0 < 0) bits = (bits << (-j0)) | ((1u << (-j0)) - 1u);
-                            const int nvalid = Kend - (key0 + 32 * q);
-                            if (nvalid < 32) bits &= nvalid <= 0 ? 0u : ((1u << nvalid) - 1u);
-                            vis[q] = bits;
-                        }
-                    }
-                }
-                // pass 1: this row's tile max
-                float tm;
-                {
-                    float m4[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
-#pragma unroll
-                    for (int hh = 0; hh < 2; ++hh) {
-                        uint32_t a[2][32];
-                        tmem_ld32(s_col + hh * 64, a[0]);
-                        tmem_ld32(s_col + hh * 64 + 32, a[1]);
-                        tmem_ld_wait();
-#pragma unroll
-                        for (int q = 0; q < 2; ++q) {
-                            if (masked) rows::mask32(a[q], vis[2 * hh + q]);
-#pragma unroll
-                            for (int i = 0; i < 32; ++i) m4[i & 3] = fmaxf(m4[i & 3], __uint_as_float(a[q][i]));
-                        }
-                    }
-                    tm = fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3])) * p.scale_log2;
-                }
-                // decision(t - 1): the reference P(t - 1) used (ignored at a segment's first tile: new rows)
-                if (lt > 0) {
-                    named_bar_sync(dec_in, 64);
-                    const float mp = mref_s[r];
-                    if (lt > lt0 && mp != m) {   // the other group raised it: rebase this group's sum
-                        l = (m == -INFINITY) ? 0.f : l * ex2(m - mp);
-                        m = mp;
-                    }
-                }
-                if (r == 0) SPI_TRACE(8 + grp);
-                // decision(t): stale running max, moved only when this tile exceeds it by more than 2^8
-                float alpha = 1.f;
-                if (tm > m + kRescaleThreshold) {
-                    alpha = (m == -INFINITY) ? 0.f : ex2(m - tm);
-                    m = tm;
-                    l *= alpha;
-                }
-                const bool moved = __any_sync(0xffffffffu, alpha != 1.f) && lt > lt0;
-                if (moved) {
-                    // O holds PV(<= t - 1) against the old reference: rescale once PV(t - 1) completed.
-                    // This group last observed pv_done of ITS parity (PV(t - 4)); the other barrier may
-                    // still be a phase behind PV(t - 1)'s, which a parity wait cannot tell apart from
-                    // "complete": first PV(t - 2) (own barrier, one phase ahead), which implies PV(t - 3).
-                    if (lt >= 2) mbar_wait(&misc->pv_done[lt & 1], ((lt - 2) >> 1) & 1);
-                    mbar_wait(&misc->pv_done[(lt - 1) & 1], ((lt - 1) >> 1) & 1);
-                    tc_fence_after();
-#pragma unroll 1
-                    for (int q2 = 0; q2 < 4; ++q2) {
-                        uint32_t v[32];
-                        tmem_ld32(o_col + q2 * 32, v);
-                        tmem_ld_wait();
-                        uint32_t w16[16];
-#pragma unroll
-                        for (int hh = 0; hh < 2; ++hh) {
-#pragma unroll
-                            for (int i = 0; i < 16; ++i) w16[i] = __float_as_uint(__uint_as_float(v[hh * 16 + i]) * alpha);
-                            tmem_st16(o_col + q2 * 32 + hh * 16, w16);
-                        }
-                    }
-                    tmem_st_wait();
-                }
-                mref_s[r] = m;
-                named_bar_arrive(dec_out, 64);   // decision(t) -> the owner of tile t + 1
-                // pass 2: P(t) = 2^(s * scale - m) as bf16 pairs into P buffer t & 1 (free once PV(t - 2)
-                // completed), row sum of the rounded values
-                if (lt >= 2) mbar_wait(&misc->pv_done[sb], ((lt - 2) >> 1) & 1);
-                tc_fence_after();
-                {
-                    const float mref = (m == -INFINITY) ? 0.f : m;
-                    const uint64_t sc2 = f2_bits(p.scale_log2, p.scale_log2), nm2 = f2_bits(-mref, -mref);
-                    const uint32_t p_col = tmem + kColP + sb * 64 + lane_off;
-                    float ls2 = 0.f;
-#pragma unroll
-                    for (int hh = 0; hh < 2; ++hh) {
-                        uint32_t a[2][32];
-                        tmem_ld32(s_col + hh * 64, a[0]);
-                        tmem_ld32(s_col + hh * 64 + 32, a[1]);
-                        tmem_ld_wait();
-                        if (hh == 1) {
-                            tc_fence_before();
-                            __syncwarp();
-                            if (lane == 0) mbar_arrive(&misc->s_free[sb]);   // S(t + 2) may overwrite it
-                        }
-#pragma unroll
-                        for (int q = 0; q < 2; ++q) {
-                            if (masked) rows::mask32(a[q], vis[2 * hh + q]);
-                            uint32_t w16[16];
-                            float dummy = 0.f;
-                            ls2 += rows::exp32<false>(a[q], sc2, nm2, w16, dummy);
-                            tmem_st16(p_col + hh * 32 + q * 16, w16);
-                        }
-                    }
-                    l += (SPI_FLAGS(p) & 8) ? 1.f : ls2;
-                }
-                tmem_st_wait();
-                tc_fence_before();
-                __syncwarp();
-                if (lane == 0) mbar_arrive(&misc->p_full[sb]);
-                if (r == 0) SPI_TRACE(6 + grp);
-            }
-
-            // ============ epilogue of this segment ============
-            // The owner of the segment's last tile combines both groups' row sums; for a whole item both
-            // groups then write half of the row's 128 dims each (the output store of one group alone
-            // stalled the other group's next tile for the whole epilogue), a split piece is written by
-            // the owner.
-            const int llast = lt - 1;
-            const int owner = llast & 1;
-            const bool full = (sd.begin == sd.ib) && (sd.end == sd.ie);
-            // (two full barriers, executed by both groups at the same two instructions: the non-owner may
-            // not overwrite the hand-over slots of the next segment before the owner has read them, and
-            // it reads the final sum only after the owner wrote it)
-            if (grp != owner) {
-                xl_l[r] = l;
-                xl_m[r] = m;
-            }
-            named_bar_sync(epi_bar, 64);
-            float lrow = 0.f;
-            if (grp == owner) {
-                const float lo_ = xl_l[r], mo = xl_m[r];
-                lrow = l + ((mo == -INFINITY || lo_ == 0.f) ? 0.f : lo_ * ex2(mo - m));
-                xl_f[r] = lrow;
-            }
-            named_bar_sync(epi_bar, 64);
-            if (grp != owner) {
-                if (full) {
-                    const float inv = 1.0f / xl_f[r];
-                    // O complete: this group last observed pv_done of ITS parity, so first wait for PV(llast - 1)
-                    // (its own tile: at most one phase ahead), which implies PV(llast - 2); only then is the
-                    // parity wait for PV(llast) on the other barrier unambiguous
-                    if (llast >= 1) mbar_wait(&misc->pv_done[(llast - 1) & 1], ((llast - 1) >> 1) & 1);
-                    mbar_wait(&misc->pv_done[llast & 1], (llast >> 1) & 1);
-                    tc_fence_after();
-                    store_o_half(o_col, inv, row_valid,
-                                 p.out + (((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim, 1,
-                                 &misc->o_free);
-                } else {
-                    tc_fence_before();
-                    __syncwarp();
-                    if (lane == 0) mbar_arrive(&misc->o_free);
-                }
-            } else {
-                mbar_wait(&misc->pv_done[llast & 1], (llast >> 1) & 1);   // O complete (in-order PVs)
-                tc_fence_after();
-                if (r == 0) SPI_TRACE(10);
-                if (full) {
-                    store_o_half(o_col, 1.0f / lrow, row_valid,
-                                 p.out + (((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim, 0,
-                                 &misc->o_free);
-                } else {
-                    // a piece of a split item: unnormalised O row, (m, l) of the row, then the last piece
-                    // merges every piece by log-sum-exp
-                    const int slot = (sd.begin == t0) ? 0 : 1;
-                    float *po = p.part_o + (((size_t)blockIdx.x * 2 + slot) * RB + r) * kHeadDim;
-#pragma unroll 1
-                    for (int q2 = 0; q2 < 4; ++q2) {
-                        uint32_t o[32];
-                        tmem_ld32(o_col + q2 * 32, o);
-                        tmem_ld_wait();
-#pragma unroll
-                        for (int i = 0; i < 32; i += 8)   // 32-byte stores (part_o rows are 512-byte aligned)
-                            asm volatile("st.global.v8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"l"(po + q2 * 32 + i),
-                                         "r"(o[i]), "r"(o[i + 1]), "r"(o[i + 2]), "r"(o[i + 3]), "r"(o[i + 4]),
-                                         "r"(o[i + 5]), "r"(o[i + 6]), "r"(o[i + 7])
-                                         : "memory");
-                    }
-                    tc_fence_before();
-                    __syncwarp();
-                    if (lane == 0) mbar_arrive(&misc->o_free);
-                    float *pml = p.part_ml + ((size_t)blockIdx.x * 2 + slot) * 2 * RB;
-                    pml[r] = m;
-                    pml[RB + r] = lrow;
-                    if (r == 0) SPI_TRACE(12);
-                    __threadfence();
-                    named_bar_sync(14, 128);   // the owner group's 4 warps
-                    if (r == 0) {
-                        const int c_first = cta_of_tile(sd.ib, T, NC);
-                        const int c_last = cta_of_tile(sd.ie - 1, T, NC);
-                        int npieces = 0;
-                        for (int cc = c_first; cc <= c_last; ++cc)
-                            npieces += cta_start(cc + 1, T, NC) > cta_start(cc, T, NC);
-                        const unsigned old = atomicAdd(&p.item_cnt[sd.x], 1u);
-                        misc->bcast = (old == (unsigned)(npieces - 1)) ? 1 : 0;
-                        if (misc->bcast) p.item_cnt[sd.x] = 0u;  // ready for the next launch
-                    }
-                    named_bar_sync(14, 128);
-                    if (r == 0) SPI_TRACE(13);
-                    if (misc->bcast) {
-                        // last piece: merge every piece's (m, l, O row) by log-sum-exp
-                        __threadfence();
-                        const int c_first = cta_of_tile(sd.ib, T, NC);
-                        const int c_last = cta_of_tile(sd.ie - 1, T, NC);
-                        auto piece = [&](int cc) -> long long {   // partial slot of CTA cc's piece, -1 if empty
-                            const int s0 = cta_start(cc, T, NC);
-                            if (cta_start(cc + 1, T, NC) <= s0) return -1;
-                            return ((long long)cc * p.lanes + cl) * 2 + ((s0 >= sd.ib) ? 0 : 1);
-                        };
-                        // (compact, rolled loops: this code runs cold in the instruction cache, once per item,
-                        // and its length -- not its loads -- set the cost: ~350 ns per missed 128-B line)
-                        if (sd.end == t1) {
-                            // the CTA's last segment: K / V rings and Q buffers are idle -> stage the pieces with
-                            // bulk copies (all in flight at once) instead of one L2 round trip per (piece, chunk):
-                            // (m, l) of every piece, then up to `cap` 64 KB O blocks per round; each warp merges
-                            // its 32 rows with lane = 4 dims (conflict-free, coalesced 256 B output rows)
-                            uint8_t *area = smem;
-                            const size_t area_bytes = (size_t)(NK + NV) * kSlotBytes + 2 * kQBuf;
-                            constexpr uint32_t kOB = RB * kHeadDim * 4, kMLB = 2 * RB * 4;
-                            int npc = 0;
-                            for (int cc = c_first; cc <= c_last; ++cc) npc += piece(cc) >= 0;
-                            float *sml = reinterpret_cast<float *>(area + area_bytes) - (size_t)npc * 3 * RB;  // [npc][m, l, w][RB]
-                            const int cap = (int)(((size_t)((uint8_t *)sml - area)) / kOB);
-                            uint32_t ph = 0;
-                            if (r == 0) {
-                                fence_proxy_async_global();
-                                mbar_arrive_expect_tx(&misc->stage_bar, (uint32_t)npc * kMLB);
-                                int k = 0;
-                                for (int cc = c_first; cc <= c_last; ++cc) {
-                                    const long long po2 = piece(cc);
-                                    if (po2 < 0) continue;
-                                    bulk_load_g2s(sml + (size_t)k * 3 * RB, p.part_ml + po2 * 2 * RB, kMLB, &misc->stage_bar);
-                                    ++k;
+        setmaxnreg_inc<kRegsSoftmax>();
+        if (ntiles > 0) {
+                // ====== softmax / epilogue: two groups of 4 warps on alternating tiles, ONE shared O ======
+                // group g (warps 3 + 4g .. 6 + 4g) owns the tiles with lt & 1 == g; thread = one query row (TMEM
+                // lane).  Both groups accumulate into the same O, so every P(t) must use the row reference the
+                // previous tile left: the owner of tile t reads decision(t - 1) (the other group's, through
+                // shared memory + a producer/consumer named barrier per lane quarter), may raise it (stale
+                // max: only beyond 2^8, then O is rescaled after PV(t - 1)), publishes decision(t) and only then
+                // computes its exponentials -- the groups run out of phase, so one group's loads / maxima /
+                // handshake overlap the other's exponentials.  The owner of a segment's last tile writes the
+                // rows (the other group hands over its partial row sums through shared memory).
+                const int sw = warp;                   // 0..7
+                const int grp = sw >> 2;               // tile parity owned by this group
+                const int qd = warp & 3;               // TMEM lane quarter
+                const int r = qd * 32 + lane;          // query row of the item = TMEM lane
+                const uint32_t lane_off = (uint32_t)(qd * 32) << 16;
+                // decision(t) hand-over between the two warps of quarter qd: one named barrier PER DIRECTION.
+                // (With a single barrier, the publisher's arrive(t) and its own sync at tile t + 2 could complete
+                // the barrier together whenever the other warp reached its sync for t + 1 late -- the publisher
+                // would then read a stale reference.  Per direction, arrivals and syncs strictly alternate.)
+                const uint32_t dec_out = grp == 0 ? 6 + qd : 1 + qd;   // the decisions this group publishes
+                const uint32_t dec_in = grp == 0 ? 1 + qd : 6 + qd;    // the other group's decisions
+                const uint32_t epi_bar = 10 + qd;      // segment-end row-sum hand-over
+                const uint32_t o_col = tmem + kColO + lane_off;
+                float *mref_s = misc->xm[0][0];        // [row] the row reference after the latest decision
+                float *xl_l = misc->xm[1][0];          // [row] the non-owner group's row sum at a segment end
+                float *xl_m = misc->xm[1][1];          //       ... and the reference it is relative to
+                float *xl_f = misc->xm[0][1];          // [row] the final row sum (owner -> the other group)
+                int lt = 0, ls = 0;
+                for (;;) {
+                    mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
+                    const SegDesc sd = misc->seg[ls % kSegRing];
+                    if (sd.x < 0) break;
+                    const int b = sd.b, g = sd.g, c = sd.c, P = sd.P, n = sd.n;
+                    const int Kend = P + n;
+                    const int G = p.G;
+                    const int rc = G * p.npc;
+                    const int node = c * p.npc + r / G, hl = r % G;
+                    const bool row_valid = (r < rc) && (node < n);
+                    // ancestor-or-self bitset of this row's node, read on masked tiles only (rows without a
+                    // node use node 0's root path, which keeps them finite; they are never written)
+                    const uint32_t *anc = p.anc + ((size_t)b * p.Nmax + (row_valid ? node : 0)) * kBitWords;
+                    // the masked (tree) tiles come last in a segment: pull the row's bitset into L1 now, so their
+                    // __ldg's hit L1 instead of paying an L2 round trip on the softmax critical path
+                    asm volatile("prefetch.global.L1 [%0];" ::"l"(anc));
+                    float m = -INFINITY, l = 0.f;      // latest known row reference (log2 units), this group's sum
+                    const int lt0 = lt;
+                    for (int t = sd.begin; t < sd.end; ++t, ++lt) {
+                        if ((lt & 1) != grp) continue;
+                        const int sb = lt & 1;
+                        const int key0 = (t - sd.ib) * kKeyTile;
+                        mbar_wait(&misc->s_full[sb], (lt >> 1) & 1);
+                        tc_fence_after();
+                        if (r == 0) SPI_TRACE(4 + grp);
+                        const uint32_t s_col = tmem + kColS + sb * 128 + lane_off;
+                        // visibility of the tile's 128 keys (4 words): committed keys visible; tree keys by the
+                        // ancestor bitset; keys past the request's end: none
+                        uint32_t vis[4] = {0xFFFFFFFFu, 0xFFFFFFFFu, 0xFFFFFFFFu, 0xFFFFFFFFu};
+                        const bool masked = key0 + kKeyTile > P;
+                        if (masked) {
+        #pragma unroll
+                            for (int q = 0; q < 4; ++q) {
+                                const int j0 = key0 + 32 * q - P;  // tree index of the group's first key
+                                if (j0 + 32 > 0) {
+                                    const int jb = max(j0, 0);
+                                    const int wi = jb >> 5, sh = jb & 31;
+                                    const uint32_t lo = __ldg(anc + wi);
+                                    const uint32_t hi = wi + 1 < kBitWords ? __ldg(anc + wi + 1) : 0u;
+                                    uint32_t bits = sh ? ((lo >> sh) | (hi << (32 - sh))) : lo;
+                                    if (j0 < 0) bits = (bits << (-j0)) | ((1u << (-j0)) - 1u);
+                                    const int nvalid = Kend - (key0 + 32 * q);
+                                    if (nvalid < 32) bits &= nvalid <= 0 ? 0u : ((1u << nvalid) - 1u);
+                                    vis[q] = bits;
                                 }
                             }
-                            mbar_wait(&misc->stage_bar, ph);
-                            ph ^= 1u;
-                            float Mx = -INFINITY, Ls = 0.f;
-                            for (int k = 0; k < npc; ++k) Mx = fmaxf(Mx, sml[(size_t)k * 3 * RB + r]);
-                            for (int k = 0; k < npc; ++k) {
-                                const float mk = sml[(size_t)k * 3 * RB + r];
-                                const float w = (mk == -INFINITY) ? 0.f : ex2(mk - Mx);
-                                Ls += w * sml[(size_t)k * 3 * RB + RB + r];
-                                sml[(size_t)k * 3 * RB + 2 * RB + r] = w;
+                        }
+                        // pass 1: this row's tile max
+                        float tm;
+                        uint32_t sv[4][32];   // the row's scores stay in registers for pass 2 (chunk 0 is reloaded there)
+                        {
+                            float m4[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
+        #pragma unroll
+                            for (int q = 0; q < 4; ++q) tmem_ld32(s_col + q * 32, sv[q]);
+                            tmem_ld_wait();
+        #pragma unroll
+                            for (int q = 0; q < 4; ++q) {
+                                if (masked) rows::mask32(sv[q], vis[q]);
+        #pragma unroll
+                                for (int i = 0; i < 32; ++i) m4[i & 3] = fmaxf(m4[i & 3], __uint_as_float(sv[q][i]));
                             }
-                            const float inv = 1.0f / Ls;
-                            for (int k = 0; k < npc; ++k) sml[(size_t)k * 3 * RB + 2 * RB + r] *= inv;
-                            named_bar_sync(14, 128);   // weights visible to the whole group
-                            float4 acc[32];   // [row of the warp] lane's 4 dims
-#pragma unroll
-                            for (int i = 0; i < 32; ++i) acc[i] = make_float4(0.f, 0.f, 0.f, 0.f);
-                            const int wrow0 = qd * 32;   // this warp's rows
-                            for (int k0 = 0; k0 < npc; k0 += cap) {
-                                const int kn = min(cap, npc - k0);
-                                if (r == 0) {
-                                    mbar_arrive_expect_tx(&misc->stage_bar, (uint32_t)kn * kOB);
-                                    int k = 0;
+                            tm = fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3])) * p.scale_log2;
+                        }
+                        // decision(t - 1): the reference P(t - 1) used (ignored at a segment's first tile: new rows)
+                        if (lt > 0) {
+                            named_bar_sync(dec_in, 64);
+                            const float mp = mref_s[r];
+                            if (lt > lt0 && mp != m) {   // the other group raised it: rebase this group's sum
+                                l = (m == -INFINITY) ? 0.f : l * ex2(m - mp);
+                                m = mp;
+                            }
+                        }
+                        if (r == 0) SPI_TRACE(8 + grp);
+                        // decision(t): stale running max, moved only when this tile exceeds it by more than 2^8
+                        float alpha = 1.f;
+                        if (tm > m + kRescaleThreshold) {
+                            alpha = (m == -INFINITY) ? 0.f : ex2(m - tm);
+                            m = tm;
+                            l *= alpha;
+                        }
+                        const bool moved = __any_sync(0xffffffffu, alpha != 1.f) && lt > lt0;
+                        // O holds PV(<= t - 1) against the old reference: rescale it once PV(t - 1) completed and
+                        // before PV(t) is issued (p_full).  This group last observed pv_done of ITS parity (PV(t - 4));
+                        // the other barrier may still be a phase behind PV(t - 1)'s, which a parity wait cannot tell
+                        // apart from "complete": first PV(t - 2) (own barrier, one phase ahead), which implies PV(t - 3).
+                        auto rescale_o = [&]() {
+                            if (lt >= 2) mbar_wait(&misc->pv_done[lt & 1], ((lt - 2) >> 1) & 1);
+                            mbar_wait(&misc->pv_done[(lt - 1) & 1], ((lt - 1) >> 1) & 1);
+                            tc_fence_after();
+        #pragma unroll 1
+                            for (int q2 = 0; q2 < 4; ++q2) {
+                                uint32_t v[32];
+                                tmem_ld32(o_col + q2 * 32, v);
+                                tmem_ld_wait();
+                                uint32_t w16[16];
+        #pragma unroll
+                                for (int hh = 0; hh < 2; ++hh) {
+        #pragma unroll
+                                    for (int i = 0; i < 16; ++i) w16[i] = __float_as_uint(__uint_as_float(v[hh * 16 + i]) * alpha);
+                                    tmem_st16(o_col + q2 * 32 + hh * 16, w16);
+                                }
+                            }
+                        };
+                        mref_s[r] = m;
+                        named_bar_arrive(dec_out, 64);   // decision(t) -> the owner of tile t + 1
+                        // pass 2: P(t) = 2^(s * scale - m) as bf16 pairs, row sum of the rounded values; every
+                        // exponential is computed into registers first, and only the TMEM stores into P buffer t & 1
+                        // wait for PV(t - 2) to have read it (that wait overlaps the exponentials)
+                        {
+                            const float mref = (m == -INFINITY) ? 0.f : m;
+                            const uint64_t sc2 = f2_bits(p.scale_log2, p.scale_log2), nm2 = f2_bits(-mref, -mref);
+                            const uint32_t p_col = tmem + kColP + sb * 64 + lane_off;
+                            float ls2 = 0.f;
+                            // chunk 0 of the scores was not kept across the decision (register pressure): reload it,
+                            // then the S buffer is free
+                            tmem_ld32(s_col, sv[0]);
+                            tmem_ld_wait();
+                            tc_fence_before();
+                            __syncwarp();
+                            if (lane == 0) mbar_arrive(&misc->s_free[sb]);
+                            if (masked) rows::mask32(sv[0], vis[0]);
+                            uint32_t w16[4][16];
+        #pragma unroll
+                            for (int q = 0; q < 4; ++q) {
+                                float dummy = 0.f;
+                                ls2 += rows::exp32<false>(sv[q], sc2, nm2, w16[q], dummy);
+                            }
+                            if (lt >= 2) mbar_wait(&misc->pv_done[sb], ((lt - 2) >> 1) & 1);
+                            tc_fence_after();
+        #pragma unroll
+                            for (int q = 0; q < 4; ++q) tmem_st16(p_col + q * 16, w16[q]);
+                            l += (SPI_FLAGS(p) & 8) ? 1.f : ls2;
+                        }
+                        if (moved) rescale_o();   // (the scores' registers are dead by now)
+                        tmem_st_wait();
+                        tc_fence_before();
+                        __syncwarp();
+                        if (lane == 0) mbar_arrive(&misc->p_full[sb]);
+                        if (r == 0) SPI_TRACE(6 + grp);
+                    }
+
+                    // ============ epilogue of this segment ============
+                    // The owner of the segment's last tile combines both groups' row sums; for a whole item both
+                    // groups then write half of the row's 128 dims each (the output store of one group alone
+                    // stalled the other group's next tile for the whole epilogue), a split piece is written by
+                    // the owner.
+                    const int llast = lt - 1;
+                    const int owner = llast & 1;
+                    const bool full = (sd.begin == sd.ib) && (sd.end == sd.ie);
+                    // (two full barriers, executed by both groups at the same two instructions: the non-owner may
+                    // not overwrite the hand-over slots of the next segment before the owner has read them, and
+                    // it reads the final sum only after the owner wrote it)
+                    if (grp != owner) {
+                        xl_l[r] = l;
+                        xl_m[r] = m;
+                    }
+                    named_bar_sync(epi_bar, 64);
+                    float lrow = 0.f;
+                    if (grp == owner) {
+                        const float lo_ = xl_l[r], mo = xl_m[r];
+                        lrow = l + ((mo == -INFINITY || lo_ == 0.f) ? 0.f : lo_ * ex2(mo - m));
+                        xl_f[r] = lrow;
+                    }
+                    named_bar_sync(epi_bar, 64);
+                    if (grp != owner) {
+                        if (full) {
+                            const float inv = 1.0f / xl_f[r];
+                            // O complete: this group last observed pv_done of ITS parity, so first wait for PV(llast - 1)
+                            // (its own tile: at most one phase ahead), which implies PV(llast - 2); only then is the
+                            // parity wait for PV(llast) on the other barrier unambiguous
+                            if (llast >= 1) mbar_wait(&misc->pv_done[(llast - 1) & 1], ((llast - 1) >> 1) & 1);
+                            mbar_wait(&misc->pv_done[llast & 1], (llast >> 1) & 1);
+                            tc_fence_after();
+                            store_o_half(o_col, inv, row_valid,
+                                         p.out + (((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim, 1,
+                                         &misc->o_free);
+                        } else {
+                            tc_fence_before();
+                            __syncwarp();
+                            if (lane == 0) mbar_arrive(&misc->o_free);
+                        }
+                    } else {
+                        mbar_wait(&misc->pv_done[llast & 1], (llast >> 1) & 1);   // O complete (in-order PVs)
+                        tc_fence_after();
+                        if (r == 0) SPI_TRACE(10);
+                        if (full) {
+                            store_o_half(o_col, 1.0f / lrow, row_valid,
+                                         p.out + (((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim, 0,
+                                         &misc->o_free);
+                        } else {
+                            // a piece of a split item: unnormalised O row, (m, l) of the row, then the last piece
+                            // merges every piece by log-sum-exp
+                            const int slot = (sd.begin == t0) ? 0 : 1;
+                            float *po = p.part_o + (((size_t)blockIdx.x * 2 + slot) * RB + r) * kHeadDim;
+        #pragma unroll 1
+                            for (int q2 = 0; q2 < 4; ++q2) {
+                                uint32_t o[32];
+                                tmem_ld32(o_col + q2 * 32, o);
+                                tmem_ld_wait();
+        #pragma unroll
+                                for (int i = 0; i < 32; i += 8)   // 32-byte stores (part_o rows are 512-byte aligned)
+                                    asm volatile("st.global.v8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"l"(po + q2 * 32 + i),
+                                                 "r"(o[i]), "r"(o[i + 1]), "r"(o[i + 2]), "r"(o[i + 3]), "r"(o[i + 4]),
+                                                 "r"(o[i + 5]), "r"(o[i + 6]), "r"(o[i + 7])
+                                                 : "memory");
+                            }
+                            tc_fence_before();
+                            __syncwarp();
+                            if (lane == 0) mbar_arrive(&misc->o_free);
+                            float *pml = p.part_ml + ((size_t)blockIdx.x * 2 + slot) * 2 * RB;
+                            pml[r] = m;
+                            pml[RB + r] = lrow;
+                            if (r == 0) SPI_TRACE(12);
+                            __threadfence();
+                            named_bar_sync(14, 128);   // the owner group's 4 warps
+                            if (r == 0) {
+                                const int c_first = cta_of_tile(sd.ib, T, NC);
+                                const int c_last = cta_of_tile(sd.ie - 1, T, NC);
+                                int npieces = 0;
+                                for (int cc = c_first; cc <= c_last; ++cc)
+                                    npieces += cta_start(cc + 1, T, NC) > cta_start(cc, T, NC);
+                                const unsigned old = atomicAdd(&p.item_cnt[sd.x], 1u);
+                                misc->bcast = (old == (unsigned)(npieces - 1)) ? 1 : 0;
+                                if (misc->bcast) p.item_cnt[sd.x] = 0u;  // ready for the next launch
+                            }
+                            named_bar_sync(14, 128);
+                            if (r == 0) SPI_TRACE(13);
+                            if (misc->bcast) {
+                                // last piece: merge every piece's (m, l, O row) by log-sum-exp
+                                __threadfence();
+                                const int c_first = cta_of_tile(sd.ib, T, NC);
+                                const int c_last = cta_of_tile(sd.ie - 1, T, NC);
+                                auto piece = [&](int cc) -> long long {   // partial slot of CTA cc's piece, -1 if empty
+                                    const int s0 = cta_start(cc, T, NC);
+                                    if (cta_start(cc + 1, T, NC) <= s0) return -1;
+                                    return ((long long)cc * p.lanes + cl) * 2 + ((s0 >= sd.ib) ? 0 : 1);
+                                };
+                                // (compact, rolled loops: this code runs cold in the instruction cache, once per item,
+                                // and its length -- not its loads -- set the cost: ~350 ns per missed 128-B line)
+                                if (sd.end == t1) {
+                                    // the CTA's last segment: K / V rings and Q buffers are idle -> stage the pieces with
+                                    // bulk copies (all in flight at once) instead of one L2 round trip per (piece, chunk):
+                                    // (m, l) of every piece, then up to `cap` 64 KB O blocks per round; each warp merges
+                                    // its 32 rows with lane = 4 dims (conflict-free, coalesced 256 B output rows)
+                                    uint8_t *area = smem;
+                                    const size_t area_bytes = (size_t)(NK + NV) * kSlotBytes + 2 * kQBuf;
+                                    constexpr uint32_t kOB = RB * kHeadDim * 4, kMLB = 2 * RB * 4;
+                                    int npc = 0;
+                                    for (int cc = c_first; cc <= c_last; ++cc) npc += piece(cc) >= 0;
+                                    float *sml = reinterpret_cast<float *>(area + area_bytes) - (size_t)npc * 3 * RB;  // [npc][m, l, w][RB]
+                                    const int cap = (int)(((size_t)((uint8_t *)sml - area)) / kOB);
+                                    uint32_t ph = 0;
+                                    if (r == 0) {
+                                        fence_proxy_async_global();
+                                        mbar_arrive_expect_tx(&misc->stage_bar, (uint32_t)npc * kMLB);
+                                        int k = 0;
+                                        for (int cc = c_first; cc <= c_last; ++cc) {
+                                            const long long po2 = piece(cc);
+                                            if (po2 < 0) continue;
+                                            bulk_load_g2s(sml + (size_t)k * 3 * RB, p.part_ml + po2 * 2 * RB, kMLB, &misc->stage_bar);
+                                            ++k;
+                                        }
+                                    }
+                                    mbar_wait(&misc->stage_bar, ph);
+                                    ph ^= 1u;
+                                    float Mx = -INFINITY, Ls = 0.f;
+                                    for (int k = 0; k < npc; ++k) Mx = fmaxf(Mx, sml[(size_t)k * 3 * RB + r]);
+                                    for (int k = 0; k < npc; ++k) {
+                                        const float mk = sml[(size_t)k * 3 * RB + r];
+                                        const float w = (mk == -INFINITY) ? 0.f : ex2(mk - Mx);
+                                        Ls += w * sml[(size_t)k * 3 * RB + RB + r];
+                                        sml[(size_t)k * 3 * RB + 2 * RB + r] = w;
+                                    }
+                                    const float inv = 1.0f / Ls;
+                                    for (int k = 0; k < npc; ++k) sml[(size_t)k * 3 * RB + 2 * RB + r] *= inv;
+                                    named_bar_sync(14, 128);   // weights visible to the whole group
+                                    float4 acc[32];   // [row of the warp] lane's 4 dims
+        #pragma unroll
+                                    for (int i = 0; i < 32; ++i) acc[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+                                    const int wrow0 = qd * 32;   // this warp's rows
+                                    for (int k0 = 0; k0 < npc; k0 += cap) {
+                                        const int kn = min(cap, npc - k0);
+                                        if (r == 0) {
+                                            mbar_arrive_expect_tx(&misc->stage_bar, (uint32_t)kn * kOB);
+                                            int k = 0;
+                                            for (int cc = c_first; cc <= c_last; ++cc) {
+                                                const long long po2 = piece(cc);
+                                                if (po2 < 0) continue;
+                                                if (k >= k0 && k < k0 + kn)
+                                                    bulk_load_g2s(area + (size_t)(k - k0) * kOB, p.part_o + po2 * RB * kHeadDim, kOB,
+                                                                  &misc->stage_bar);
+                                                ++k;
+                                            }
+                                        }
+                                        mbar_wait(&misc->stage_bar, ph);
+                                        ph ^= 1u;
+        #pragma unroll 1
+                                        for (int k = 0; k < kn; ++k) {
+                                            const float *blk = reinterpret_cast<const float *>(area + (size_t)k * kOB);
+                                            const float *wk = sml + (size_t)(k0 + k) * 3 * RB + 2 * RB + wrow0;
+        #pragma unroll
+                                            for (int i = 0; i < 32; ++i) {
+                                                const float4 x = *reinterpret_cast<const float4 *>(blk + (size_t)(wrow0 + i) * kHeadDim + 4 * lane);
+                                                const float w = wk[i];
+                                                acc[i].x += w * x.x;
+                                                acc[i].y += w * x.y;
+                                                acc[i].z += w * x.z;
+                                                acc[i].w += w * x.w;
+                                            }
+                                        }
+                                        named_bar_sync(14, 128);   // the staging area is reused by the next round
+                                    }
+                                    // rows of this warp: row wrow0 + i -> its node / head (padding rows skipped)
+        #pragma unroll
+                                    for (int i = 0; i < 32; ++i) {
+                                        const int rr = wrow0 + i;
+                                        const int nd = c * p.npc + rr / G, hh = rr % G;
+                                        if (rr < rc && nd < n) {
+                                            uint2 o2;
+                                            o2.x = pack_bf16x2(acc[i].x, acc[i].y);
+                                            o2.y = pack_bf16x2(acc[i].z, acc[i].w);
+                                            *reinterpret_cast<uint2 *>(p.out + (((size_t)b * p.Nmax + nd) * p.Hq + g * G + hh) * kHeadDim +
+                                                                       4 * lane) = o2;
+                                        }
+                                    }
+                                } else {
+                                    float Mx = -INFINITY, Ls = 0.f;
+            #pragma unroll 1
                                     for (int cc = c_first; cc <= c_last; ++cc) {
                                         const long long po2 = piece(cc);
                                         if (po2 < 0) continue;
-                                        if (k >= k0 && k < k0 + kn)
-                                            bulk_load_g2s(area + (size_t)(k - k0) * kOB, p.part_o + po2 * RB * kHeadDim, kOB,
-                                                          &misc->stage_bar);
-                                        ++k;
+                                        const float mp = ldcg_f32(p.part_ml + po2 * 2 * RB + r);
+                                        const float lp = ldcg_f32(p.part_ml + po2 * 2 * RB + RB + r);
+                                        if (mp == -INFINITY) continue;
+                                        const float nM = fmaxf(Mx, mp);
+                                        Ls = (Mx == -INFINITY ? 0.f : Ls * ex2(Mx - nM)) + ex2(mp - nM) * lp;
+                                        Mx = nM;
                                     }
-                                }
-                                mbar_wait(&misc->stage_bar, ph);
-                                ph ^= 1u;
-#pragma unroll 1
-                                for (int k = 0; k < kn; ++k) {
-                                    const float *blk = reinterpret_cast<const float *>(area + (size_t)k * kOB);
-                                    const float *wk = sml + (size_t)(k0 + k) * 3 * RB + 2 * RB + wrow0;
-#pragma unroll
-                                    for (int i = 0; i < 32; ++i) {
-                                        const float4 x = *reinterpret_cast<const float4 *>(blk + (size_t)(wrow0 + i) * kHeadDim + 4 * lane);
-                                        const float w = wk[i];
-                                        acc[i].x += w * x.x;
-                                        acc[i].y += w * x.y;
-                                        acc[i].z += w * x.z;
-                                        acc[i].w += w * x.w;
+                                    const float inv = 1.0f / Ls;
+                                    if (r == 0) SPI_TRACE(14);
+                                    __nv_bfloat16 *orow = p.out + (((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim;
+            #pragma unroll 1
+                                    for (int q2 = 0; q2 < 8; ++q2) {   // 16 dims at a time
+                                        float4 a0 = make_float4(0.f, 0.f, 0.f, 0.f), a1 = a0, a2 = a0, a3 = a0;
+            #pragma unroll 1
+                                        for (int cc = c_first; cc <= c_last; ++cc) {
+                                            const long long po2 = piece(cc);
+                                            if (po2 < 0) continue;
+                                            const float mp = ldcg_f32(p.part_ml + po2 * 2 * RB + r);
+                                            const float4 *src = reinterpret_cast<const float4 *>(
+                                                p.part_o + (po2 * RB + r) * kHeadDim + q2 * 16);
+                                            const float4 x0 = __ldcg(src), x1 = __ldcg(src + 1), x2 = __ldcg(src + 2),
+                                                         x3 = __ldcg(src + 3);
+                                            const float w = (mp == -INFINITY) ? 0.f : ex2(mp - Mx) * inv;
+                                            a0.x += w * x0.x; a0.y += w * x0.y; a0.z += w * x0.z; a0.w += w * x0.w;
+                                            a1.x += w * x1.x; a1.y += w * x1.y; a1.z += w * x1.z; a1.w += w * x1.w;
+                                            a2.x += w * x2.x; a2.y += w * x2.y; a2.z += w * x2.z; a2.w += w * x2.w;
+                                            a3.x += w * x3.x; a3.y += w * x3.y; a3.z += w * x3.z; a3.w += w * x3.w;
+                                        }
+                                        if (row_valid) {
+                                            uint4 o4;
+                                            o4.x = pack_bf16x2(a0.x, a0.y);
+                                            o4.y = pack_bf16x2(a0.z, a0.w);
+                                            o4.z = pack_bf16x2(a1.x, a1.y);
+                                            o4.w = pack_bf16x2(a1.z, a1.w);
+                                            *reinterpret_cast<uint4 *>(orow + q2 * 16) = o4;
+                                            o4.x = pack_bf16x2(a2.x, a2.y);
+                                            o4.y = pack_bf16x2(a2.z, a2.w);
+                                            o4.z = pack_bf16x2(a3.x, a3.y);
+                                            o4.w = pack_bf16x2(a3.z, a3.w);
+                                            *reinterpret_cast<uint4 *>(orow + q2 * 16 + 8) = o4;
+                                        }
                                     }
-                                }
-                                named_bar_sync(14, 128);   // the staging area is reused by the next round
-                            }
-                            // rows of this warp: row wrow0 + i -> its node / head (padding rows skipped)
-#pragma unroll
-                            for (int i = 0; i < 32; ++i) {
-                                const int rr = wrow0 + i;
-                                const int nd = c * p.npc + rr / G, hh = rr % G;
-                                if (rr < rc && nd < n) {
-                                    uint2 o2;
-                                    o2.x = pack_bf16x2(acc[i].x, acc[i].y);
-                                    o2.y = pack_bf16x2(acc[i].z, acc[i].w);
-                                    *reinterpret_cast<uint2 *>(p.out + (((size_t)b * p.Nmax + nd) * p.Hq + g * G + hh) * kHeadDim +
-                                                               4 * lane) = o2;
-                                }
-                            }
-                        } else {
-                            float Mx = -INFINITY, Ls = 0.f;
-    #pragma unroll 1
-                            for (int cc = c_first; cc <= c_last; ++cc) {
-                                const long long po2 = piece(cc);
-                                if (po2 < 0) continue;
-                                const float mp = ldcg_f32(p.part_ml + po2 * 2 * RB + r);
-                                const float lp = ldcg_f32(p.part_ml + po2 * 2 * RB + RB + r);
-                                if (mp == -INFINITY) continue;
-                                const float nM = fmaxf(Mx, mp);
-                                Ls = (Mx == -INFINITY ? 0.f : Ls * ex2(Mx - nM)) + ex2(mp - nM) * lp;
-                                Mx = nM;
-                            }
-                            const float inv = 1.0f / Ls;
-                            if (r == 0) SPI_TRACE(14);
-                            __nv_bfloat16 *orow = p.out + (((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim;
-    #pragma unroll 1
-                            for (int q2 = 0; q2 < 8; ++q2) {   // 16 dims at a time
-                                float4 a0 = make_float4(0.f, 0.f, 0.f, 0.f), a1 = a0, a2 = a0, a3 = a0;
-    #pragma unroll 1
-                                for (int cc = c_first; cc <= c_last; ++cc) {
-                                    const long long po2 = piece(cc);
-                                    if (po2 < 0) continue;
-                                    const float mp = ldcg_f32(p.part_ml + po2 * 2 * RB + r);
-                                    const float4 *src = reinterpret_cast<const float4 *>(
-                                        p.part_o + (po2 * RB + r) * kHeadDim + q2 * 16);
-                                    const float4 x0 = __ldcg(src), x1 = __ldcg(src + 1), x2 = __ldcg(src + 2),
-                                                 x3 = __ldcg(src + 3);
-                                    const float w = (mp == -INFINITY) ? 0.f : ex2(mp - Mx) * inv;
-                                    a0.x += w * x0.x; a0.y += w * x0.y; a0.z += w * x0.z; a0.w += w * x0.w;
-                                    a1.x += w * x1.x; a1.y += w * x1.y; a1.z += w * x1.z; a1.w += w * x1.w;
-                                    a2.x += w * x2.x; a2.y += w * x2.y; a2.z += w * x2.z; a2.w += w * x2.w;
-                                    a3.x += w * x3.x; a3.y += w * x3.y; a3.z += w * x3.z; a3.w += w * x3.w;
-                                }
-                                if (row_valid) {
-                                    uint4 o4;
-                                    o4.x = pack_bf16x2(a0.x, a0.y);
-                                    o4.y = pack_bf16x2(a0.z, a0.w);
-                                    o4.z = pack_bf16x2(a1.x, a1.y);
-                                    o4.w = pack_bf16x2(a1.z, a1.w);
-                                    *reinterpret_cast<uint4 *>(orow + q2 * 16) = o4;
-                                    o4.x = pack_bf16x2(a2.x, a2.y);
-                                    o4.y = pack_bf16x2(a2.z, a2.w);
-                                    o4.z = pack_bf16x2(a3.x, a3.y);
-                                    o4.w = pack_bf16x2(a3.z, a3.w);
-                                    *reinterpret_cast<uint4 *>(orow + q2 * 16 + 8) = o4;
                                 }
                             }
                         }
+                        if (r == 0) SPI_TRACE(11);
                     }
+                    ++ls;
                 }
-                if (r == 0) SPI_TRACE(11);
-            }
-            ++ls;
+                // the last tile's decision has no next owner: consume it so every barrier phase completes
+                if (lt > 0 && ((lt - 1) & 1) != grp) named_bar_sync(dec_in, 64);
         }
-        // the last tile's decision has no next owner: consume it so every barrier phase completes
-        if (lt > 0 && ((lt - 1) & 1) != grp) named_bar_sync(dec_in, 64);
     }
 
     tc_fence_before();
     __syncthreads();
-    if (warp == 1) {
+    if (warp == kWarpS) {
         tc_fence_after();
         tmem_dealloc<kTmemCols>(tmem);
     }
@@ -887,7 +895,7 @@ cudaError_t launch_tree_attention_rows(const AttnParams &prm0, const void *q, co
     }
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(num_ctas);
-    cfg.blockDim = dim3(352);
+    cfg.blockDim = dim3(rows::kThreads);
     cfg.dynamicSmemBytes = smem;
     cfg.stream = stream;
     cudaLaunchAttribute attr[1];
