@@ -4,18 +4,21 @@
 //  * a work item is (request, kv-head, block of 128 query rows); the UMMA M dimension is the query
 //    rows (one TMEM lane per row), N = 128 keys for S = Q K^T and N = 128 dims for O += P V;
 //  * TMEM = S0 | S1 | O | P0 | P1 (128 + 128 + 128 + 64 + 64 columns): S double-buffered, ONE O
-//    accumulator, P (bf16 pairs) in its own columns, so the S buffer of tile t is free as soon as
-//    the softmax has loaded it and S(t + 2) never waits for PV(t) (round 1 aliased P over S and the
-//    chain S -> softmax -> PV -> S(t + 2) bounded the kernel);
+//    accumulator, P (bf16 pairs) in its own columns.  The softmax reads a tile's 128 scores per row
+//    into registers ONCE and releases the S buffer right there, so S(t + 2) is issued while tile t's
+//    softmax runs (round 1 aliased P over S: S -> softmax -> PV -> S(t + 2) was one chain);
 //  * 8 softmax warps in two groups of 4 (one warp per TMEM lane quarter each, thread = query row);
 //    group g owns the tiles with t & 1 == g and both accumulate into the one O, so every P(t) uses
 //    the row reference the previous tile left: the owner of tile t reads decision(t - 1) from the
 //    other group (shared memory + one named barrier per direction and lane quarter), may raise it
 //    (stale max: only beyond 2^8, then O is rescaled in TMEM after PV(t - 1)), publishes decision(t)
-//    and only then computes its exponentials -- the groups run out of phase;
+//    and only then computes its exponentials into registers; only their TMEM store waits for PV(t - 2)
+//    to have released the P buffer -- the groups run out of phase;
 //  * segment end: the owner of the last tile combines both groups' row sums, then both groups write
 //    half of the output row each (a whole item) or the owner writes the fp32 partial (a split piece);
-//  * K and V in separate TMA rings fed by two producer lanes; S issuer and PV issuer threads;
+//  * K and V in separate TMA rings fed by two producer warps; S issuer and PV issuer threads;
+//  * warpgroups: 0-1 softmax, 2 control (producers, issuers); setmaxnreg moves registers from the
+//    control warpgroup (56 per thread) to the softmax warpgroups (224: the scores stay in registers);
 //  * lane mode (schedule_kernel): the row blocks of one (request, kv-head) run on `lanes` CTAs in
 //    lock-step over the same tile range, so each KV tile is read from HBM once;
 //  * tree keys are masked with the ancestor-or-self bitset of the row's node (tree_prepare);
@@ -31,11 +34,11 @@ constexpr int RB = kRowsBlock;              // 128 query rows per item
 constexpr int kQBuf = 2 * RB * 128;          // one Q buffer: 2 halves x 128 rows x 128 B
 constexpr int kTmemCols = 512;
 constexpr int kColS = 0, kColO = 256, kColP = 384;
-// warp roles: 0-7 softmax / epilogue (two groups of 4, warp & 3 = TMEM lane quarter), 8 TMA producers,
-// 9 S issuer (+ TMEM allocation), 10 PV issuer, 11 idle.  The control warpgroup (8-11) gives registers
+// warp roles: 0-7 softmax / epilogue (two groups of 4, warp & 3 = TMEM lane quarter), 8 Q / K producer,
+// 9 S issuer (+ TMEM allocation), 10 PV issuer, 11 V producer.  The control warpgroup (8-11) gives registers
 // to the softmax warpgroups (setmaxnreg): 168 per thread at launch -> 56 / 224
 constexpr int kThreads = 384;
-constexpr int kWarpProd = 8, kWarpS = 9, kWarpPV = 10;
+constexpr int kWarpProd = 8, kWarpS = 9, kWarpPV = 10, kWarpV = 11;
 constexpr int kRegsCtl = 56, kRegsSoftmax = 224;
 constexpr int kMaxK = 4, kMaxV = 4;          // ring slots (the launch picks 3 K + 2 V)
 
@@ -249,7 +252,7 @@ __global__ void __maxnreg__(168)
 
     // Programmatic dependent launch (see tree_attention.cu): the producer warp may stage
     // committed-prefix tiles of its first segment before the dependency resolves (early_prefix)
-    const bool early = p.early_prefix != 0 && warp == kWarpProd;
+    const bool early = p.early_prefix != 0 && (warp == kWarpProd || warp == kWarpV);
     if (!early) grid_dependency_wait();
     const int4 ci = __ldg(p.cta_info + 2 * blockIdx.x);
     const int4 first_info = __ldg(p.cta_info + 2 * blockIdx.x + 1);
@@ -262,9 +265,9 @@ __global__ void __maxnreg__(168)
         setmaxnreg_dec<kRegsCtl>();
         if (ntiles <= 0) {
             if (early) grid_dependency_wait();
-        } else if (warp == kWarpProd) {
+        } else if (warp == kWarpProd || warp == kWarpV) {
             // ============================ TMA producers ============================
-            // lane 0: segment descriptors, Q and the K ring; lane 1: the V ring (follows the descriptors)
+            // warp 8: segment descriptors, Q and the K ring; warp 11: the V ring (follows the descriptors)
             const uint64_t pol = p.lanes > 1 ? l2_evict_normal_policy() : l2_evict_first_policy();
             auto issue = [&](const SegDesc &d, int t, int lt, bool is_v) {
                 const int key0 = (t - d.ib) * kKeyTile;
@@ -299,7 +302,7 @@ __global__ void __maxnreg__(168)
                 while (c < NS && d.begin + c < d.end && (d.begin + c - d.ib + 1) * kKeyTile <= d.P) ++c;
                 return c;
             };
-            if (lane == 0) {
+            if (warp == kWarpProd && lane == 0) {
                 int x = x_first, ls = 0, lt = 0;
                 int4 next_info = first_info;
                 for (;;) {
@@ -349,7 +352,7 @@ __global__ void __maxnreg__(168)
                     ++ls;
                 }
                 grid_launch_dependents();
-            } else if (lane == 1) {
+            } else if (warp == kWarpV && lane == 0) {
                 int ls = 0, lt = 0;
                 for (;;) {
                     mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
@@ -502,7 +505,7 @@ __global__ void __maxnreg__(168)
                         uint32_t vis[4] = {0xFFFFFFFFu, 0xFFFFFFFFu, 0xFFFFFFFFu, 0xFFFFFFFFu};
                         const bool masked = key0 + kKeyTile > P;
                         if (masked) {
-        #pragma unroll
+#pragma unroll
                             for (int q = 0; q < 4; ++q) {
                                 const int j0 = key0 + 32 * q - P;  // tree index of the group's first key
                                 if (j0 + 32 > 0) {
@@ -520,16 +523,20 @@ __global__ void __maxnreg__(168)
                         }
                         // pass 1: this row's tile max
                         float tm;
-                        uint32_t sv[4][32];   // the row's scores stay in registers for pass 2 (chunk 0 is reloaded there)
+                        uint32_t sv[4][32];   // the row's 128 scores stay in registers for pass 2
                         {
                             float m4[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
-        #pragma unroll
+#pragma unroll
                             for (int q = 0; q < 4; ++q) tmem_ld32(s_col + q * 32, sv[q]);
                             tmem_ld_wait();
-        #pragma unroll
+                            // S buffer t & 1 is free now: S(t + 2) may overwrite it while this tile's softmax runs
+                            tc_fence_before();
+                            __syncwarp();
+                            if (lane == 0) mbar_arrive(&misc->s_free[sb]);
+#pragma unroll
                             for (int q = 0; q < 4; ++q) {
                                 if (masked) rows::mask32(sv[q], vis[q]);
-        #pragma unroll
+#pragma unroll
                                 for (int i = 0; i < 32; ++i) m4[i & 3] = fmaxf(m4[i & 3], __uint_as_float(sv[q][i]));
                             }
                             tm = fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3])) * p.scale_log2;
@@ -560,15 +567,15 @@ __global__ void __maxnreg__(168)
                             if (lt >= 2) mbar_wait(&misc->pv_done[lt & 1], ((lt - 2) >> 1) & 1);
                             mbar_wait(&misc->pv_done[(lt - 1) & 1], ((lt - 1) >> 1) & 1);
                             tc_fence_after();
-        #pragma unroll 1
+#pragma unroll 1
                             for (int q2 = 0; q2 < 4; ++q2) {
                                 uint32_t v[32];
                                 tmem_ld32(o_col + q2 * 32, v);
                                 tmem_ld_wait();
                                 uint32_t w16[16];
-        #pragma unroll
+#pragma unroll
                                 for (int hh = 0; hh < 2; ++hh) {
-        #pragma unroll
+#pragma unroll
                                     for (int i = 0; i < 16; ++i) w16[i] = __float_as_uint(__uint_as_float(v[hh * 16 + i]) * alpha);
                                     tmem_st16(o_col + q2 * 32 + hh * 16, w16);
                                 }
@@ -584,23 +591,15 @@ __global__ void __maxnreg__(168)
                             const uint64_t sc2 = f2_bits(p.scale_log2, p.scale_log2), nm2 = f2_bits(-mref, -mref);
                             const uint32_t p_col = tmem + kColP + sb * 64 + lane_off;
                             float ls2 = 0.f;
-                            // chunk 0 of the scores was not kept across the decision (register pressure): reload it,
-                            // then the S buffer is free
-                            tmem_ld32(s_col, sv[0]);
-                            tmem_ld_wait();
-                            tc_fence_before();
-                            __syncwarp();
-                            if (lane == 0) mbar_arrive(&misc->s_free[sb]);
-                            if (masked) rows::mask32(sv[0], vis[0]);
                             uint32_t w16[4][16];
-        #pragma unroll
+#pragma unroll
                             for (int q = 0; q < 4; ++q) {
                                 float dummy = 0.f;
                                 ls2 += rows::exp32<false>(sv[q], sc2, nm2, w16[q], dummy);
                             }
                             if (lt >= 2) mbar_wait(&misc->pv_done[sb], ((lt - 2) >> 1) & 1);
                             tc_fence_after();
-        #pragma unroll
+#pragma unroll
                             for (int q = 0; q < 4; ++q) tmem_st16(p_col + q * 16, w16[q]);
                             l += (SPI_FLAGS(p) & 8) ? 1.f : ls2;
                         }
@@ -665,12 +664,12 @@ __global__ void __maxnreg__(168)
                             // merges every piece by log-sum-exp
                             const int slot = (sd.begin == t0) ? 0 : 1;
                             float *po = p.part_o + (((size_t)blockIdx.x * 2 + slot) * RB + r) * kHeadDim;
-        #pragma unroll 1
+#pragma unroll 1
                             for (int q2 = 0; q2 < 4; ++q2) {
                                 uint32_t o[32];
                                 tmem_ld32(o_col + q2 * 32, o);
                                 tmem_ld_wait();
-        #pragma unroll
+#pragma unroll
                                 for (int i = 0; i < 32; i += 8)   // 32-byte stores (part_o rows are 512-byte aligned)
                                     asm volatile("st.global.v8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"l"(po + q2 * 32 + i),
                                                  "r"(o[i]), "r"(o[i + 1]), "r"(o[i + 2]), "r"(o[i + 3]), "r"(o[i + 4]),
@@ -748,7 +747,7 @@ __global__ void __maxnreg__(168)
                                     for (int k = 0; k < npc; ++k) sml[(size_t)k * 3 * RB + 2 * RB + r] *= inv;
                                     named_bar_sync(14, 128);   // weights visible to the whole group
                                     float4 acc[32];   // [row of the warp] lane's 4 dims
-        #pragma unroll
+#pragma unroll
                                     for (int i = 0; i < 32; ++i) acc[i] = make_float4(0.f, 0.f, 0.f, 0.f);
                                     const int wrow0 = qd * 32;   // this warp's rows
                                     for (int k0 = 0; k0 < npc; k0 += cap) {
@@ -767,11 +766,11 @@ __global__ void __maxnreg__(168)
                                         }
                                         mbar_wait(&misc->stage_bar, ph);
                                         ph ^= 1u;
-        #pragma unroll 1
+#pragma unroll 1
                                         for (int k = 0; k < kn; ++k) {
                                             const float *blk = reinterpret_cast<const float *>(area + (size_t)k * kOB);
                                             const float *wk = sml + (size_t)(k0 + k) * 3 * RB + 2 * RB + wrow0;
-        #pragma unroll
+#pragma unroll
                                             for (int i = 0; i < 32; ++i) {
                                                 const float4 x = *reinterpret_cast<const float4 *>(blk + (size_t)(wrow0 + i) * kHeadDim + 4 * lane);
                                                 const float w = wk[i];
@@ -784,7 +783,7 @@ __global__ void __maxnreg__(168)
                                         named_bar_sync(14, 128);   // the staging area is reused by the next round
                                     }
                                     // rows of this warp: row wrow0 + i -> its node / head (padding rows skipped)
-        #pragma unroll
+#pragma unroll
                                     for (int i = 0; i < 32; ++i) {
                                         const int rr = wrow0 + i;
                                         const int nd = c * p.npc + rr / G, hh = rr % G;
@@ -798,7 +797,7 @@ __global__ void __maxnreg__(168)
                                     }
                                 } else {
                                     float Mx = -INFINITY, Ls = 0.f;
-            #pragma unroll 1
+    #pragma unroll 1
                                     for (int cc = c_first; cc <= c_last; ++cc) {
                                         const long long po2 = piece(cc);
                                         if (po2 < 0) continue;
@@ -812,10 +811,10 @@ __global__ void __maxnreg__(168)
                                     const float inv = 1.0f / Ls;
                                     if (r == 0) SPI_TRACE(14);
                                     __nv_bfloat16 *orow = p.out + (((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim;
-            #pragma unroll 1
+    #pragma unroll 1
                                     for (int q2 = 0; q2 < 8; ++q2) {   // 16 dims at a time
                                         float4 a0 = make_float4(0.f, 0.f, 0.f, 0.f), a1 = a0, a2 = a0, a3 = a0;
-            #pragma unroll 1
+    #pragma unroll 1
                                         for (int cc = c_first; cc <= c_last; ++cc) {
                                             const long long po2 = piece(cc);
                                             if (po2 < 0) continue;
