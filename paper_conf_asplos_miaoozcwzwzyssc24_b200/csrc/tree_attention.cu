@@ -13,7 +13,7 @@
 //    last piece to finish merges them (log-sum-exp): one launch per layer, no tail wave.
 //  * Each KV tile is read from HBM once by TMA (128B-swizzled 16 KB boxes) and shared by ALL
 //    G*n_b query rows of the kv-head.  K and V have separate smem rings (K tiles are released
-//    right after S = K Q^T, so K prefetch never waits for a PV), fed by two producer lanes.
+//    right after S = K Q^T, so K prefetch never waits for a PV), fed by two producer warps.
 //  * "Swapped" tensor-core formulation for few query rows: S^T = K Q^T (UMMA M = 128 keys,
 //    N = NT query rows, K = 128 dims) and O^T += V^T P^T (M = 128 dims, N = NT, K = 128 keys);
 //    tcgen05.mma kind::f16 issued by one thread, fp32 accumulators in TMEM.
@@ -24,7 +24,7 @@
 //    recomputed exactly and O^T is rescaled in TMEM (the rare path).
 //  * Segment metadata is decoded once by the producer and passed through an smem ring, so no
 //    consumer waits on a global load at item boundaries.
-//  * warp 0: TMA producers (lane 0: Q + K + segment ring, lane 1: V); warp 1: TMEM allocator +
+//  * warp 0: Q + K + segment ring producer; last warp: V producer; warp 1: TMEM allocator +
 //    MMA issuer; warps 2-5: softmax / epilogue / split combine.
 #include "attn_shared.cuh"
 
@@ -68,8 +68,19 @@ struct SmemMisc {
     int32_t npieces;
 };
 
+// warp roles: 0 Q / K producer, 1 S issuer (+ TMEM allocation), 2 PV issuer, 3 .. 3 + kSoft / 32 - 1
+// softmax / epilogue, last: V producer (its own warp: as a second lane of warp 0, a lane spinning on
+// one ring's empty barrier held the other ring's lane at the warp's divergence point -- at batch 2
+// K and V loads were issued 1-2K cycles after their slots freed)
 template <int NT>
-__global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
+struct SwRoles {
+    static constexpr int kSoftWarps = NT >= 32 ? 8 : 4;
+    static constexpr int kWarpV = 3 + kSoftWarps;
+    static constexpr int kThreads = 32 * (kWarpV + 1);
+};
+
+template <int NT>
+__global__ void __launch_bounds__(SwRoles<NT>::kThreads, 1)
     tree_attn_kernel(const __grid_constant__ CUtensorMap tm_q, const __grid_constant__ CUtensorMap tm_k,
                      const __grid_constant__ CUtensorMap tm_v, const __grid_constant__ CUtensorMap tm_k16,
                      const __grid_constant__ CUtensorMap tm_v16, const __grid_constant__ CUtensorMap tm_k4,
@@ -130,7 +141,9 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
         tma_prefetch_desc(&tm_k1);
         tma_prefetch_desc(&tm_v1);
     }
-    if (warp >= 3) {
+    constexpr int kWarpV = SwRoles<NT>::kWarpV;
+    const bool softw = warp >= 3 && warp < kWarpV;   // softmax / epilogue warp
+    if (softw) {
         // Q rows beyond a chunk's G*npc rows are never written by TMA: keep them zero
         for (int i = threadIdx.x - 96; i < Plan::kNQ * Plan::kQBuf / 16; i += kSoft)
             reinterpret_cast<uint4 *>(s_q)[i] = make_uint4(0, 0, 0, 0);
@@ -150,11 +163,11 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
     // Programmatic dependent launch: everything above overlapped the previous kernel's tail;
     // from here on we read inputs it may have produced.  With early_prefix (the caller guarantees
     // that neither the committed prefix of the caches nor the schedule in the workspace was written
-    // by the immediately preceding kernel), the two producer lanes first stage the committed-prefix
+    // by the immediately preceding kernel), the two producer threads first stage the committed-prefix
     // tiles of their first segment and only then wait; every other warp waits here.
-    // (the whole producer warp skips this wait: a wait on lanes 2-31 alone would hold lanes 0-1 at the
-    // warp's reconvergence point; lanes 0-1 wait after staging, lanes 2-31 read nothing)
-    const bool early = p.early_prefix != 0 && warp == 0;
+    // (the whole producer warps skip this wait: a wait on lanes 1-31 alone would hold lane 0 at the
+    // warp's reconvergence point; lane 0 waits after staging, lanes 1-31 read nothing)
+    const bool early = p.early_prefix != 0 && (warp == 0 || warp == kWarpV);
     if (!early) grid_dependency_wait();
     if (threadIdx.x == 0) SPI_TRACE_K(5);
     // this CTA's slice of the tile sequence (precomputed by tree_prepare for this grid)
@@ -167,10 +180,10 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
     if (ntiles <= 0) {
         // no work for this CTA (fewer tiles than CTAs)
         if (early) grid_dependency_wait();
-    } else if (warp == 0) {
+    } else if (warp == 0 || warp == kWarpV) {
         // ============================ TMA producers ============================
         const uint64_t pol = l2_evict_first_policy();
-        // one K (lane 0) or V (lane 1) tile of segment d into ring slot lt % NS
+        // one K (warp 0) or V (V warp) tile of segment d into ring slot lt % NS
         auto issue = [&](const SegDesc &d, int t, int lt, bool is_v) {
             const int key0 = (t - d.ib) * kKeyTile;
             const int nv = min(kKeyTile, d.P + d.n - key0);
@@ -205,7 +218,7 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
             while (c < NS && d.begin + c < d.end && (d.begin + c - d.ib + 1) * kKeyTile <= d.P) ++c;
             return c;
         };
-        if (lane == 0) {
+        if (warp == 0 && lane == 0) {
             // segment descriptors for every role, Q, and the K tiles
             int lt = 0, ls = 0;
             int4 next_info = first_info;
@@ -248,8 +261,8 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
                 ++ls;
             }
             grid_launch_dependents();  // all of this CTA's K loads are issued
-        } else if (lane == 1) {
-            // V tiles, following the segment ring written by lane 0
+        } else if (warp == kWarpV && lane == 0) {
+            // V tiles, following the segment ring written by warp 0
             int lt = 0, ls = 0;
             while (lt < ntiles) {
                 mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
@@ -331,7 +344,7 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
                 ++ls;
             }
         }
-    } else {
+    } else if (softw) {
         // ======================= softmax / epilogue warps =======================
         const int st = threadIdx.x - 96;       // 0..kSoft-1
         const int half = st >> 7;              // which half of the query rows (kSplit = 2)
@@ -790,7 +803,7 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
         }
     }
 
-    if (warp >= 3) bulk_wait_all();  // output bulk stores complete before smem goes away
+    if (softw) bulk_wait_all();  // output bulk stores complete before smem goes away
     tc_fence_before();
     __syncthreads();
     if (p.splitk > 1) {
@@ -818,7 +831,7 @@ __global__ void __launch_bounds__(NT >= 32 ? 352 : 224, 1)
         const int x = blockIdx.x / K;
         const int4 info = __ldg(p.item_info + x);
         const bool whole = t0 == info.x && t1 == info.y;  // rank 0 streamed (and wrote) the whole item
-        if (rank == 0 && warp >= 3 && !whole && info.y > info.x) {
+        if (rank == 0 && softw && !whole && info.y > info.x) {
             const int st = threadIdx.x - 96;
             const int r0 = (st >> 7) * NTH;
             const int d = (warp & 3) * 32 + lane;
@@ -919,7 +932,7 @@ static cudaError_t launch_nt(const AttnParams &prm0, const void *q, const void *
     // this grid overlaps the tail of the previous kernel on the stream
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(num_sms);  // (the caller's grid: w.grid)
-    cfg.blockDim = dim3(NT >= 32 ? 352 : 224);
+    cfg.blockDim = dim3(SwRoles<NT>::kThreads);
     cfg.dynamicSmemBytes = smem;
     cfg.stream = stream;
     cudaLaunchAttribute attr[2];

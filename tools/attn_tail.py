@@ -45,6 +45,13 @@ t0 = kt[:, 0].min()
 ex = (kt[:, 1] - t0) / 1e3
 fk = np.where(kt[:, 2] > 0, (kt[:, 2] - t0) / 1e3, -1)
 order = np.argsort(ex)
+names = ["entry", "exit", "first K issue", "cluster barrier", "prologue done", "dependency wait passed",
+         "schedule read", "first S ready"]
+for k in [0, 4, 5, 6, 2, 7, 3, 1]:
+    v = kt[:, k]
+    v = v[v > 0]
+    if len(v):
+        print(f"  {names[k]:24s} us p0/p50/p100: {np.percentile((v - t0) / 1e3, [0, 50, 100]).round(2)}")
 print("exit us percentiles 0/25/50/75/90/100:", np.percentile(ex, [0, 25, 50, 75, 90, 100]).round(2))
 print("latest 12 CTAs (cta, entry, firstK, exit):")
 for c in order[-12:]:
