@@ -24,8 +24,8 @@
 //    recomputed exactly and O^T is rescaled in TMEM (the rare path).
 //  * Segment metadata is decoded once by the producer and passed through an smem ring, so no
 //    consumer waits on a global load at item boundaries.
-//  * warp 0: Q + K + segment ring producer; last warp: V producer; warp 1: TMEM allocator +
-//    MMA issuer; warps 2-5: softmax / epilogue / split combine.
+//  * warp 0: Q + K + segment ring producer; warp 1: TMEM allocator + S issuer; warp 2: PV issuer;
+//    warps 3 .. (8 at NT >= 32, 4 at NT = 16): softmax / epilogue / split combine; last warp: V producer.
 #include "attn_shared.cuh"
 
 #include <cooperative_groups.h>
