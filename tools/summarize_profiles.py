@@ -86,30 +86,32 @@ if os.path.exists(raw_csv):
     old.update(traffic)
     json.dump(old, open(path, "w"), indent=1)
 
-rows_csv = os.path.join(OUT, f"rows_full_C3_{R}_raw.csv")
-if os.path.exists(rows_csv):
-    raw = read_raw(rows_csv)
-    keys = ["gpu__time_duration.sum", "sm__cycles_elapsed.avg.per_second", "dram__bytes_read.sum",
-            "dram__bytes_write.sum", "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_active",
-            "sm__inst_executed_pipe_xu.avg.pct_of_peak_sustained_active",
-            "sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active",
-            "smsp__issue_active.avg.pct_of_peak_sustained_active", "launch__registers_per_thread",
-            "launch__grid_size", "launch__block_size"]
-    lines += ["## tree_attn_rows_kernel, `ncu --set full` (C3 shape, one launch = one layer)", "",
-              "| metric | value |", "|---|---|"]
-    for k in keys:
-        if k in raw:
-            lines.append(f"| `{k}` | {raw[k][0]} {raw[k][1]} |")
-    def to_bytes(v, u):
-        return float(v.replace(",", "")) * {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}[u]
-    rd, wr = to_bytes(*raw["dram__bytes_read.sum"]), to_bytes(*raw["dram__bytes_write.sum"])
-    alg = 612368384   # C3: K and V of 32 x 8 (request, kv-head) streams of 4096 + 64 rows, q in, out
-    lines += ["", f"DRAM traffic per launch {rd + wr:,.0f} B vs algorithmic {alg:,} B (ratio {(rd + wr) / alg:.3f}).", ""]
-    path = os.path.join(PROF, "ncu_traffic.json")
-    old = json.load(open(path)) if os.path.exists(path) else {}
-    old["C3"] = {"dram_bytes_per_launch": int(rd + wr), "round": R,
-                 "source": f"gpurun_out/rows_full_C3_{R}.ncu-rep (ncu --set full)"}
-    json.dump(old, open(path, "w"), indent=1)
+for cfg_name, alg in (("C3", 612368384), ("C4", 2734161920)):
+  # C3: K and V of 32 x 8 (request, kv-head) streams of 4096 + 64 rows, q in, out;
+  # C4: 64 x 56 streams of 1024 + 233 rows, q in, out (bench.py's algorithmic_bytes_per_launch)
+  rows_csv = os.path.join(OUT, f"rows_full_{cfg_name}_{R}_raw.csv")
+  if os.path.exists(rows_csv):
+      raw = read_raw(rows_csv)
+      keys = ["gpu__time_duration.sum", "sm__cycles_elapsed.avg.per_second", "dram__bytes_read.sum",
+              "dram__bytes_write.sum", "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_active",
+              "sm__inst_executed_pipe_xu.avg.pct_of_peak_sustained_active",
+              "sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active",
+              "smsp__issue_active.avg.pct_of_peak_sustained_active", "launch__registers_per_thread",
+              "launch__grid_size", "launch__block_size"]
+      lines += [f"## tree_attn_rows_kernel, `ncu --set full` ({cfg_name} shape, one launch = one layer)", "",
+                "| metric | value |", "|---|---|"]
+      for k in keys:
+          if k in raw:
+              lines.append(f"| `{k}` | {raw[k][0]} {raw[k][1]} |")
+      def to_bytes(v, u):
+          return float(v.replace(",", "")) * {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}[u]
+      rd, wr = to_bytes(*raw["dram__bytes_read.sum"]), to_bytes(*raw["dram__bytes_write.sum"])
+      lines += ["", f"DRAM traffic per launch {rd + wr:,.0f} B vs algorithmic {alg:,} B (ratio {(rd + wr) / alg:.3f}).", ""]
+      path = os.path.join(PROF, "ncu_traffic.json")
+      old = json.load(open(path)) if os.path.exists(path) else {}
+      old[cfg_name] = {"dram_bytes_per_launch": int(rd + wr), "round": R,
+                   "source": f"gpurun_out/rows_full_{cfg_name}_{R}.ncu-rep (ncu --set full)"}
+      json.dump(old, open(path, "w"), indent=1)
 
 det_lines = []
 for k in ("verify_mss", "verify_greedy", "kv_commit", "tree_validate", "gather_wait"):
