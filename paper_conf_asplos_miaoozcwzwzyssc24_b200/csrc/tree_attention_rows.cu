@@ -141,13 +141,23 @@ __device__ __forceinline__ uint64_t exp2_poly2(uint64_t x2) {
     return (uint64_t)((uint32_t)q + (n0 << 23)) | ((uint64_t)((uint32_t)(q >> 32) + (n1 << 23)) << 32);
 }
 
+// acc + float(bf16 half of w), one instruction (sm_100 mixed-precision add reads the half in place)
+__device__ __forceinline__ float add_bf16lo(uint32_t w, float acc) {
+    asm("{\n\t.reg .b16 lo, hi;\n\tmov.b32 {lo, hi}, %1;\n\tadd.rn.f32.bf16 %0, lo, %0;\n\t}" : "+f"(acc) : "r"(w));
+    return acc;
+}
+__device__ __forceinline__ float add_bf16hi(uint32_t w, float acc) {
+    asm("{\n\t.reg .b16 lo, hi;\n\tmov.b32 {lo, hi}, %1;\n\tadd.rn.f32.bf16 %0, hi, %0;\n\t}" : "+f"(acc) : "r"(w));
+    return acc;
+}
+
 // P = 2^(s * scale_log2 - mref) of 32 keys as 16 bf16 pairs (into w, not yet stored); returns the fp32
 // sum of the bf16-ROUNDED values, so the normalisation matches the numerator the PV MMA computes.
 // kMax: also the max of the (raw) s values, for the deferred stale-max check.
 template <bool kMax>
 __device__ __forceinline__ float exp32(const uint32_t (&v)[32], uint64_t sc2, uint64_t nm2, uint32_t (&w)[16],
                                        float &pm) {
-    uint64_t la = f2_bits(0.f, 0.f), lb = f2_bits(0.f, 0.f);
+    float acc[4] = {0.f, 0.f, 0.f, 0.f};
     float m2[2] = {-INFINITY, -INFINITY};
 #pragma unroll
     for (int i = 0; i < 16; ++i) {
@@ -167,13 +177,12 @@ __device__ __forceinline__ float exp32(const uint32_t (&v)[32], uint64_t sc2, ui
             e1 = ex2(__uint_as_float((uint32_t)(y >> 32)));
         }
         w[i] = pack_bf16x2(e0, e1);
-        const uint64_t r2 = f2_bits(__uint_as_float(w[i] << 16), __uint_as_float(w[i] & 0xFFFF0000u));
-        if (i & 1) lb = fadd2(lb, r2);
-        else la = fadd2(la, r2);
+        // row sum of the rounded values: the bf16 halves added in place (no unpacking)
+        acc[2 * (i & 1)] = add_bf16lo(w[i], acc[2 * (i & 1)]);
+        acc[2 * (i & 1) + 1] = add_bf16hi(w[i], acc[2 * (i & 1) + 1]);
     }
     if (kMax) pm = fmaxf(pm, fmaxf(m2[0], m2[1]));
-    const uint64_t s = fadd2(la, lb);
-    return __uint_as_float((uint32_t)s) + __uint_as_float((uint32_t)(s >> 32));
+    return (acc[0] + acc[1]) + (acc[2] + acc[3]);
 }
 
 // masks 32 S values in place (invisible -> -inf)
