@@ -491,8 +491,8 @@ __global__ void __launch_bounds__(SwRoles<NT>::kThreads, 1)
 #pragma unroll
                 for (int i = 0; i < NTH / 2; ++i) {
                     pk[i] = pack_bf16x2(xv[2 * i], xv[2 * i + 1]);
-                    lsum[2 * i] += __uint_as_float(pk[i] << 16);
-                    lsum[2 * i + 1] += __uint_as_float(pk[i] & 0xFFFF0000u);
+                    lsum[2 * i] = add_bf16lo(pk[i], lsum[2 * i]);       // the bf16 halves added in place
+                    lsum[2 * i + 1] = add_bf16hi(pk[i], lsum[2 * i + 1]);
                 }
                 // ---- P^T row (this key) into smem as bf16, MN-major + swizzle ----
                 if (lt >= Plan::kNP)  // PV(t - kNP) has read this buffer

@@ -141,16 +141,6 @@ __device__ __forceinline__ uint64_t exp2_poly2(uint64_t x2) {
     return (uint64_t)((uint32_t)q + (n0 << 23)) | ((uint64_t)((uint32_t)(q >> 32) + (n1 << 23)) << 32);
 }
 
-// acc + float(bf16 half of w), one instruction (sm_100 mixed-precision add reads the half in place)
-__device__ __forceinline__ float add_bf16lo(uint32_t w, float acc) {
-    asm("{\n\t.reg .b16 lo, hi;\n\tmov.b32 {lo, hi}, %1;\n\tadd.rn.f32.bf16 %0, lo, %0;\n\t}" : "+f"(acc) : "r"(w));
-    return acc;
-}
-__device__ __forceinline__ float add_bf16hi(uint32_t w, float acc) {
-    asm("{\n\t.reg .b16 lo, hi;\n\tmov.b32 {lo, hi}, %1;\n\tadd.rn.f32.bf16 %0, hi, %0;\n\t}" : "+f"(acc) : "r"(w));
-    return acc;
-}
-
 // P = 2^(s * scale_log2 - mref) of 32 keys as 16 bf16 pairs (into w, not yet stored); returns the fp32
 // sum of the bf16-ROUNDED values, so the normalisation matches the numerator the PV MMA computes.
 // kMax: also the max of the (raw) s values, for the deferred stale-max check.
