@@ -394,6 +394,16 @@ __device__ __forceinline__ uint32_t pack_bf16x2(float lo, float hi) {
     return *reinterpret_cast<uint32_t *>(&v);
 }
 
+// acc + float(bf16 half of w), one instruction (sm_100 mixed-precision add reads the half in place)
+__device__ __forceinline__ float add_bf16lo(uint32_t w, float acc) {
+    asm("{\n\t.reg .b16 lo, hi;\n\tmov.b32 {lo, hi}, %1;\n\tadd.rn.f32.bf16 %0, lo, %0;\n\t}" : "+f"(acc) : "r"(w));
+    return acc;
+}
+__device__ __forceinline__ float add_bf16hi(uint32_t w, float acc) {
+    asm("{\n\t.reg .b16 lo, hi;\n\tmov.b32 {lo, hi}, %1;\n\tadd.rn.f32.bf16 %0, hi, %0;\n\t}" : "+f"(acc) : "r"(w));
+    return acc;
+}
+
 __device__ __forceinline__ float ldcg_f32(const float *p) { return __ldcg(p); }
 
 }  // namespace specinfer
