@@ -14,11 +14,15 @@
 //    (stale max: only beyond 2^8, then O is rescaled in TMEM after PV(t - 1)), publishes decision(t)
 //    and only then computes its exponentials into registers; only their TMEM store waits for PV(t - 2)
 //    to have released the P buffer -- the groups run out of phase;
-//  * segment end: the owner of the last tile combines both groups' row sums, then both groups write
-//    half of the output row each (a whole item) or the owner writes the fp32 partial (a split piece);
+//  * segment end: the non-owner group hands its row sums to the owner of the last tile (mbarriers,
+//    neither group blocks), the owner hands the combined (row sum, reference) to an EPILOGUE
+//    WARPGROUP, which waits for the segment's last PV, reads O and writes the rows (a whole item) or
+//    the fp32 partial (a split piece; the last piece merges) -- the softmax groups go straight on with
+//    the next segment, whose PVs wait only until the epilogue has read O;
 //  * K and V in separate TMA rings fed by two producer warps; S issuer and PV issuer threads;
-//  * warpgroups: 0-1 softmax, 2 control (producers, issuers); setmaxnreg moves registers from the
-//    control warpgroup (56 per thread) to the softmax warpgroups (224: the scores stay in registers);
+//  * warpgroups: 0-1 softmax, 2 control (producers, issuers), 3 epilogue; setmaxnreg moves registers
+//    from the control and epilogue warpgroups (56 per thread) to the softmax warpgroups (200: the
+//    scores stay in registers);
 //  * lane mode (schedule_kernel): the row blocks of one (request, kv-head) run on `lanes` CTAs in
 //    lock-step over the same tile range, so each KV tile is read from HBM once;
 //  * tree keys are masked with the ancestor-or-self bitset of the row's node (tree_prepare);
@@ -34,12 +38,13 @@ constexpr int RB = kRowsBlock;              // 128 query rows per item
 constexpr int kQBuf = 2 * RB * 128;          // one Q buffer: 2 halves x 128 rows x 128 B
 constexpr int kTmemCols = 512;
 constexpr int kColS = 0, kColO = 256, kColP = 384;
-// warp roles: 0-7 softmax / epilogue (two groups of 4, warp & 3 = TMEM lane quarter), 8 Q / K producer,
-// 9 S issuer (+ TMEM allocation), 10 PV issuer, 11 V producer.  The control warpgroup (8-11) gives registers
-// to the softmax warpgroups (setmaxnreg): 168 per thread at launch -> 56 / 224
-constexpr int kThreads = 384;
+// warp roles: 0-7 softmax (two groups of 4, warp & 3 = TMEM lane quarter), 8 Q / K producer, 9 S issuer
+// (+ TMEM allocation), 10 PV issuer, 11 V producer, 12-15 epilogue (warp & 3 = TMEM lane quarter).  The
+// control (8-11) and epilogue (12-15) warpgroups give registers to the softmax warpgroups (setmaxnreg):
+// 128 per thread at launch -> 56 / 56 / 200
+constexpr int kThreads = 512;
 constexpr int kWarpProd = 8, kWarpS = 9, kWarpPV = 10, kWarpV = 11;
-constexpr int kRegsCtl = 56, kRegsSoftmax = 224;
+constexpr int kRegsCtl = 56, kRegsEpi = 56, kRegsSoftmax = 200;
 constexpr int kMaxK = 4, kMaxV = 4;          // ring slots (the launch picks 3 K + 2 V)
 
 struct Misc {
@@ -49,13 +54,17 @@ struct Misc {
     uint64_t s_full[2], s_free[2];           // S(t) ready / S buffer t & 1 loaded by the softmax
     uint64_t p_full[2], pv_done[2];          // P(t) written / PV(t) complete (P buffer free, O advanced)
     uint64_t o_free;                         // the epilogue has read O (next segment may overwrite it)
+    uint64_t o_full;                         // a segment's last PV complete (O final)
+    uint64_t epi_full[2], epi_empty[2];      // fin[slot] written by the segment's owner group / read
+    uint64_t xl_full[2], xl_empty[2];        // xl[slot] written by the non-owner group / read by the owner
+    float xl[2][2][RB];                      // [segment & 1][non-owner row sum, its reference][row]
+    float fin[2][2][RB];                     // [segment & 1][row sum, row reference][row] -> epilogue
     uint64_t seg_full[kSegRing];
     SegDesc seg[kSegRing];
     uint64_t stage_bar;                      // bulk staging of split pieces (CTA's last segment)
     uint32_t tmem_base;
     int32_t bcast;
-    float xm[2][2][RB];                      // [0][0]: row references; [0][1]: the row's final sum;
-                                             // [1][0] / [1][1]: segment-end hand-over
+    float mref[RB];                          // [row] the row reference after the latest decision
 };
 
 __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
@@ -69,45 +78,39 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
         : "r"(taddr));
 }
 
-// The normalised bf16 output of one query row, dims [64 h, 64 h + 64) (TMEM columns of O): both
-// TMEM loads, one wait, the bf16 packing -- then the warp releases O (arrives on `o_free`: the next
-// segment's first PV may overwrite it) BEFORE its 16-byte global stores, which stay off the
-// critical path of the next segment.
-__device__ __forceinline__ void store_o_half(uint32_t o_col, float inv, bool row_valid, __nv_bfloat16 *orow, int h,
-                                             uint64_t *o_free) {
-    uint32_t o[2][32];
-    tmem_ld32(o_col + h * 64, o[0]);
-    tmem_ld32(o_col + h * 64 + 32, o[1]);
-    tmem_ld_wait();
-    uint4 w[8];
-#pragma unroll
-    for (int q = 0; q < 2; ++q) {
-#pragma unroll
-        for (int i = 0; i < 32; i += 8) {
-            uint4 &x = w[q * 4 + i / 8];
-            x.x = pack_bf16x2(__uint_as_float(o[q][i]) * inv, __uint_as_float(o[q][i + 1]) * inv);
-            x.y = pack_bf16x2(__uint_as_float(o[q][i + 2]) * inv, __uint_as_float(o[q][i + 3]) * inv);
-            x.z = pack_bf16x2(__uint_as_float(o[q][i + 4]) * inv, __uint_as_float(o[q][i + 5]) * inv);
-            x.w = pack_bf16x2(__uint_as_float(o[q][i + 6]) * inv, __uint_as_float(o[q][i + 7]) * inv);
+// The normalised bf16 output of one query row (TMEM columns of O), 32 dims per TMEM load: the warp
+// releases O (arrives on `o_free`: the next segment's first PV may overwrite it) right after its last
+// TMEM load; the 32-byte global stores stay off the critical path.
+__device__ __forceinline__ void store_o_row(uint32_t o_col, float inv, bool row_valid, __nv_bfloat16 *orow,
+                                            uint64_t *o_free) {
+    const bool al32 = (reinterpret_cast<uintptr_t>(orow) & 31u) == 0;
+#pragma unroll 1
+    for (int q = 0; q < 4; ++q) {
+        uint32_t o[32];
+        tmem_ld32(o_col + q * 32, o);
+        tmem_ld_wait();
+        if (q == 3) {
+            tc_fence_before();
+            __syncwarp();
+            if ((threadIdx.x & 31) == 0) mbar_arrive(o_free);
         }
-    }
-    tc_fence_before();
-    __syncwarp();
-    if ((threadIdx.x & 31) == 0) mbar_arrive(o_free);
-    if (!row_valid) return;
-    __nv_bfloat16 *dst = orow + h * 64;
-    if ((reinterpret_cast<uintptr_t>(dst) & 31u) == 0) {
-        // 32-byte stores (one full L2 sector per thread and instruction): each warp instruction writes
-        // 32 different rows, so the store cost is per instruction -- half as many as 16-byte stores
+        if (!row_valid) continue;
+        uint32_t w[16];
 #pragma unroll
-        for (int k = 0; k < 4; ++k)
-            asm volatile("st.global.v8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"l"(dst + k * 16),
-                         "r"(w[2 * k].x), "r"(w[2 * k].y), "r"(w[2 * k].z), "r"(w[2 * k].w), "r"(w[2 * k + 1].x),
-                         "r"(w[2 * k + 1].y), "r"(w[2 * k + 1].z), "r"(w[2 * k + 1].w)
-                         : "memory");
-    } else {
+        for (int i = 0; i < 16; ++i) w[i] = pack_bf16x2(__uint_as_float(o[2 * i]) * inv, __uint_as_float(o[2 * i + 1]) * inv);
+        __nv_bfloat16 *dst = orow + q * 32;
+        if (al32) {
 #pragma unroll
-        for (int k = 0; k < 8; ++k) *reinterpret_cast<uint4 *>(dst + k * 8) = w[k];
+            for (int k = 0; k < 2; ++k)
+                asm volatile("st.global.v8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"l"(dst + k * 16),
+                             "r"(w[8 * k]), "r"(w[8 * k + 1]), "r"(w[8 * k + 2]), "r"(w[8 * k + 3]), "r"(w[8 * k + 4]),
+                             "r"(w[8 * k + 5]), "r"(w[8 * k + 6]), "r"(w[8 * k + 7])
+                             : "memory");
+        } else {
+#pragma unroll
+            for (int k = 0; k < 4; ++k)
+                *reinterpret_cast<uint4 *>(dst + k * 8) = make_uint4(w[4 * k], w[4 * k + 1], w[4 * k + 2], w[4 * k + 3]);
+        }
     }
 }
 
@@ -184,7 +187,7 @@ __device__ __forceinline__ void mask32(uint32_t (&v)[32], uint32_t vis) {
 
 }  // namespace rows
 
-__global__ void __maxnreg__(168)
+__global__ void __launch_bounds__(rows::kThreads, 1)
     tree_attn_rows_kernel(const __grid_constant__ CUtensorMap tm_q, const __grid_constant__ CUtensorMap tm_k,
                           const __grid_constant__ CUtensorMap tm_v, const __grid_constant__ CUtensorMap tm_k16,
                           const __grid_constant__ CUtensorMap tm_v16, const __grid_constant__ CUtensorMap tm_k4,
@@ -224,7 +227,14 @@ __global__ void __maxnreg__(168)
             mbar_init(&misc->p_full[i], 4);
             mbar_init(&misc->pv_done[i], 1);
         }
-        mbar_init(&misc->o_free, 8);   // every softmax warp (both groups share the epilogue)
+        mbar_init(&misc->o_free, 4);   // the epilogue warpgroup's 4 warps
+        mbar_init(&misc->o_full, 1);
+        for (int i = 0; i < 2; ++i) {
+            mbar_init(&misc->epi_full[i], 4);
+            mbar_init(&misc->epi_empty[i], 4);
+            mbar_init(&misc->xl_full[i], 4);
+            mbar_init(&misc->xl_empty[i], 4);
+        }
         mbar_init(&misc->stage_bar, 1);
         for (int i = 0; i < kSegRing; ++i) mbar_init(&misc->seg_full[i], 1);
         fence_barrier_init();
@@ -258,7 +268,241 @@ __global__ void __maxnreg__(168)
     const int t0 = ci.x, t1 = ci.y, x_first = ci.z, T = ci.w;
     const int ntiles = t1 - t0;
 
-    if (warp >= 8) {
+    if (warp >= 12) {
+        // epilogue warpgroup (warp & 3 = TMEM lane quarter): its registers go to the softmax warps
+        setmaxnreg_dec<kRegsEpi>();
+        if (ntiles > 0) {
+            // ====== epilogue: per segment, once the owner group handed over (row sum, reference) and the
+            // segment's last PV completed, O -> normalised bf16 rows (a whole item) or the fp32 partial of a
+            // split piece (the last piece merges every piece); O is released after its TMEM loads ======
+            const int qd = warp & 3;
+            const int r = qd * 32 + lane;
+            const uint32_t lane_off = (uint32_t)(qd * 32) << 16;
+            const uint32_t o_col = tmem + kColO + lane_off;
+            int ls = 0, lt_end = 0;
+            for (;;) {
+                mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
+                const SegDesc sd = misc->seg[ls % kSegRing];
+                if (sd.x < 0) break;
+                lt_end += sd.end - sd.begin;
+                const int lt = lt_end - 1;   // (trace slots: the segment's last tile)
+                const int b = sd.b, g = sd.g, c = sd.c, n = sd.n;
+                const int G = p.G;
+                const int rc = G * p.npc;
+                const int node = c * p.npc + r / G, hl = r % G;
+                const bool row_valid = (r < rc) && (node < n);
+                const bool full = (sd.begin == sd.ib) && (sd.end == sd.ie);
+                const int fs = ls & 1;
+                mbar_wait(&misc->epi_full[fs], (ls >> 1) & 1);
+                if (r == 0) SPI_TRACE(10);
+                const float lrow = misc->fin[fs][0][r], m = misc->fin[fs][1][r];
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&misc->epi_empty[fs]);
+                mbar_wait(&misc->o_full, ls & 1);   // one phase per segment, consumed in order
+                tc_fence_after();
+                if (r == 0) SPI_TRACE(11);
+                if (full) {
+                    store_o_row(o_col, 1.0f / lrow, row_valid,
+                                p.out + (((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim, &misc->o_free);
+                } else {
+                    // a piece of a split item: unnormalised O row, (m, l) of the row, then the last piece
+                    // merges every piece by log-sum-exp
+                    const int slot = (sd.begin == t0) ? 0 : 1;
+                    float *po = p.part_o + (((size_t)blockIdx.x * 2 + slot) * RB + r) * kHeadDim;
+#pragma unroll 1
+                    for (int q2 = 0; q2 < 4; ++q2) {
+                        uint32_t o[32];
+                        tmem_ld32(o_col + q2 * 32, o);
+                        tmem_ld_wait();
+#pragma unroll
+                        for (int i = 0; i < 32; i += 8)   // 32-byte stores (part_o rows are 512-byte aligned)
+                            asm volatile("st.global.v8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"l"(po + q2 * 32 + i),
+                                         "r"(o[i]), "r"(o[i + 1]), "r"(o[i + 2]), "r"(o[i + 3]), "r"(o[i + 4]),
+                                         "r"(o[i + 5]), "r"(o[i + 6]), "r"(o[i + 7])
+                                         : "memory");
+                    }
+                    tc_fence_before();
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(&misc->o_free);
+                    float *pml = p.part_ml + ((size_t)blockIdx.x * 2 + slot) * 2 * RB;
+                    pml[r] = m;
+                    pml[RB + r] = lrow;
+                    __threadfence();
+                    named_bar_sync(14, 128);   // the epilogue warpgroup
+                    if (r == 0) {
+                        const int c_first = cta_of_tile(sd.ib, T, NC);
+                        const int c_last = cta_of_tile(sd.ie - 1, T, NC);
+                        int npieces = 0;
+                        for (int cc = c_first; cc <= c_last; ++cc)
+                            npieces += cta_start(cc + 1, T, NC) > cta_start(cc, T, NC);
+                        const unsigned old = atomicAdd(&p.item_cnt[sd.x], 1u);
+                        misc->bcast = (old == (unsigned)(npieces - 1)) ? 1 : 0;
+                        if (misc->bcast) p.item_cnt[sd.x] = 0u;  // ready for the next launch
+                    }
+                    named_bar_sync(14, 128);
+                    if (misc->bcast) {
+                        // last piece: merge every piece's (m, l, O row) by log-sum-exp
+                        __threadfence();
+                        const int c_first = cta_of_tile(sd.ib, T, NC);
+                        const int c_last = cta_of_tile(sd.ie - 1, T, NC);
+                        auto piece = [&](int cc) -> long long {   // partial slot of CTA cc's piece, -1 if empty
+                            const int s0 = cta_start(cc, T, NC);
+                            if (cta_start(cc + 1, T, NC) <= s0) return -1;
+                            return ((long long)cc * p.lanes + cl) * 2 + ((s0 >= sd.ib) ? 0 : 1);
+                        };
+                        // (compact, rolled loops: this code runs cold in the instruction cache, once per item,
+                        // and its length -- not its loads -- set the cost: ~350 ns per missed 128-B line)
+                        if (sd.end == t1) {
+                            // the CTA's last segment: K / V rings and Q buffers are idle -> stage the pieces with
+                            // bulk copies (all in flight at once) instead of one L2 round trip per (piece, chunk):
+                            // (m, l) of every piece, then up to `cap` 64 KB O blocks per round; each warp merges
+                            // its 32 rows with lane = 4 dims (conflict-free, coalesced 256 B output rows)
+                            uint8_t *area = smem;
+                            const size_t area_bytes = (size_t)(NK + NV) * kSlotBytes + 2 * kQBuf;
+                            constexpr uint32_t kOB = RB * kHeadDim * 4, kMLB = 2 * RB * 4;
+                            int npc = 0;
+                            for (int cc = c_first; cc <= c_last; ++cc) npc += piece(cc) >= 0;
+                            float *sml = reinterpret_cast<float *>(area + area_bytes) - (size_t)npc * 3 * RB;  // [npc][m, l, w][RB]
+                            const int cap = (int)(((size_t)((uint8_t *)sml - area)) / kOB);
+                            uint32_t ph = 0;
+                            if (r == 0) {
+                                fence_proxy_async_global();
+                                mbar_arrive_expect_tx(&misc->stage_bar, (uint32_t)npc * kMLB);
+                                int k = 0;
+                                for (int cc = c_first; cc <= c_last; ++cc) {
+                                    const long long po2 = piece(cc);
+                                    if (po2 < 0) continue;
+                                    bulk_load_g2s(sml + (size_t)k * 3 * RB, p.part_ml + po2 * 2 * RB, kMLB, &misc->stage_bar);
+                                    ++k;
+                                }
+                            }
+                            mbar_wait(&misc->stage_bar, ph);
+                            ph ^= 1u;
+                            float Mx = -INFINITY, Ls = 0.f;
+                            for (int k = 0; k < npc; ++k) Mx = fmaxf(Mx, sml[(size_t)k * 3 * RB + r]);
+                            for (int k = 0; k < npc; ++k) {
+                                const float mk = sml[(size_t)k * 3 * RB + r];
+                                const float w = (mk == -INFINITY) ? 0.f : ex2(mk - Mx);
+                                Ls += w * sml[(size_t)k * 3 * RB + RB + r];
+                                sml[(size_t)k * 3 * RB + 2 * RB + r] = w;
+                            }
+                            const float inv = 1.0f / Ls;
+                            for (int k = 0; k < npc; ++k) sml[(size_t)k * 3 * RB + 2 * RB + r] *= inv;
+                            named_bar_sync(14, 128);   // weights visible to the whole group
+                            // rows in 4 batches of 8 (registers: the epilogue warpgroup runs on a small budget);
+                            // all pieces staged once when they fit the area, else re-staged per batch and round
+                            const int wrow0 = qd * 32;   // this warp's rows
+                            const bool one_round = npc <= cap;
+#pragma unroll 1
+                            for (int rb = 0; rb < 4; ++rb) {
+                                float4 acc[8];   // [row of the batch] lane's 4 dims
+#pragma unroll
+                                for (int i = 0; i < 8; ++i) acc[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll 1
+                                for (int k0 = 0; k0 < npc; k0 += cap) {
+                                    const int kn = min(cap, npc - k0);
+                                    if (rb == 0 || !one_round) {
+                                        if (r == 0) {
+                                            mbar_arrive_expect_tx(&misc->stage_bar, (uint32_t)kn * kOB);
+                                            int k = 0;
+                                            for (int cc = c_first; cc <= c_last; ++cc) {
+                                                const long long po2 = piece(cc);
+                                                if (po2 < 0) continue;
+                                                if (k >= k0 && k < k0 + kn)
+                                                    bulk_load_g2s(area + (size_t)(k - k0) * kOB, p.part_o + po2 * RB * kHeadDim,
+                                                                  kOB, &misc->stage_bar);
+                                                ++k;
+                                            }
+                                        }
+                                        mbar_wait(&misc->stage_bar, ph);
+                                        ph ^= 1u;
+                                    }
+#pragma unroll 1
+                                    for (int k = 0; k < kn; ++k) {
+                                        const float *blk = reinterpret_cast<const float *>(area + (size_t)k * kOB);
+                                        const float *wk = sml + (size_t)(k0 + k) * 3 * RB + 2 * RB + wrow0 + rb * 8;
+#pragma unroll
+                                        for (int i = 0; i < 8; ++i) {
+                                            const float4 x = *reinterpret_cast<const float4 *>(
+                                                blk + (size_t)(wrow0 + rb * 8 + i) * kHeadDim + 4 * lane);
+                                            const float w = wk[i];
+                                            acc[i].x += w * x.x;
+                                            acc[i].y += w * x.y;
+                                            acc[i].z += w * x.z;
+                                            acc[i].w += w * x.w;
+                                        }
+                                    }
+                                    if (!one_round) named_bar_sync(14, 128);   // the staging area is reused
+                                }
+                                // rows of this batch: row wrow0 + rb * 8 + i -> its node / head (padding rows skipped)
+#pragma unroll
+                                for (int i = 0; i < 8; ++i) {
+                                    const int rr = wrow0 + rb * 8 + i;
+                                    const int nd = c * p.npc + rr / G, hh = rr % G;
+                                    if (rr < rc && nd < n) {
+                                        uint2 o2;
+                                        o2.x = pack_bf16x2(acc[i].x, acc[i].y);
+                                        o2.y = pack_bf16x2(acc[i].z, acc[i].w);
+                                        *reinterpret_cast<uint2 *>(p.out + (((size_t)b * p.Nmax + nd) * p.Hq + g * G + hh) *
+                                                                               kHeadDim + 4 * lane) = o2;
+                                    }
+                                }
+                            }
+                        } else {
+                            float Mx = -INFINITY, Ls = 0.f;
+#pragma unroll 1
+                            for (int cc = c_first; cc <= c_last; ++cc) {
+                                const long long po2 = piece(cc);
+                                if (po2 < 0) continue;
+                                const float mp = ldcg_f32(p.part_ml + po2 * 2 * RB + r);
+                                const float lp = ldcg_f32(p.part_ml + po2 * 2 * RB + RB + r);
+                                if (mp == -INFINITY) continue;
+                                const float nM = fmaxf(Mx, mp);
+                                Ls = (Mx == -INFINITY ? 0.f : Ls * ex2(Mx - nM)) + ex2(mp - nM) * lp;
+                                Mx = nM;
+                            }
+                            const float inv = 1.0f / Ls;
+                            __nv_bfloat16 *orow = p.out + (((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim;
+#pragma unroll 1
+                            for (int q2 = 0; q2 < 8; ++q2) {   // 16 dims at a time
+                                float4 a0 = make_float4(0.f, 0.f, 0.f, 0.f), a1 = a0, a2 = a0, a3 = a0;
+#pragma unroll 1
+                                for (int cc = c_first; cc <= c_last; ++cc) {
+                                    const long long po2 = piece(cc);
+                                    if (po2 < 0) continue;
+                                    const float mp = ldcg_f32(p.part_ml + po2 * 2 * RB + r);
+                                    const float4 *src = reinterpret_cast<const float4 *>(
+                                        p.part_o + (po2 * RB + r) * kHeadDim + q2 * 16);
+                                    const float4 x0 = __ldcg(src), x1 = __ldcg(src + 1), x2 = __ldcg(src + 2),
+                                                 x3 = __ldcg(src + 3);
+                                    const float w = (mp == -INFINITY) ? 0.f : ex2(mp - Mx) * inv;
+                                    a0.x += w * x0.x; a0.y += w * x0.y; a0.z += w * x0.z; a0.w += w * x0.w;
+                                    a1.x += w * x1.x; a1.y += w * x1.y; a1.z += w * x1.z; a1.w += w * x1.w;
+                                    a2.x += w * x2.x; a2.y += w * x2.y; a2.z += w * x2.z; a2.w += w * x2.w;
+                                    a3.x += w * x3.x; a3.y += w * x3.y; a3.z += w * x3.z; a3.w += w * x3.w;
+                                }
+                                if (row_valid) {
+                                    uint4 o4;
+                                    o4.x = pack_bf16x2(a0.x, a0.y);
+                                    o4.y = pack_bf16x2(a0.z, a0.w);
+                                    o4.z = pack_bf16x2(a1.x, a1.y);
+                                    o4.w = pack_bf16x2(a1.z, a1.w);
+                                    *reinterpret_cast<uint4 *>(orow + q2 * 16) = o4;
+                                    o4.x = pack_bf16x2(a2.x, a2.y);
+                                    o4.y = pack_bf16x2(a2.z, a2.w);
+                                    o4.z = pack_bf16x2(a3.x, a3.y);
+                                    o4.w = pack_bf16x2(a3.z, a3.w);
+                                    *reinterpret_cast<uint4 *>(orow + q2 * 16 + 8) = o4;
+                                }
+                            }
+                        }
+                    }
+
+                }
+                ++ls;
+            }
+        }
+    } else if (warp >= 8) {
         // control warpgroup: its registers go to the softmax warps (all 4 warps execute this one
         // instruction; no code path below rejoins the softmax path)
         setmaxnreg_dec<kRegsCtl>();
@@ -438,6 +682,7 @@ __global__ void __maxnreg__(168)
                         }
                         umma_commit(&misc->pv_done[pb]);
                         umma_commit(&misc->v_empty[slot]);
+                        if (t == d.end - 1) umma_commit(&misc->o_full);   // the segment's O is final
                     }
                     ++ls;
                 }
@@ -466,22 +711,18 @@ __global__ void __maxnreg__(168)
                 // would then read a stale reference.  Per direction, arrivals and syncs strictly alternate.)
                 const uint32_t dec_out = grp == 0 ? 6 + qd : 1 + qd;   // the decisions this group publishes
                 const uint32_t dec_in = grp == 0 ? 1 + qd : 6 + qd;    // the other group's decisions
-                const uint32_t epi_bar = 10 + qd;      // segment-end row-sum hand-over
                 const uint32_t o_col = tmem + kColO + lane_off;
-                float *mref_s = misc->xm[0][0];        // [row] the row reference after the latest decision
-                float *xl_l = misc->xm[1][0];          // [row] the non-owner group's row sum at a segment end
-                float *xl_m = misc->xm[1][1];          //       ... and the reference it is relative to
-                float *xl_f = misc->xm[0][1];          // [row] the final row sum (owner -> the other group)
+                float *mref_s = misc->mref;            // [row] the row reference after the latest decision
                 int lt = 0, ls = 0;
                 for (;;) {
                     mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
                     const SegDesc sd = misc->seg[ls % kSegRing];
                     if (sd.x < 0) break;
-                    const int b = sd.b, g = sd.g, c = sd.c, P = sd.P, n = sd.n;
+                    const int b = sd.b, c = sd.c, P = sd.P, n = sd.n;
                     const int Kend = P + n;
                     const int G = p.G;
                     const int rc = G * p.npc;
-                    const int node = c * p.npc + r / G, hl = r % G;
+                    const int node = c * p.npc + r / G;
                     const bool row_valid = (r < rc) && (node < n);
                     // ancestor-or-self bitset of this row's node, read on masked tiles only (rows without a
                     // node use node 0's root path, which keeps them finite; they are never written)
@@ -610,242 +851,31 @@ __global__ void __maxnreg__(168)
                         if (r == 0) SPI_TRACE(6 + grp);
                     }
 
-                    // ============ epilogue of this segment ============
-                    // The owner of the segment's last tile combines both groups' row sums; for a whole item both
-                    // groups then write half of the row's 128 dims each (the output store of one group alone
-                    // stalled the other group's next tile for the whole epilogue), a split piece is written by
-                    // the owner.
+                    // ============ end of this segment ============
+                    // The non-owner group hands its (row sum, reference) to the owner of the segment's last tile
+                    // through xl[segment & 1] (mbarriers: neither group blocks on the other here); the owner
+                    // combines both and hands (row sum, reference) to the epilogue warpgroup, which reads O once
+                    // the last PV completed.  Neither softmax group waits for that PV or touches O here.
                     const int llast = lt - 1;
                     const int owner = llast & 1;
-                    const bool full = (sd.begin == sd.ib) && (sd.end == sd.ie);
-                    // (two full barriers, executed by both groups at the same two instructions: the non-owner may
-                    // not overwrite the hand-over slots of the next segment before the owner has read them, and
-                    // it reads the final sum only after the owner wrote it)
+                    const int fs = ls & 1;
                     if (grp != owner) {
-                        xl_l[r] = l;
-                        xl_m[r] = m;
-                    }
-                    named_bar_sync(epi_bar, 64);
-                    float lrow = 0.f;
-                    if (grp == owner) {
-                        const float lo_ = xl_l[r], mo = xl_m[r];
-                        lrow = l + ((mo == -INFINITY || lo_ == 0.f) ? 0.f : lo_ * ex2(mo - m));
-                        xl_f[r] = lrow;
-                    }
-                    named_bar_sync(epi_bar, 64);
-                    if (grp != owner) {
-                        if (full) {
-                            const float inv = 1.0f / xl_f[r];
-                            // O complete: this group last observed pv_done of ITS parity, so first wait for PV(llast - 1)
-                            // (its own tile: at most one phase ahead), which implies PV(llast - 2); only then is the
-                            // parity wait for PV(llast) on the other barrier unambiguous
-                            if (llast >= 1) mbar_wait(&misc->pv_done[(llast - 1) & 1], ((llast - 1) >> 1) & 1);
-                            mbar_wait(&misc->pv_done[llast & 1], (llast >> 1) & 1);
-                            tc_fence_after();
-                            store_o_half(o_col, inv, row_valid,
-                                         p.out + (((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim, 1,
-                                         &misc->o_free);
-                        } else {
-                            tc_fence_before();
-                            __syncwarp();
-                            if (lane == 0) mbar_arrive(&misc->o_free);
-                        }
+                        if (ls >= 2) mbar_wait(&misc->xl_empty[fs], ((ls >> 1) - 1) & 1);
+                        misc->xl[fs][0][r] = l;
+                        misc->xl[fs][1][r] = m;
+                        __syncwarp();
+                        if (lane == 0) mbar_arrive(&misc->xl_full[fs]);
                     } else {
-                        mbar_wait(&misc->pv_done[llast & 1], (llast >> 1) & 1);   // O complete (in-order PVs)
-                        tc_fence_after();
-                        if (r == 0) SPI_TRACE(10);
-                        if (full) {
-                            store_o_half(o_col, 1.0f / lrow, row_valid,
-                                         p.out + (((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim, 0,
-                                         &misc->o_free);
-                        } else {
-                            // a piece of a split item: unnormalised O row, (m, l) of the row, then the last piece
-                            // merges every piece by log-sum-exp
-                            const int slot = (sd.begin == t0) ? 0 : 1;
-                            float *po = p.part_o + (((size_t)blockIdx.x * 2 + slot) * RB + r) * kHeadDim;
-#pragma unroll 1
-                            for (int q2 = 0; q2 < 4; ++q2) {
-                                uint32_t o[32];
-                                tmem_ld32(o_col + q2 * 32, o);
-                                tmem_ld_wait();
-#pragma unroll
-                                for (int i = 0; i < 32; i += 8)   // 32-byte stores (part_o rows are 512-byte aligned)
-                                    asm volatile("st.global.v8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"l"(po + q2 * 32 + i),
-                                                 "r"(o[i]), "r"(o[i + 1]), "r"(o[i + 2]), "r"(o[i + 3]), "r"(o[i + 4]),
-                                                 "r"(o[i + 5]), "r"(o[i + 6]), "r"(o[i + 7])
-                                                 : "memory");
-                            }
-                            tc_fence_before();
-                            __syncwarp();
-                            if (lane == 0) mbar_arrive(&misc->o_free);
-                            float *pml = p.part_ml + ((size_t)blockIdx.x * 2 + slot) * 2 * RB;
-                            pml[r] = m;
-                            pml[RB + r] = lrow;
-                            if (r == 0) SPI_TRACE(12);
-                            __threadfence();
-                            named_bar_sync(14, 128);   // the owner group's 4 warps
-                            if (r == 0) {
-                                const int c_first = cta_of_tile(sd.ib, T, NC);
-                                const int c_last = cta_of_tile(sd.ie - 1, T, NC);
-                                int npieces = 0;
-                                for (int cc = c_first; cc <= c_last; ++cc)
-                                    npieces += cta_start(cc + 1, T, NC) > cta_start(cc, T, NC);
-                                const unsigned old = atomicAdd(&p.item_cnt[sd.x], 1u);
-                                misc->bcast = (old == (unsigned)(npieces - 1)) ? 1 : 0;
-                                if (misc->bcast) p.item_cnt[sd.x] = 0u;  // ready for the next launch
-                            }
-                            named_bar_sync(14, 128);
-                            if (r == 0) SPI_TRACE(13);
-                            if (misc->bcast) {
-                                // last piece: merge every piece's (m, l, O row) by log-sum-exp
-                                __threadfence();
-                                const int c_first = cta_of_tile(sd.ib, T, NC);
-                                const int c_last = cta_of_tile(sd.ie - 1, T, NC);
-                                auto piece = [&](int cc) -> long long {   // partial slot of CTA cc's piece, -1 if empty
-                                    const int s0 = cta_start(cc, T, NC);
-                                    if (cta_start(cc + 1, T, NC) <= s0) return -1;
-                                    return ((long long)cc * p.lanes + cl) * 2 + ((s0 >= sd.ib) ? 0 : 1);
-                                };
-                                // (compact, rolled loops: this code runs cold in the instruction cache, once per item,
-                                // and its length -- not its loads -- set the cost: ~350 ns per missed 128-B line)
-                                if (sd.end == t1) {
-                                    // the CTA's last segment: K / V rings and Q buffers are idle -> stage the pieces with
-                                    // bulk copies (all in flight at once) instead of one L2 round trip per (piece, chunk):
-                                    // (m, l) of every piece, then up to `cap` 64 KB O blocks per round; each warp merges
-                                    // its 32 rows with lane = 4 dims (conflict-free, coalesced 256 B output rows)
-                                    uint8_t *area = smem;
-                                    const size_t area_bytes = (size_t)(NK + NV) * kSlotBytes + 2 * kQBuf;
-                                    constexpr uint32_t kOB = RB * kHeadDim * 4, kMLB = 2 * RB * 4;
-                                    int npc = 0;
-                                    for (int cc = c_first; cc <= c_last; ++cc) npc += piece(cc) >= 0;
-                                    float *sml = reinterpret_cast<float *>(area + area_bytes) - (size_t)npc * 3 * RB;  // [npc][m, l, w][RB]
-                                    const int cap = (int)(((size_t)((uint8_t *)sml - area)) / kOB);
-                                    uint32_t ph = 0;
-                                    if (r == 0) {
-                                        fence_proxy_async_global();
-                                        mbar_arrive_expect_tx(&misc->stage_bar, (uint32_t)npc * kMLB);
-                                        int k = 0;
-                                        for (int cc = c_first; cc <= c_last; ++cc) {
-                                            const long long po2 = piece(cc);
-                                            if (po2 < 0) continue;
-                                            bulk_load_g2s(sml + (size_t)k * 3 * RB, p.part_ml + po2 * 2 * RB, kMLB, &misc->stage_bar);
-                                            ++k;
-                                        }
-                                    }
-                                    mbar_wait(&misc->stage_bar, ph);
-                                    ph ^= 1u;
-                                    float Mx = -INFINITY, Ls = 0.f;
-                                    for (int k = 0; k < npc; ++k) Mx = fmaxf(Mx, sml[(size_t)k * 3 * RB + r]);
-                                    for (int k = 0; k < npc; ++k) {
-                                        const float mk = sml[(size_t)k * 3 * RB + r];
-                                        const float w = (mk == -INFINITY) ? 0.f : ex2(mk - Mx);
-                                        Ls += w * sml[(size_t)k * 3 * RB + RB + r];
-                                        sml[(size_t)k * 3 * RB + 2 * RB + r] = w;
-                                    }
-                                    const float inv = 1.0f / Ls;
-                                    for (int k = 0; k < npc; ++k) sml[(size_t)k * 3 * RB + 2 * RB + r] *= inv;
-                                    named_bar_sync(14, 128);   // weights visible to the whole group
-                                    float4 acc[32];   // [row of the warp] lane's 4 dims
-#pragma unroll
-                                    for (int i = 0; i < 32; ++i) acc[i] = make_float4(0.f, 0.f, 0.f, 0.f);
-                                    const int wrow0 = qd * 32;   // this warp's rows
-                                    for (int k0 = 0; k0 < npc; k0 += cap) {
-                                        const int kn = min(cap, npc - k0);
-                                        if (r == 0) {
-                                            mbar_arrive_expect_tx(&misc->stage_bar, (uint32_t)kn * kOB);
-                                            int k = 0;
-                                            for (int cc = c_first; cc <= c_last; ++cc) {
-                                                const long long po2 = piece(cc);
-                                                if (po2 < 0) continue;
-                                                if (k >= k0 && k < k0 + kn)
-                                                    bulk_load_g2s(area + (size_t)(k - k0) * kOB, p.part_o + po2 * RB * kHeadDim, kOB,
-                                                                  &misc->stage_bar);
-                                                ++k;
-                                            }
-                                        }
-                                        mbar_wait(&misc->stage_bar, ph);
-                                        ph ^= 1u;
-#pragma unroll 1
-                                        for (int k = 0; k < kn; ++k) {
-                                            const float *blk = reinterpret_cast<const float *>(area + (size_t)k * kOB);
-                                            const float *wk = sml + (size_t)(k0 + k) * 3 * RB + 2 * RB + wrow0;
-#pragma unroll
-                                            for (int i = 0; i < 32; ++i) {
-                                                const float4 x = *reinterpret_cast<const float4 *>(blk + (size_t)(wrow0 + i) * kHeadDim + 4 * lane);
-                                                const float w = wk[i];
-                                                acc[i].x += w * x.x;
-                                                acc[i].y += w * x.y;
-                                                acc[i].z += w * x.z;
-                                                acc[i].w += w * x.w;
-                                            }
-                                        }
-                                        named_bar_sync(14, 128);   // the staging area is reused by the next round
-                                    }
-                                    // rows of this warp: row wrow0 + i -> its node / head (padding rows skipped)
-#pragma unroll
-                                    for (int i = 0; i < 32; ++i) {
-                                        const int rr = wrow0 + i;
-                                        const int nd = c * p.npc + rr / G, hh = rr % G;
-                                        if (rr < rc && nd < n) {
-                                            uint2 o2;
-                                            o2.x = pack_bf16x2(acc[i].x, acc[i].y);
-                                            o2.y = pack_bf16x2(acc[i].z, acc[i].w);
-                                            *reinterpret_cast<uint2 *>(p.out + (((size_t)b * p.Nmax + nd) * p.Hq + g * G + hh) * kHeadDim +
-                                                                       4 * lane) = o2;
-                                        }
-                                    }
-                                } else {
-                                    float Mx = -INFINITY, Ls = 0.f;
-    #pragma unroll 1
-                                    for (int cc = c_first; cc <= c_last; ++cc) {
-                                        const long long po2 = piece(cc);
-                                        if (po2 < 0) continue;
-                                        const float mp = ldcg_f32(p.part_ml + po2 * 2 * RB + r);
-                                        const float lp = ldcg_f32(p.part_ml + po2 * 2 * RB + RB + r);
-                                        if (mp == -INFINITY) continue;
-                                        const float nM = fmaxf(Mx, mp);
-                                        Ls = (Mx == -INFINITY ? 0.f : Ls * ex2(Mx - nM)) + ex2(mp - nM) * lp;
-                                        Mx = nM;
-                                    }
-                                    const float inv = 1.0f / Ls;
-                                    if (r == 0) SPI_TRACE(14);
-                                    __nv_bfloat16 *orow = p.out + (((size_t)b * p.Nmax + node) * p.Hq + g * G + hl) * kHeadDim;
-    #pragma unroll 1
-                                    for (int q2 = 0; q2 < 8; ++q2) {   // 16 dims at a time
-                                        float4 a0 = make_float4(0.f, 0.f, 0.f, 0.f), a1 = a0, a2 = a0, a3 = a0;
-    #pragma unroll 1
-                                        for (int cc = c_first; cc <= c_last; ++cc) {
-                                            const long long po2 = piece(cc);
-                                            if (po2 < 0) continue;
-                                            const float mp = ldcg_f32(p.part_ml + po2 * 2 * RB + r);
-                                            const float4 *src = reinterpret_cast<const float4 *>(
-                                                p.part_o + (po2 * RB + r) * kHeadDim + q2 * 16);
-                                            const float4 x0 = __ldcg(src), x1 = __ldcg(src + 1), x2 = __ldcg(src + 2),
-                                                         x3 = __ldcg(src + 3);
-                                            const float w = (mp == -INFINITY) ? 0.f : ex2(mp - Mx) * inv;
-                                            a0.x += w * x0.x; a0.y += w * x0.y; a0.z += w * x0.z; a0.w += w * x0.w;
-                                            a1.x += w * x1.x; a1.y += w * x1.y; a1.z += w * x1.z; a1.w += w * x1.w;
-                                            a2.x += w * x2.x; a2.y += w * x2.y; a2.z += w * x2.z; a2.w += w * x2.w;
-                                            a3.x += w * x3.x; a3.y += w * x3.y; a3.z += w * x3.z; a3.w += w * x3.w;
-                                        }
-                                        if (row_valid) {
-                                            uint4 o4;
-                                            o4.x = pack_bf16x2(a0.x, a0.y);
-                                            o4.y = pack_bf16x2(a0.z, a0.w);
-                                            o4.z = pack_bf16x2(a1.x, a1.y);
-                                            o4.w = pack_bf16x2(a1.z, a1.w);
-                                            *reinterpret_cast<uint4 *>(orow + q2 * 16) = o4;
-                                            o4.x = pack_bf16x2(a2.x, a2.y);
-                                            o4.y = pack_bf16x2(a2.z, a2.w);
-                                            o4.z = pack_bf16x2(a3.x, a3.y);
-                                            o4.w = pack_bf16x2(a3.z, a3.w);
-                                            *reinterpret_cast<uint4 *>(orow + q2 * 16 + 8) = o4;
-                                        }
-                                    }
-                                }
-                            }
-                        }
-                        if (r == 0) SPI_TRACE(11);
+                        mbar_wait(&misc->xl_full[fs], (ls >> 1) & 1);
+                        const float lo_ = misc->xl[fs][0][r], mo = misc->xl[fs][1][r];
+                        __syncwarp();
+                        if (lane == 0) mbar_arrive(&misc->xl_empty[fs]);
+                        const float lrow = l + ((mo == -INFINITY || lo_ == 0.f) ? 0.f : lo_ * ex2(mo - m));
+                        if (ls >= 2) mbar_wait(&misc->epi_empty[fs], ((ls >> 1) - 1) & 1);
+                        misc->fin[fs][0][r] = lrow;
+                        misc->fin[fs][1][r] = m;
+                        __syncwarp();
+                        if (lane == 0) mbar_arrive(&misc->epi_full[fs]);
                     }
                     ++ls;
                 }
