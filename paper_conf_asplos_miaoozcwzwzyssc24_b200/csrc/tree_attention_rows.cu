@@ -891,6 +891,13 @@ __global__ void __launch_bounds__(rows::kThreads, 1)
         tmem_dealloc<kTmemCols>(tmem);
     }
     if (threadIdx.x == 0) SPI_TRACE_K(1);
+#ifdef SPECINFER_DEBUG_HOOKS
+    if (threadIdx.x == 0 && SPI_TRACING(p)) {   // slot 3 (unused here): the SM this CTA ran on
+        uint32_t smid;
+        asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+        p.trace[(size_t)kTraceCtas * kTraceTiles * kTraceEv + blockIdx.x * 8 + 3] = smid + 1;
+    }
+#endif
 }
 
 static size_t rows_smem_bytes(int nk, int nv) {

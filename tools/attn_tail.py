@@ -57,6 +57,9 @@ print("latest 12 CTAs (cta, entry, firstK, exit):")
 for c in order[-12:]:
     print(f"  {c:4d} {(kt[c,0]-t0)/1e3:7.2f} {fk[c]:7.2f} {ex[c]:7.2f}")
 print("earliest 5:", [(int(c), round(float(ex[c]), 2)) for c in order[:5]])
+if a.config in ("C3", "C4"):   # rows kernel: slot 3 holds smid + 1
+    sm = kt[:, 3] - 1
+    print("exit us by CTA:", " ".join(f"{c}:{ex[c]:.0f}/sm{sm[c]}" for c in range(len(ex))))
 if (kt[:, 3] > 0).any():
     s3 = (kt[:, 3] - t0) / 1e3
     print("split-KV: first cluster barrier passed (us) min/median/max:", np.percentile(s3[kt[:, 3] > 0], [0, 50, 100]).round(2))
