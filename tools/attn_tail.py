@@ -6,7 +6,6 @@ import numpy as np
 import torch
 import paper_conf_asplos_miaoozcwzwzyssc24_b200 as spi
 from paper_conf_asplos_miaoozcwzwzyssc24_b200 import build_lib
-spi.load_library(build_lib.build(debug_hooks=True))  # traces exist only in the development build
 import workloads as W
 
 ap = argparse.ArgumentParser()
@@ -16,7 +15,9 @@ ap.add_argument("--prefix", type=int, default=None)
 ap.add_argument("--expansion", default=None, help="override the tree: comma list <k1,..,km>")
 ap.add_argument("--flags", type=int, default=0, help="debug flags (64: no split-KV clusters)")
 ap.add_argument("--all", action="store_true", help="print every traced tile of CTAs 0-1")
+ap.add_argument("--lib", default=None, help="a debug-hooks library built elsewhere (A/B experiments)")
 a = ap.parse_args()
+spi.load_library(a.lib or build_lib.build(debug_hooks=True))  # traces exist only in the development build
 os.environ["SPECINFER_DEBUG_FLAGS"] = str(a.flags)
 spi.specinfer_debug_set_trace(None)
 cfg = W.CONFIGS[a.config]
