@@ -440,6 +440,28 @@ def test_attention_rescales_across_segments(name, batch):
     assert np.all(e <= MAX_ABS * np.maximum(1.0, np.abs(ref_o[0, :n[0]]))) and e.mean() <= MEAN_ABS
 
 
+@pytest.mark.parametrize("case", ["five_pieces", "many_pieces"])
+def test_rows_kernel_split_merge_paths(case):
+    """Rows-as-M kernel (G * Nmax > 64) with stream-K split units, merged by the epilogue warpgroup:
+    'five_pieces' = 32 MHA units of 65 tiles over 148 CTAs (each unit cut into ~5 pieces: more than one
+    staging round of the idle rings); 'many_pieces' = one 40000-key request among short ones (its unit is
+    cut into ~100 pieces: the batched-load merge and the multi-round staged merge)."""
+    if case == "five_pieces":
+        tb = W.random_tree_batch(1, 128, 8192, seed=11, device=DEV)
+        Hq = Hkv = 32
+    else:
+        parent, depth = W.expansion_tree((2, 3, 4, 4))   # 129 nodes: two 128-row blocks (lock-step lanes)
+        B = 6
+        pls = [40000] + [5 + 97 * b for b in range(B - 1)]
+        tb = W.make_tree_batch([(parent, depth)] * B, pls, device=DEV, max_depth=8)
+        Hq = Hkv = 2
+    smax = int(tb.prefix_len.max()) + tb.max_nodes + 1
+    ai = W.make_attention_inputs(tb, 1, Hq, Hkv, smax, seed=21, device=DEV, poison=True)
+    out, _ = _gpu_attention(tb, ai, Hq, Hkv)
+    bs = [0] if tb.parent.shape[0] == 1 else [0, tb.parent.shape[0] - 1]
+    _check_rows(out, _oracle_attention(ai, tb, bs=bs), tb, bs=bs)
+
+
 @pytest.mark.parametrize("n,B,P", [(8, 64, 512), (32, 8, 2048), (128, 4, 8192), (256, 2, 2048), (64, 1, 512)])
 def test_config_c5_points(n, B, P):
     """C5 sweep points (random trees, depth <= 8), one layer, sampled requests vs the oracle."""
