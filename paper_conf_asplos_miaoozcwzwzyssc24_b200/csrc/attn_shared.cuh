@@ -26,6 +26,10 @@ struct AttnParams {
     int early_prefix;  // SPECINFER_ATTN_EARLY_PREFIX: the producers read the schedule and stage the
                        // first committed-prefix tiles before the programmatic dependency resolves
     int lanes;  // CTAs per lock-step group (schedule_kernel); 1 = plain stream-K over items
+    // rows kernel, many short items (dyn = 1): whole items claimed from an atomic ticket counter (reset by
+    // tree_prepare) instead of the static stream-K ranges -- CTA c starts with item c, then claims
+    uint32_t *dyn_ctr;
+    int dyn;
     // paged KV (NEXT-4): page_table[b][t] = page holding keys [128 t, 128 t + 128) of request b;
     // a page is [Hkv][128][128] bf16.  nullptr = contiguous [B][Hkv][Smax][128] caches.
     const int32_t *page_table;

@@ -31,6 +31,7 @@ struct WsLayout {
     size_t item_cnt;    // uint32[n_items]       split-combine counters
     size_t item_info;   // int4[n_items]         {first tile, end tile, P_b, n_b}
     size_t cta_info;    // int4[max_ctas][2]     {t0, t1, first item, total tiles}, item_info[first item]
+    size_t dyn_ctr;     // uint32                 rows kernel's dynamic item tickets (reset by tree_prepare)
     size_t part_o;      // float[max_ctas][2][NT][128]
     size_t part_ml;     // float[max_ctas][2][2][NT]
     size_t argmax;      // int32[B][Nmax]
@@ -97,6 +98,7 @@ inline WsLayout ws_layout(const specinfer_shape_t &s, int num_sms, bool allow_sp
     w.item_cnt = take(size_t(w.n_items) * 4);
     w.item_info = take(size_t(w.n_items + 1) * 16);  // + sentinel
     w.cta_info = take(size_t(w.max_ctas) * 32);
+    w.dyn_ctr = take(4);
     w.part_o = take(size_t(w.max_ctas) * 2 * w.nt * kHeadDim * 4);
     w.part_ml = take(size_t(w.max_ctas) * 2 * 2 * w.nt * 4);
     w.argmax = take(size_t(B) * N * 4);

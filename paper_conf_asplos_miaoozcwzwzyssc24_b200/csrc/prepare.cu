@@ -290,7 +290,8 @@ __global__ void __launch_bounds__(kPrepThreads) schedule_kernel(
     const int32_t *__restrict__ prefix_len, const int32_t *__restrict__ n_nodes, const int32_t *req_ok, int B,
     int Hkv, int chunks, int npc, int lanes, int32_t *__restrict__ item_start, uint32_t *__restrict__ item_cnt,
     int4 *__restrict__ item_info, int4 *__restrict__ cta_info, int num_ctas, int splitk,
-    uint32_t *__restrict__ verify_cnt, int32_t *__restrict__ status, int no_split_slack) {
+    uint32_t *__restrict__ verify_cnt, int32_t *__restrict__ status, int no_split_slack, uint32_t *dyn_ctr) {
+    if (threadIdx.x == 0) *dyn_ctr = 0u;   // the rows kernel's item tickets start over every step
     schedule(prefix_len, n_nodes, req_ok, B, Hkv, chunks, npc, lanes, item_start, item_cnt, item_info, cta_info,
              num_ctas, splitk, verify_cnt, status, no_split_slack);
 }
@@ -312,7 +313,8 @@ cudaError_t launch_tree_prepare(const specinfer_shape_t &s, const WsLayout &w,
         prefix_len, n_nodes, req_ok, s.batch, s.num_kv_heads, w.chunks, w.npc, w.lanes,
         reinterpret_cast<int32_t *>(ws + w.item_start), reinterpret_cast<uint32_t *>(ws + w.item_cnt),
         reinterpret_cast<int4 *>(ws + w.item_info), reinterpret_cast<int4 *>(ws + w.cta_info), num_ctas, w.splitk,
-        reinterpret_cast<uint32_t *>(ws + w.verify_cnt), status, w.nt == kRowsBlock ? 24 : 8);
+        reinterpret_cast<uint32_t *>(ws + w.verify_cnt), status, w.nt == kRowsBlock ? 24 : 8,
+        reinterpret_cast<uint32_t *>(ws + w.dyn_ctr));
     return cudaGetLastError();
 }
 

@@ -997,6 +997,10 @@ cudaError_t launch_tree_attention(const specinfer_shape_t &s, const WsLayout &w,
 #endif
     prm.splitk = w.splitk;
     const int grid = w.grid;  // persistent one CTA per SM, or n_items x splitk in split-KV mode
+    // rows kernel with at least 12 items per CTA: dynamic whole-item claims (per-CTA speed differs by
+    // ~10% across the SMs of a B200, which a static tile split cannot see; the tail is one short item)
+    prm.dyn_ctr = reinterpret_cast<uint32_t *>(ws + w.dyn_ctr);
+    prm.dyn = (w.nt == kRowsBlock && w.n_items >= 12 * grid) ? 1 : 0;
     switch (w.nt) {
         case 16: return launch_nt<16>(prm, q, k, v, grid, max_smem, stream);
         case 32: return launch_nt<32>(prm, q, k, v, grid, max_smem, stream);

@@ -266,7 +266,7 @@ __global__ void __launch_bounds__(rows::kThreads, 1)
     const int4 ci = __ldg(p.cta_info + 2 * blockIdx.x);
     const int4 first_info = __ldg(p.cta_info + 2 * blockIdx.x + 1);
     const int t0 = ci.x, t1 = ci.y, x_first = ci.z, T = ci.w;
-    const int ntiles = t1 - t0;
+    const int ntiles = p.dyn ? 1 : t1 - t0;   // (dynamic mode: every CTA starts with item blockIdx.x)
 
     if (warp >= 12) {
         // epilogue warpgroup (warp & 3 = TMEM lane quarter): its registers go to the softmax warps
@@ -511,7 +511,7 @@ __global__ void __launch_bounds__(rows::kThreads, 1)
         } else if (warp == kWarpProd || warp == kWarpV) {
             // ============================ TMA producers ============================
             // warp 8: segment descriptors, Q and the K ring; warp 11: the V ring (follows the descriptors)
-            const uint64_t pol = p.lanes > 1 ? l2_evict_normal_policy() : l2_evict_first_policy();
+            const uint64_t pol = (p.lanes > 1 || (p.dyn && p.chunks > 1)) ? l2_evict_normal_policy() : l2_evict_first_policy();
             auto issue = [&](const SegDesc &d, int t, int lt, bool is_v) {
                 const int key0 = (t - d.ib) * kKeyTile;
                 const int nv = min(kKeyTile, d.P + d.n - key0);
@@ -545,7 +545,68 @@ __global__ void __launch_bounds__(rows::kThreads, 1)
                 while (c < NS && d.begin + c < d.end && (d.begin + c - d.ib + 1) * kKeyTile <= d.P) ++c;
                 return c;
             };
-            if (warp == kWarpProd && lane == 0) {
+            if (warp == kWarpProd && lane == 0 && p.dyn) {
+                // dynamic mode: whole items; the first is item blockIdx.x, the next ones are claimed from the
+                // ticket counter (after the dependency wait), each one while the current item streams.  Every
+                // launch draws exactly n_items tickets (n_items - grid claims + one failing claim per CTA) and
+                // launches draw in turn, so ticket t names item grid + t mod n_items (>= n_items: none left).
+                bool waited = !early;
+                auto claim = [&]() -> int {
+                    if (!waited) {
+                        grid_dependency_wait();
+                        waited = true;
+                    }
+                    const uint32_t t = atomicAdd(p.dyn_ctr, 1u);
+                    const int idx = (int)(t % (uint32_t)p.n_items) + (int)gridDim.x;
+                    return idx < p.n_items ? idx : -1;
+                };
+                int dx = (int)blockIdx.x < p.n_items ? (int)blockIdx.x : -1;
+                int ls = 0, lt = 0;
+                for (;;) {
+                    SegDesc d{};
+                    d.x = -1;
+                    while (dx >= 0) {
+                        const int4 info = __ldg(p.item_info + dx);
+                        if (info.y > info.x && info.w > 0) {
+                            d.x = dx;
+                            d.begin = d.ib = info.x;
+                            d.end = d.ie = info.y;
+                            d.c = dx % p.chunks;
+                            d.g = (dx / p.chunks) % p.Hkv;
+                            d.b = dx / (p.chunks * p.Hkv);
+                            d.P = info.z;
+                            d.n = info.w;
+                            break;
+                        }
+                        dx = claim();   // an empty item (invalid tree / padding chunk)
+                    }
+                    misc->seg[ls % kSegRing] = d;
+                    mbar_arrive(&misc->seg_full[ls % kSegRing]);
+                    if (d.x < 0) {
+                        if (!waited) grid_dependency_wait();
+                        break;
+                    }
+                    int pre = 0;
+                    if (!waited) {   // (early mode, first item: committed-prefix tiles before the wait)
+                        pre = n_early(d, NK);
+                        for (int i = 0; i < pre; ++i) issue(d, d.begin + i, i, false);
+                        grid_dependency_wait();
+                        waited = true;
+                    }
+                    dx = claim();   // the next item (the atomic's latency overlaps this item's loads)
+                    const int qb = ls & 1;
+                    if (ls >= 2) mbar_wait(&misc->q_empty[qb], ((ls >> 1) - 1) & 1);
+                    mbar_arrive_expect_tx(&misc->q_full[qb], 2u * (uint32_t)(p.G * p.npc) * 128u);
+                    uint8_t *qdst = s_q + qb * kQBuf;
+                    const int node0 = d.b * p.Nmax + d.c * p.npc;
+                    tma_load_3d(qdst, &tm_q, &misc->q_full[qb], 0, d.g * p.G, node0);
+                    tma_load_3d(qdst + RB * 128, &tm_q, &misc->q_full[qb], 64, d.g * p.G, node0);
+                    lt += pre;
+                    for (int t = d.begin + pre; t < d.end; ++t, ++lt) issue(d, t, lt, false);
+                    ++ls;
+                }
+                grid_launch_dependents();
+            } else if (warp == kWarpProd && lane == 0) {
                 int x = x_first, ls = 0, lt = 0;
                 int4 next_info = first_info;
                 for (;;) {
