@@ -997,10 +997,12 @@ cudaError_t launch_tree_attention(const specinfer_shape_t &s, const WsLayout &w,
 #endif
     prm.splitk = w.splitk;
     const int grid = w.grid;  // persistent one CTA per SM, or n_items x splitk in split-KV mode
-    // rows kernel with at least 12 items per CTA: dynamic whole-item claims (per-CTA speed differs by
-    // ~10% across the SMs of a B200, which a static tile split cannot see; the tail is one short item)
+    // rows kernel with at least one item per CTA: dynamic whole-item claims instead of the static stream-K
+    // split (measured faster at every C3 / C4 batch from 1.7 items per CTA up: per-CTA speed differs by ~10%
+    // across a B200's SMs, which a static split cannot see, and whole items need no lock-step lanes or
+    // split merges); fewer items than CTAs keep the stream-K split (long items over many CTAs)
     prm.dyn_ctr = reinterpret_cast<uint32_t *>(ws + w.dyn_ctr);
-    prm.dyn = (w.nt == kRowsBlock && w.n_items >= 12 * grid) ? 1 : 0;
+    prm.dyn = (w.nt == kRowsBlock && w.n_items >= grid) ? 1 : 0;
     switch (w.nt) {
         case 16: return launch_nt<16>(prm, q, k, v, grid, max_smem, stream);
         case 32: return launch_nt<32>(prm, q, k, v, grid, max_smem, stream);
