@@ -174,7 +174,7 @@ __global__ void __launch_bounds__(SwRoles<NT>::kThreads, 1)
     const int4 ci = __ldg(p.cta_info + 2 * blockIdx.x);
     const int4 first_info = __ldg(p.cta_info + 2 * blockIdx.x + 1);
     const int t0 = ci.x, t1 = ci.y, x_first = ci.z, T = ci.w;
-    const int ntiles = t1 - t0;
+    const int ntiles = p.dyn ? 1 : t1 - t0;   // (dynamic mode: every CTA starts with item blockIdx.x)
     if (threadIdx.x == 0 && ntiles > -1000000) SPI_TRACE_K(6);
 
     if (ntiles <= 0) {
@@ -218,7 +218,67 @@ __global__ void __launch_bounds__(SwRoles<NT>::kThreads, 1)
             while (c < NS && d.begin + c < d.end && (d.begin + c - d.ib + 1) * kKeyTile <= d.P) ++c;
             return c;
         };
-        if (warp == 0 && lane == 0) {
+        if (warp == 0 && lane == 0 && p.dyn) {
+            // dynamic mode (see tree_attention_rows.cu): whole items, the first one is item blockIdx.x, the
+            // next ones are claimed from the ticket counter after the dependency wait, each while the
+            // current item streams; ticket t names item grid + t mod n_items (>= n_items: none left)
+            bool waited = !early;
+            auto claim = [&]() -> int {
+                if (!waited) {
+                    grid_dependency_wait();
+                    waited = true;
+                }
+                const uint32_t t = atomicAdd(p.dyn_ctr, 1u);
+                const int idx = (int)(t % (uint32_t)p.n_items) + (int)gridDim.x;
+                return idx < p.n_items ? idx : -1;
+            };
+            int dx = (int)blockIdx.x < p.n_items ? (int)blockIdx.x : -1;
+            int lt = 0, ls = 0;
+            for (;;) {
+                SegDesc d{};
+                d.x = -1;
+                while (dx >= 0) {
+                    const int4 info = __ldg(p.item_info + dx);
+                    if (info.y > info.x) {
+                        d.x = dx;
+                        d.begin = d.ib = info.x;
+                        d.end = d.ie = info.y;
+                        d.c = dx % p.chunks;
+                        d.g = (dx / p.chunks) % p.Hkv;
+                        d.b = dx / (p.chunks * p.Hkv);
+                        d.P = info.z;
+                        d.n = info.w;
+                        break;
+                    }
+                    dx = claim();   // an empty item
+                }
+                misc->seg[ls % kSegRing] = d;
+                mbar_arrive(&misc->seg_full[ls % kSegRing]);
+                if (d.x < 0) {
+                    if (!waited) grid_dependency_wait();
+                    break;
+                }
+                int pre = 0;
+                if (!waited) {   // (early mode, first item: committed-prefix tiles before the wait)
+                    pre = n_early(d, NK);
+                    for (int i = 0; i < pre; ++i) issue(d, d.begin + i, i, false);
+                    grid_dependency_wait();
+                    waited = true;
+                }
+                dx = claim();   // the next item (the atomic's latency overlaps this item's loads)
+                const int qb = ls % Plan::kNQ;
+                if (ls >= Plan::kNQ) mbar_wait(&misc->q_empty[qb], ((ls / Plan::kNQ) - 1) & 1);
+                mbar_arrive_expect_tx(&misc->q_full[qb], 2u * (uint32_t)(p.G * p.npc) * 128u);
+                uint8_t *qdst = s_q + qb * Plan::kQBuf;
+                const int node0 = d.b * p.Nmax + d.c * p.npc;
+                tma_load_3d(qdst, &tm_q, &misc->q_full[qb], 0, d.g * p.G, node0);
+                tma_load_3d(qdst + NT * 128, &tm_q, &misc->q_full[qb], 64, d.g * p.G, node0);
+                lt += pre;
+                for (int t = d.begin + pre; t < d.end; ++t, ++lt) issue(d, t, lt, false);
+                ++ls;
+            }
+            grid_launch_dependents();
+        } else if (warp == 0 && lane == 0) {
             // segment descriptors for every role, Q, and the K tiles
             int lt = 0, ls = 0;
             int4 next_info = first_info;
@@ -260,13 +320,23 @@ __global__ void __launch_bounds__(SwRoles<NT>::kThreads, 1)
                 for (int t = d.begin + pre; t < d.end; ++t, ++lt) issue(d, t, lt, false);
                 ++ls;
             }
+            {   // terminal descriptor: the consumers stop here
+                SegDesc d{};
+                d.x = -1;
+                misc->seg[ls % kSegRing] = d;
+                mbar_arrive(&misc->seg_full[ls % kSegRing]);
+            }
             grid_launch_dependents();  // all of this CTA's K loads are issued
         } else if (warp == kWarpV && lane == 0) {
             // V tiles, following the segment ring written by warp 0
             int lt = 0, ls = 0;
-            while (lt < ntiles) {
+            for (;;) {
                 mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
                 const SegDesc d = misc->seg[ls % kSegRing];
+                if (d.x < 0) {   // terminal descriptor
+                    if (early && ls == 0) grid_dependency_wait();
+                    break;
+                }
                 int pre = 0;
                 if (early && ls == 0) {
                     pre = n_early(d, NV);
@@ -285,9 +355,10 @@ __global__ void __launch_bounds__(SwRoles<NT>::kThreads, 1)
             const uint32_t idesc_s = make_idesc_bf16(128, NT, false, false);
             const uint32_t k_addr = smem_u32(s_k), q_addr = smem_u32(s_q);
             int lt = 0, ls = 0;
-            while (lt < ntiles) {
+            for (;;) {
                 mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
                 const SegDesc d = misc->seg[ls % kSegRing];
+                if (d.x < 0) break;   // terminal descriptor
                 const int qb = ls % Plan::kNQ;
                 mbar_wait(&misc->q_full[qb], (ls / Plan::kNQ) & 1);
                 for (int t = d.begin; t < d.end; ++t, ++lt) {
@@ -320,9 +391,10 @@ __global__ void __launch_bounds__(SwRoles<NT>::kThreads, 1)
             const uint32_t idesc_o = make_idesc_bf16(128, NT, true, true);
             const uint32_t v_addr = smem_u32(s_v), p_addr = smem_u32(s_p);
             int lt = 0, ls = 0;
-            while (lt < ntiles) {
+            for (;;) {
                 mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
                 const SegDesc d = misc->seg[ls % kSegRing];
+                if (d.x < 0) break;   // terminal descriptor
                 for (int t = d.begin; t < d.end; ++t, ++lt) {
                     mbar_wait(&misc->p_full[lt % Plan::kNP], (lt / Plan::kNP) & 1);
                     const int slot = lt % NV;
@@ -354,9 +426,10 @@ __global__ void __launch_bounds__(SwRoles<NT>::kThreads, 1)
         const int d = kt;
         const uint32_t lane_off = (uint32_t)(qd * 32) << 16;
         int lt = 0, ls = 0;
-        while (lt < ntiles) {
+        for (;;) {
             mbar_wait(&misc->seg_full[ls % kSegRing], (ls / kSegRing) & 1);
             const SegDesc sd = misc->seg[ls % kSegRing];
+            if (sd.x < 0) break;   // terminal descriptor
             const int b = sd.b, g = sd.g, c = sd.c, P = sd.P, n = sd.n;
             const int Kend = P + n;
             const int node0 = c * p.npc;
@@ -997,12 +1070,14 @@ cudaError_t launch_tree_attention(const specinfer_shape_t &s, const WsLayout &w,
 #endif
     prm.splitk = w.splitk;
     const int grid = w.grid;  // persistent one CTA per SM, or n_items x splitk in split-KV mode
-    // rows kernel with at least one item per CTA: dynamic whole-item claims instead of the static stream-K
-    // split (measured faster at every C3 / C4 batch from 1.7 items per CTA up: per-CTA speed differs by ~10%
-    // across a B200's SMs, which a static split cannot see, and whole items need no lock-step lanes or
-    // split merges); fewer items than CTAs keep the stream-K split (long items over many CTAs)
+    // at least one item per CTA (and no split-KV clusters): dynamic whole-item claims instead of the static
+    // stream-K split.  Per-CTA speed differs by ~10% across a B200's SMs, which a static split cannot see,
+    // and whole items need no lock-step lanes or split merges: measured faster at every C3 / C4 batch from
+    // 1.7 items per CTA up (bench A/B: C3 345 -> 314 us, C4 885 -> 787 us per launch) and for the swapped
+    // kernel at C2 batch 16 (89.2 -> 87.3 us per layer; batch 8 unchanged).  Fewer items than CTAs keep
+    // the stream-K split (long items spread over many CTAs).
     prm.dyn_ctr = reinterpret_cast<uint32_t *>(ws + w.dyn_ctr);
-    prm.dyn = (w.nt == kRowsBlock && w.n_items >= grid) ? 1 : 0;
+    prm.dyn = (w.splitk == 1 && w.n_items >= grid) ? 1 : 0;
     switch (w.nt) {
         case 16: return launch_nt<16>(prm, q, k, v, grid, max_smem, stream);
         case 32: return launch_nt<32>(prm, q, k, v, grid, max_smem, stream);
