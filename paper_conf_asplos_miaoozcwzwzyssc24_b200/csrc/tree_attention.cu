@@ -1070,14 +1070,17 @@ cudaError_t launch_tree_attention(const specinfer_shape_t &s, const WsLayout &w,
 #endif
     prm.splitk = w.splitk;
     const int grid = w.grid;  // persistent one CTA per SM, or n_items x splitk in split-KV mode
-    // at least one item per CTA (and no split-KV clusters): dynamic whole-item claims instead of the static
+    // enough items per CTA (and no split-KV clusters): dynamic whole-item claims instead of the static
     // stream-K split.  Per-CTA speed differs by ~10% across a B200's SMs, which a static split cannot see,
     // and whole items need no lock-step lanes or split merges: measured faster at every C3 / C4 batch from
     // 1.7 items per CTA up (bench A/B: C3 345 -> 314 us, C4 885 -> 787 us per launch) and for the swapped
     // kernel at C2 batch 16 (89.2 -> 87.3 us per layer; batch 8 unchanged).  Fewer items than CTAs keep
     // the stream-K split (long items spread over many CTAs).
     prm.dyn_ctr = reinterpret_cast<uint32_t *>(ws + w.dyn_ctr);
-    prm.dyn = (w.splitk == 1 && w.n_items >= grid) ? 1 : 0;
+    // (the rows kernel's static path -- lock-step lanes, split merges -- costs more: it switches to whole
+    // items from half an item per CTA up, C3 batch 4 48.3 -> 43.6 us; the swapped kernel keeps stream-K
+    // below one item per CTA, C2 batch 4 24.3 vs 24.7 us)
+    prm.dyn = (w.splitk == 1 && (w.nt == kRowsBlock ? 2 * w.n_items >= grid : w.n_items >= grid)) ? 1 : 0;
     switch (w.nt) {
         case 16: return launch_nt<16>(prm, q, k, v, grid, max_smem, stream);
         case 32: return launch_nt<32>(prm, q, k, v, grid, max_smem, stream);
