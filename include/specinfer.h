@@ -108,7 +108,11 @@ specinfer_status_t specinfer_tree_prepare(const specinfer_shape_t *shape, const 
  * Cache slots >= P_b + n_b are never used (may hold anything, NaN included).
  * parent/depth are accepted for the record of the call (the mask comes from `workspace`,
  * which tree_prepare built from the same arrays).  Rows i >= n_b, and all rows of an invalid
- * request, are left untouched.  k_cache/v_cache must be 16-byte aligned. */
+ * request, are left untouched.  k_cache/v_cache must be 16-byte aligned.
+ * Work distribution: with enough (request, kv-head, row-block) items per SM the CTAs claim whole
+ * items from a ticket counter in `workspace` (reset by tree_prepare; each call draws exactly one
+ * ticket per item), so calls on one workspace must not overlap in time (one stream, as above) and
+ * at most 2^32 / items calls may follow one tree_prepare.  Results do not depend on the order. */
 specinfer_status_t specinfer_tree_attention(const specinfer_shape_t *shape, const void *q,
                                             const void *k_cache, const void *v_cache,
                                             const int32_t *parent, const int32_t *depth,
