@@ -211,6 +211,31 @@ def test_attention_invalid_tree_status():
     _check_rows(out, ref, tb, bs=[0])
 
 
+@pytest.mark.parametrize("Hq,Hkv,expansion,B", [(32, 32, (1, 1, 3, 1, 1, 1, 1, 1), 24),   # swapped, 768 items
+                                                 (64, 8, (1, 2, 2, 2, 2, 2), 8)])            # rows, 256 items
+def test_dynamic_schedule_with_invalid_requests(Hq, Hkv, expansion, B):
+    """Enough items per CTA for the dynamic whole-item schedule (ticket counter), with two invalid
+    trees among the requests: their items are empty (skipped by the claims), their rows stay
+    untouched, every other request matches the oracle; a second call on the same workspace (the
+    next layer: tickets continue from the first call's) gives bit-identical rows."""
+    parent, depth = W.expansion_tree(expansion)
+    pls = [300 + 37 * b for b in range(B)]
+    tb = W.make_tree_batch([(parent, depth)] * B, pls, device=DEV, max_depth=8)
+    tb.parent[3, 2] = 7    # parent not < i
+    tb.parent[B - 2, 1] = 1
+    ai = W.make_attention_inputs(tb, 2, Hq, Hkv, max(pls) + tb.max_nodes + 1, seed=8, device=DEV)
+    out, st = _gpu_attention(tb, ai, Hq, Hkv)
+    assert spi.specinfer_read_device_status(st.workspace) & 1
+    for bad in (3, B - 2):
+        assert torch.isnan(out[bad].float()).all()
+    again = torch.full_like(out, float("nan"))
+    st.attention(ai.q[0], ai.k_cache[0], ai.v_cache[0], again)
+    torch.cuda.synchronize()
+    assert torch.equal(torch.nan_to_num(again, nan=7.0), torch.nan_to_num(out, nan=7.0))
+    bs = [0, 1, B - 1]
+    _check_rows(out, _oracle_attention(ai, tb, bs=bs), tb, bs=bs)
+
+
 @pytest.mark.parametrize("name,batch", [("C2", 3), ("C3", 2), ("C1", 1)])
 def test_prepare_initialises_a_garbage_workspace(name, batch):
     """tree_prepare needs no zeroed workspace (no memset since round 2): with every byte of the workspace
