@@ -23,8 +23,12 @@
 //  * warpgroups: 0-1 softmax, 2 control (producers, issuers), 3 epilogue; setmaxnreg moves registers
 //    from the control and epilogue warpgroups (56 per thread) to the softmax warpgroups (200: the
 //    scores stay in registers);
-//  * lane mode (schedule_kernel): the row blocks of one (request, kv-head) run on `lanes` CTAs in
-//    lock-step over the same tile range, so each KV tile is read from HBM once;
+//  * schedule: with at least half an item per CTA, whole items claimed dynamically (item blockIdx.x
+//    first, then tickets from an atomic counter reset by tree_prepare): the row blocks of one (request,
+//    kv-head) are consecutive tickets, so they stream the same KV tiles at about the same time and the
+//    second reads them from L2 (ncu: DRAM bytes = the algorithmic bytes).  Fewer items: the static
+//    stream-K split in lane mode -- the row blocks of a (request, kv-head) on `lanes` CTAs in lock-step
+//    over the same tile range;
 //  * tree keys are masked with the ancestor-or-self bitset of the row's node (tree_prepare);
 //  * the stream-K schedule, segment descriptors, row-exact tail loads, split combine and PDL are
 //    shared with the swapped kernel (attn_shared.cuh).
