@@ -236,6 +236,21 @@ def test_dynamic_schedule_with_invalid_requests(Hq, Hkv, expansion, B):
     _check_rows(out, _oracle_attention(ai, tb, bs=bs), tb, bs=bs)
 
 
+def test_rows_kernel_dynamic_ragged_chunks():
+    """Rows kernel in the dynamic whole-item mode with two 128-row chunks per (request, kv-head) and
+    ragged trees: requests with 15 nodes leave their second chunk empty (skipped by the claims), requests
+    with 129 nodes fill both; sampled requests of both kinds match the oracle."""
+    big, small = W.expansion_tree((2, 3, 4, 4)), W.expansion_tree((2, 2, 2))
+    B = 48
+    trees = [big if b % 2 == 0 else small for b in range(B)]
+    pls = [200 + 13 * b for b in range(B)]
+    tb = W.make_tree_batch(trees, pls, device=DEV, max_depth=8)
+    ai = W.make_attention_inputs(tb, 1, 4, 4, max(pls) + tb.max_nodes + 1, seed=12, device=DEV, poison=True)
+    out, _ = _gpu_attention(tb, ai, 4, 4)
+    bs = [0, 1, B - 2, B - 1]
+    _check_rows(out, _oracle_attention(ai, tb, bs=bs), tb, bs=bs)
+
+
 @pytest.mark.parametrize("name,batch", [("C2", 3), ("C3", 2), ("C1", 1)])
 def test_prepare_initialises_a_garbage_workspace(name, batch):
     """tree_prepare needs no zeroed workspace (no memset since round 2): with every byte of the workspace
