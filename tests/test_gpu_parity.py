@@ -236,6 +236,24 @@ def test_dynamic_schedule_with_invalid_requests(Hq, Hkv, expansion, B):
     _check_rows(out, _oracle_attention(ai, tb, bs=bs), tb, bs=bs)
 
 
+@pytest.mark.parametrize("Br,Bs", [(2, 18), (3, 19)])
+def test_schedule_mode_boundaries(Br, Bs):
+    """Either side of the schedule switches (148-SM grid): the rows kernel claims whole items from
+    n_items >= 74 (half an item per CTA; Br x 8 kv-heads x 4 chunks = 64 / 96 items), the swapped kernel
+    from n_items >= 148 (Bs x 8 kv-heads = 144 / 152 items); sampled requests vs the oracle."""
+    parent, depth = W.expansion_tree((1, 2, 2, 2, 2, 2))        # 63 nodes: rows kernel at G = 8 (4 chunks)
+    tb = W.make_tree_batch([(parent, depth)] * Br, [150 + 11 * b for b in range(Br)], device=DEV, max_depth=8)
+    ai = W.make_attention_inputs(tb, 1, 64, 8, 150 + 11 * Br + tb.max_nodes, seed=Br, device=DEV, poison=True)
+    out, _ = _gpu_attention(tb, ai, 64, 8)
+    _check_rows(out, _oracle_attention(ai, tb), tb)
+    parent, depth = W.expansion_tree((1, 1, 3, 1, 1, 1, 1, 1))  # 21 nodes: swapped kernel, 1 chunk
+    tb = W.make_tree_batch([(parent, depth)] * Bs, [300 + 7 * b for b in range(Bs)], device=DEV, max_depth=8)
+    ai = W.make_attention_inputs(tb, 1, 8, 8, 300 + 7 * Bs + tb.max_nodes, seed=Bs, device=DEV, poison=True)
+    out, _ = _gpu_attention(tb, ai, 8, 8)
+    bs = [0, Bs // 2, Bs - 1]
+    _check_rows(out, _oracle_attention(ai, tb, bs=bs), tb, bs=bs)
+
+
 def test_rows_kernel_dynamic_ragged_chunks():
     """Rows kernel in the dynamic whole-item mode with two 128-row chunks per (request, kv-head) and
     ragged trees: requests with 15 nodes leave their second chunk empty (skipped by the claims), requests
